@@ -1,0 +1,325 @@
+#!/usr/bin/env python
+"""Benchmark of the SPH time step (libsph) -- the driver's contract.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload turbulence200]
+    python bench.py --impl reference ...      # the CPU oracle arm
+
+A *step* is one full pass of the hot path (sph_step: keys, sort, cells,
+neighbours, density, EOS, IAD, momentum-energy, dt, update) over the particle
+state, which stays resident in HBM.  Metric (BASELINE.json): particle-updates/s
+per SPH step.  Default workload: subsonic turbulence 200^3 (8M particles per
+GPU; BASELINE.json configs[2], the north star's headline target).  Inputs are
+~1 GB of particle state plus ~3 GB of neighbour lists per GPU, far larger than
+the 126 MB L2, so no flush is needed between steps.
+
+The JSON line carries: value (device-timed, CUDA events on libsph's stream,
+max over ranks), e2e (the same metric through the C ABI with the state copied
+from pinned host buffers in and back out every step), roofline (dominant
+kernel: momentum-energy, FP64 pipe), energy (per-phase J/step from NVML in a
+separate accounted pass), cpu_baseline (the oracle on a bounded sample),
+clocks (nvidia-smi sampled during the timed region) and gpu_launches.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "particle-updates/s per SPH step"
+UNIT = "particle-updates/s"
+
+# Algorithmic FP64 flops per neighbour pair, counting
+# add/sub/mul as 1 and fma as 2, sinc as its 13-FMA polynomial; the artificial
+# viscosity's 17 flops (approaching pairs only) are NOT counted (lower bound).
+FLOPS_PER_PAIR = {"density": 40, "iad": 55, "momentum_energy": 157}
+# FP64 peak: 148 SMs x 64 FP64 FMA/clk x 2 flop x 1.965 GHz (guide's SM count and
+# max SM clock; DFMA microbenchmark measured 34.1 TF, tools/probe_fp64.cu).
+FP64_PEAK_TFLOPS = 148 * 64 * 2 * 1.965e9 / 1e12
+# Algorithmic HBM bytes per particle of the momentum-energy launch (i-side fields
+# once, neighbour list once, outputs once): 19 doubles + nc + 4 B per neighbour + 4 doubles.
+MOM_BYTES_PER_PARTICLE = 19 * 8 + 4 + 4 * 8   # + 4 * nc
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--workload", default="turbulence200")
+    ap.add_argument("--impl", default="libsph", choices=["libsph", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--energy-steps", type=int, default=5)
+    ap.add_argument("--cpu-sample", type=int, default=0, help="oracle targets (0 = auto)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--out", default=None)
+    return ap.parse_args()
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def make_workload(name: str, rank: int):
+    from paper_conf_sc_simsekpc24_b200 import ics
+    if name.startswith("turbulence"):
+        return ics.turbulence(int(name[len("turbulence"):]))
+    if name.startswith("sedov"):
+        return ics.sedov(int(name[len("sedov"):]))
+    if name.startswith("noh"):
+        return ics.noh(int(name[len("noh"):]))
+    raise SystemExit(f"unknown workload {name}")
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled every 100 ms during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            self.p = None
+        time.sleep(0.3)
+        return self
+
+    def __exit__(self, *a):
+        self.lines = []
+        if self.p:
+            time.sleep(0.25)
+            self.p.terminate()
+            out, _ = self.p.communicate(timeout=10)
+            self.lines = [l for l in out.splitlines() if l.strip()]
+
+    def summary(self):
+        sm, mx, pw = [], [], []
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for l in getattr(self, "lines", []):
+            f = [x.strip() for x in l.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx.append(float(f[1]))
+                pw.append(float(f[2]))
+            except ValueError:
+                continue
+            for k, v in zip(names, f[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(k)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx), "reasons": sorted(reasons),
+                "power_w_median": statistics.median(pw), "samples": len(sm)}
+
+
+def cpu_baseline(w, n_targets: int, seed: int = 3):
+    """The oracle as it stands on a bounded sample: one step at n_targets random
+    particles of the same workload (sampled mode: exact global sort/dt, each
+    target's dependency ball brute-forced).  Returns (targets/s, seconds, threads)."""
+    import numpy as np
+    import oracle
+    rng = np.random.default_rng(seed)
+    tg = np.sort(rng.choice(w.n, size=n_targets, replace=False))
+    t0 = time.perf_counter()
+    oracle.sample_step({k: v for k, v in w.state.items()}, w.params, w.params.dt_first, True, tg)
+    dt = time.perf_counter() - t0
+    threads = int(os.environ.get("OMP_NUM_THREADS", os.cpu_count() or 1))
+    return n_targets / dt, dt, threads
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle timed on this host's cores (rank 0 only)."""
+    if rank != 0:
+        return
+    w = make_workload(args.workload, rank)
+    k = args.cpu_sample or 48
+    vals = []
+    for s in range(args.warmup + args.steps):
+        v, sec, threads = cpu_baseline(w, k, seed=100 + s)
+        if s >= args.warmup:
+            vals.append((v, sec))
+    tot_t = sum(s for _, s in vals)
+    value = k * len(vals) / tot_t
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 0, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1e3 * tot_t / len(vals), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "impl": "reference",
+            "config": {"workload": args.workload, "n_particles": w.n, "parallelism": "cpu-openmp"},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
+                             "sample": f"{k} random targets per step of {args.workload} (oracle sampled mode)"},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    rank, world, local = dist_env()
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_simsekpc24_b200 import sph
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", init_method="env://")
+    w = make_workload(args.workload, rank)
+    n = w.n
+    sim = sph.Simulation(w.params, n_capacity=n, device=local)
+    stream = sim.stream
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    host_state = {k: np.ascontiguousarray(v) for k, v in w.state.items()}
+    sim.set_particles(host_state)
+    sim.set_time(0.0, w.params.dt_first, True)
+
+    infos = []
+    for _ in range(args.warmup):
+        sim.step()
+    barrier()
+    launches0 = sph.kernel_launches()
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    mom_ms = []
+    with ClockSampler(local) as clk:
+        barrier()
+        ev0.record(stream)
+        for _ in range(args.steps):
+            info = sim.step()
+            infos.append(info)
+            mom_ms.append(info["phase_ms"]["momentum_energy"])
+        ev1.record(stream)
+        barrier()
+    launches = sph.kernel_launches() - launches0
+    ms = ev0.elapsed_time(ev1)
+    ms_t = torch.tensor([ms], device="cuda")
+    if world > 1:
+        dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
+    ms_max = float(ms_t.item())
+    value = n * world * args.steps / (ms_max * 1e-3)
+    phase_ms = {p: statistics.mean(i["phase_ms"][p] for i in infos) for p in sph.PHASES}
+    mean_nc = statistics.mean(i["mean_nc"] for i in infos)
+
+    # --- roofline of the dominant kernel (momentum-energy; FP64 pipe) ---
+    pairs = mean_nc * n
+    mom_s = statistics.mean(mom_ms) * 1e-3
+    achieved = FLOPS_PER_PAIR["momentum_energy"] * pairs / mom_s / 1e12
+    roofline = {"bound": "alu", "achieved": achieved, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
+                "frac": achieved / FP64_PEAK_TFLOPS, "traffic": None, "kernel": "momentum_energy_kernel",
+                "peak_source": "148 SM x 64 DFMA/clk x 2 x 1.965 GHz (FP64 pipe; DESIGN.md 6)",
+                "hbm_GBps_algorithmic": (MOM_BYTES_PER_PARTICLE + 4 * mean_nc) * n / mom_s / 1e9,
+                "share_of_step": statistics.mean(mom_ms) / (ms_max / args.steps)}
+    other = {}
+    for p in ("density", "iad"):
+        t = phase_ms[p] * 1e-3
+        other[p] = {"tflops": FLOPS_PER_PAIR[p] * pairs / t / 1e12,
+                    "frac_fp64": FLOPS_PER_PAIR[p] * pairs / t / 1e12 / FP64_PEAK_TFLOPS}
+
+    # --- e2e: same metric through the C ABI with host buffers ---
+    e2e = None
+    if args.e2e_steps > 0:
+        pinned = {k: torch.from_numpy(v).pin_memory() for k, v in sim.get_state().items()}
+        outbuf = {k: torch.empty_like(v).pin_memory() for k, v in pinned.items()}
+        t_now, dtp, _ = sim.get_time()
+        h2d = sum(v.numel() * v.element_size() for v in pinned.values())
+        d2h = sum(v.numel() * v.element_size() for v in outbuf.values())
+        barrier()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.e2e_steps):
+            sim.set_particles(pinned)
+            sim.step()
+            for k, v in outbuf.items():
+                sim.get_field(k, out=v)
+        e1.record(stream)
+        barrier()
+        e_ms = torch.tensor([e0.elapsed_time(e1)], device="cuda")
+        if world > 1:
+            dist.all_reduce(e_ms, op=dist.ReduceOp.MAX)
+        e2e = {"value": n * world * args.e2e_steps / (float(e_ms.item()) * 1e-3), "unit": UNIT,
+               "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+               "path": "sph_set_particles(pinned host) + sph_step + sph_get_field x11 (host)"}
+
+    # --- per-phase energy (NVML counter deltas at synchronised phase edges) ---
+    energy = None
+    if args.energy_steps > 0:
+        sim.energy_reset()
+        sim.set_accounting(sph.ACCOUNTING_PHASE)
+        e_start = sim.energy_counter_mj()
+        t0 = time.perf_counter()
+        for _ in range(args.energy_steps):
+            sim.step()
+        wall = time.perf_counter() - t0
+        e_end = sim.energy_counter_mj()
+        rows = sim.energy_report()
+        sim.set_accounting(sph.ACCOUNTING_OFF)
+        k = args.energy_steps
+        energy = {"mode": "phase (stream sync + NVML total-energy counter at every phase edge)",
+                  "steps": k, "clock_policy": "default (DVFS); clock locking not permitted on this host",
+                  "J_per_step": {r["name"]: (r["joules"] / k if r["joules"] is not None else None) for r in rows},
+                  "ms_per_step": {r["name"]: 1e3 * r["seconds"] / k for r in rows},
+                  "mean_sm_mhz": {r["name"]: r["mean_sm_mhz"] for r in rows},
+                  "step_J": ((e_end - e_start) * 1e-3 / k) if (e_start is not None and e_end is not None) else None,
+                  "step_ms_accounted": 1e3 * wall / k}
+        if energy["step_J"] is not None:
+            energy["uJ_per_particle_update"] = energy["step_J"] / n * 1e6
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        k = args.cpu_sample or 48
+        v, sec, threads = cpu_baseline(w, k)
+        cpu = {"value": v, "unit": UNIT, "cores": threads, "kind": "oracle",
+               "sample": f"{k} random targets of {args.workload}, one step (oracle sampled mode), {sec:.1f} s"}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "config": {"workload": args.workload, "n_particles_per_gpu": n,
+                           "n_particles_total": n * world,
+                           "parallelism": "single GPU" if world == 1 else
+                           f"{world} independent replicas (SFC decomposition not yet built)",
+                           "l2": "inputs (~1 GB state + ~3 GB lists) >> 126 MB L2; no flush",
+                           "mean_nc": mean_nc},
+                "phase_ms": phase_ms, "fp64_other": other, "roofline": roofline, "e2e": e2e,
+                "energy": energy, "cpu_baseline": cpu, "clocks": clk.summary(),
+                "gpu_launches": launches}
+        s = json.dumps(line)
+        print(s, flush=True)
+        if args.out:
+            with open(args.out, "w") as f:
+                f.write(s + "\n")
+    sim.finalize()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

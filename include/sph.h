@@ -1,0 +1,294 @@
+/*
+ * sph.h -- C ABI of libsph, the B200-native SPH time-step library.
+ *
+ * What it computes.  One SPH-EXA hydro time step as measured by Simsek,
+ * Piccinali and Ciorba (SC'24 workshops, /root/reference/PAPER.md, "P:NN" =
+ * line NN): the particle keys of DomainDecompAndSync, neighbour
+ * search, XMass / density, equation of state, IADVelocityDivCurl
+ * (matrix part), MomentumEnergy, the end-of-step
+ * time-step collective and the update -- each wrapped by the
+ * per-function energy hooks of P:69-73 and, optionally, the per-function SM
+ * clock of P:73.  PAPER.md prints no SPH formula; the formulas are
+ * the readings of SURVEY.md 8(c) "Algorithm, step by step" (items 1-10),
+ * restated in DESIGN.md section 3.  Each entry point below cites its item.
+ *
+ * Conventions (apply to every function):
+ *  - Return value: SPH_OK (0) or one of the sph_status codes.  The message of
+ *    the last error is sph_last_error(ctx).  No C++ exception or abort crosses
+ *    this boundary.
+ *  - Argument errors (SPH_ERR_ARG) leave the context unchanged.
+ *  - CUDA errors are sticky: the context is poisoned and every later call
+ *    returns SPH_ERR_STATE until sph_finalize.
+ *  - Data errors detected on the device (degenerate open box, neighbour
+ *    capacity exceeded, singular IAD matrix) are reported at the next call that
+ *    synchronises (sph_find_neighbors, sph_timestep, sph_step, sph_get_*), do
+ *    not poison, and leave the outputs of the failing phase unspecified.
+ *  - NVML errors never poison: energy rows are marked unavailable, a refused
+ *    clock policy reverts to SPH_CLOCK_DEFAULT.
+ *  - Ownership: the caller owns ALL device memory (one byte arena of at least
+ *    sph_workspace_size bytes, 256-byte aligned, that must outlive the context)
+ *    and the CUDA stream.  The library sub-allocates fields, double buffers and
+ *    scratch inside the arena and allocates nothing on the device itself.  It
+ *    owns only its NVML handle and small host bookkeeping.
+ *  - Work is enqueued asynchronously on the caller's stream.  Calls that return
+ *    host values (sph_find_neighbors stats, sph_timestep, sph_step, sph_get_*,
+ *    accounting phase edges) synchronise that stream.
+ *  - One context per device per thread; a context is not internally
+ *    thread-safe.
+ *  - Particle arrays are fp64 structure-of-arrays; after sph_build_tree the
+ *    particles are held in Morton (SFC) order and every per-particle output is
+ *    in that order (SPH_F_ID gives the original ids).
+ */
+#ifndef SPH_H
+#define SPH_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SPH_ABI_VERSION 1
+
+typedef enum sph_status {
+  SPH_OK = 0,
+  SPH_ERR_ARG = 1,           /* invalid argument; nothing changed            */
+  SPH_ERR_STATE = 2,         /* call out of order, or context poisoned       */
+  SPH_ERR_CUDA = 3,          /* CUDA runtime error (poisons the context)     */
+  SPH_ERR_NCCL = 4,          /* reserved: multi-GPU communicator error        */
+  SPH_ERR_NVML = 5,          /* NVML unavailable or failed (never poisons)   */
+  SPH_ERR_NO_PERMISSION = 6, /* clock control refused by the host            */
+  SPH_ERR_NOT_SUPPORTED = 7, /* feature not supported on this device/host   */
+  SPH_ERR_CAPACITY = 8,      /* n > n_capacity or neighbour count > ngmax    */
+  SPH_ERR_HCAP = 9,          /* reserved                                      */
+  SPH_ERR_SINGULAR = 10,     /* IAD matrix with det <= 0 or non-finite       */
+  SPH_ERR_BOX = 11           /* open axis with max == min                    */
+} sph_status;
+
+typedef enum sph_eos_kind { SPH_EOS_IDEAL = 0, SPH_EOS_ISOTHERMAL = 1 } sph_eos_kind;
+typedef enum sph_mem_kind { SPH_MEM_HOST = 0, SPH_MEM_DEVICE = 1 } sph_mem_kind;
+typedef enum sph_accounting_mode {
+  SPH_ACCOUNTING_OFF = 0,   /* CUDA-event phase times only, no phase-edge syncs  */
+  SPH_ACCOUNTING_PHASE = 1  /* + stream sync and NVML energy read at every phase
+                               edge ("from the start of each function call
+                               until its completion")                             */
+} sph_accounting_mode;
+
+/* Phases = the functions whose energy the paper measures (Fig. 5).
+ * DomainDecompAndSync = KEYS + SORT + CELLS on one GPU. */
+typedef enum sph_phase {
+  SPH_PHASE_KEYS = 0,            /* box reduction + 63-bit Morton keys (item 1-2) */
+  SPH_PHASE_SORT = 1,            /* radix sort + permutation of all fields (3)    */
+  SPH_PHASE_CELLS = 2,           /* cell table over the sorted keys               */
+  SPH_PHASE_NEIGHBORS = 3,       /* neighbour lists (item 4)                      */
+  SPH_PHASE_DENSITY = 4,         /* XMass / density (item 5)                      */
+  SPH_PHASE_EOS = 5,             /* equation of state (item 6)                    */
+  SPH_PHASE_IAD = 6,             /* IAD matrices (item 7)                         */
+  SPH_PHASE_MOMENTUM_ENERGY = 7, /* momentum + energy + AV, local dt min (item 8) */
+  SPH_PHASE_TIMESTEP = 8,        /* global dt (item 9; the P:220 collective)      */
+  SPH_PHASE_UPDATE = 9,          /* positions, velocities, energy, h (item 10)    */
+  SPH_NPHASES = 10
+} sph_phase;
+
+typedef enum sph_clock_mode {
+  SPH_CLOCK_DEFAULT = 0,   /* driver DVFS (the paper's "DVFS" arm)            */
+  SPH_CLOCK_STATIC = 1,    /* one locked SM clock for every phase        */
+  SPH_CLOCK_PER_PHASE = 2  /* SM clock set before each phase ("ManDyn")   */
+} sph_clock_mode;
+
+/* Per-particle fields readable with sph_get_field (all in the current order). */
+typedef enum sph_field {
+  SPH_F_X = 0, SPH_F_Y, SPH_F_Z, SPH_F_VX, SPH_F_VY, SPH_F_VZ, SPH_F_H, SPH_F_M, SPH_F_U,
+  SPH_F_DU_M1,
+  SPH_F_ID,     /* int64: original particle id (the Morton order as an id list)   */
+  SPH_F_KEY,    /* uint64: Morton key (valid after sph_build_tree)                */
+  SPH_F_NC,     /* int32: neighbour count (valid after sph_find_neighbors)        */
+  SPH_F_RHO, SPH_F_P, SPH_F_C,
+  SPH_F_C11, SPH_F_C12, SPH_F_C13, SPH_F_C22, SPH_F_C23, SPH_F_C33,
+  SPH_F_AX, SPH_F_AY, SPH_F_AZ, SPH_F_DU,
+  SPH_NFIELDS
+} sph_field;
+
+/* Step configuration.  Values are inputs to the method (SURVEY 8(c) parameter
+ * table); sph_config_default fills the proposed defaults. */
+typedef struct sph_config {
+  int64_t n_capacity;       /* max particles held (< 2^30)                        */
+  double box_min[3];        /* periodic axes: the fixed box; open axes: ignored   */
+  double box_max[3];
+  int32_t periodic[3];      /* 1 = periodic axis (minimum image + wrap)           */
+  int32_t eos;              /* sph_eos_kind                                        */
+  double gamma;             /* ideal-gas gamma                                     */
+  double cs0;               /* isothermal sound speed                              */
+  double K;                 /* sinc-kernel (n = 6) normalisation                   */
+  double ng0;               /* target neighbour count of the h update              */
+  int32_t ngmax;            /* neighbour-list capacity per particle (never truncates:
+                               overflow -> SPH_ERR_CAPACITY)                       */
+  int32_t max_cell_level;   /* finest cell-grid level L (8^L cells), <= 10         */
+  double h_cap;             /* h <= h_cap after the update (periodic: <= min L / 4) */
+  double k_cour;            /* Courant factor                                      */
+  double dt_max_growth;     /* dt <= growth * dt_prev                              */
+  double dt_first;          /* dt_prev before the first step                       */
+  double av_alpha, av_beta, av_eps;
+  int32_t device;           /* CUDA device ordinal the arena lives on              */
+  int32_t accounting;       /* sph_accounting_mode                                 */
+  int32_t rank, nranks;     /* reserved for SFC domain decomposition (1 rank now)  */
+  int32_t reserved[16];
+} sph_config;
+
+typedef struct sph_nbr_stats {
+  int32_t min_nc, max_nc;   /* over all particles                                  */
+  double mean_nc;
+  int64_t total;            /* sum of nc                                           */
+} sph_nbr_stats;
+
+typedef struct sph_step_info {
+  double t;                 /* simulation time after the step                      */
+  double dt;                /* the step's dt                                       */
+  sph_nbr_stats nbr;
+  int32_t cell_level;       /* cell-grid level used by the neighbour search        */
+  int32_t reserved;
+  double phase_ms[SPH_NPHASES]; /* CUDA-event time of each phase in this step      */
+} sph_step_info;
+
+typedef struct sph_energy_row {
+  int32_t phase;            /* sph_phase                                           */
+  char name[32];
+  int64_t calls;
+  double seconds;           /* accumulated CUDA-event time                         */
+  double joules;            /* accumulated NVML energy delta (PHASE accounting)    */
+  double mean_sm_mhz;       /* mean SM clock read at the phase's end edges         */
+  uint32_t locked_mhz;      /* clock requested by the policy, 0 = default          */
+  int32_t available;        /* 1 if joules are valid                               */
+} sph_energy_row;
+
+typedef struct sph_ctx sph_ctx;
+
+/* --- configuration and lifetime --------------------------------------------- */
+
+/* Fills *cfg with the defaults of SURVEY 8(c): unit periodic box [-0.5,0.5]^3,
+ * ideal gas gamma 5/3, exact K, ng0 100, ngmax 150, L <= 8, h_cap 0.25, C 0.2,
+ * growth 1.1, dt_first 1e-6, alpha 1, beta 2, eps 0.01.  Pure. */
+int sph_config_default(sph_config* cfg);
+
+/* Bytes of device arena needed for cfg (pure; no CUDA call). */
+int sph_workspace_size(const sph_config* cfg, size_t* bytes);
+
+/* Creates a context on cfg->device using the caller's arena (device pointer,
+ * >= sph_workspace_size bytes, 256-B aligned) and stream (cudaStream_t, may be
+ * NULL for the legacy stream).  Initialises NVML when available. */
+int sph_init(const sph_config* cfg, void* arena, size_t arena_bytes, void* stream, sph_ctx** out);
+
+/* Resets any locked clock this context set (NVML), releases host bookkeeping.
+ * The arena is the caller's to free afterwards.  NULL is a no-op. */
+void sph_finalize(sph_ctx* ctx);
+
+const char* sph_last_error(const sph_ctx* ctx);
+const char* sph_phase_name(int phase);
+
+/* --- particle I/O ------------------------------------------------------------ */
+
+/* Copies n particles in (mem = SPH_MEM_HOST or SPH_MEM_DEVICE pointers, each an
+ * array of n values).  du_m1 may be NULL (zeros); id may be NULL (0..n-1).
+ * n > n_capacity -> SPH_ERR_CAPACITY.  n = 0 is allowed (every phase is then a
+ * no-op and sph_step returns dt = growth * dt_prev).  Resets the stage machine
+ * to "particles set".  Periodic coordinates must lie in [box_min, box_max]. */
+int sph_set_particles(sph_ctx* ctx, int64_t n, const double* x, const double* y, const double* z,
+                      const double* vx, const double* vy, const double* vz, const double* h,
+                      const double* m, const double* u, const double* du_m1, const int64_t* id,
+                      int mem);
+
+/* Sets the integrator clock: current time, dt of the previous step (dt_m1 of
+ * item 10) and whether the next step is the first (du_m1 := du). */
+int sph_set_time(sph_ctx* ctx, double t, double dt_prev, int first_step);
+int sph_get_time(sph_ctx* ctx, double* t, double* dt_prev, int* first_step);
+
+int sph_get_n(const sph_ctx* ctx, int64_t* n);
+
+/* Copies field f (n values; int64 for SPH_F_ID, uint64 for SPH_F_KEY, int32 for
+ * SPH_F_NC, double otherwise) to dst (host or device).  Synchronises. */
+int sph_get_field(sph_ctx* ctx, int field, void* dst, int mem);
+
+/* --- the hot path (each call = one accounted phase group) ------------------- */
+
+/* Items 1-3: box (open axes: exact min/max), 63-bit Morton keys, stable LSD
+ * radix sort (onesweep, 8 x 8-bit digits) and permutation of every particle
+ * field into key order; then the cell table (level L = finest with cell side >=
+ * 2 h_max on every axis, L <= max_cell_level).  Phases KEYS, SORT, CELLS. */
+int sph_build_tree(sph_ctx* ctx);
+
+/* Item 4: j in N(i) iff j != i and d2 < (2 h_i)^2 with d the minimum image,
+ * d2 = (dx*dx + dy*dy) + dz*dz rounded per operation (bit-exact vs brute force).
+ * Lists are ascending in the current order.  Fills *stats when non-NULL
+ * (synchronises).  max nc > ngmax -> SPH_ERR_CAPACITY, stats.max_nc = needed. */
+int sph_find_neighbors(sph_ctx* ctx, sph_nbr_stats* stats);
+
+/* Copies the neighbour lists to host CSR: offsets[n+1] (int64), idx (int32,
+ * current-order indices, ascending per particle).  idx_cap < total ->
+ * SPH_ERR_CAPACITY with offsets still filled. */
+int sph_get_neighbors(sph_ctx* ctx, int64_t* offsets, int32_t* idx, int64_t idx_cap);
+
+/* Item 5 (XMass): rho_i = (K/h_i^3) [m_i + sum_j m_j S(pi r_ij/2h_i)^6].  DENSITY. */
+int sph_density(sph_ctx* ctx);
+
+/* Item 6: ideal p = (gamma-1) rho u, c = sqrt(gamma (gamma-1) u); isothermal
+ * p = c0^2 rho, c = c0.  EOS. */
+int sph_eos(sph_ctx* ctx);
+
+/* Item 7 (IADVelocityDivCurl, matrix part): tau_i = sum_j (m_j/rho_j) W(r,h_i)
+ * Delta Delta^T, C_i = tau_i^{-1} (adjugate).  SPH_ERR_SINGULAR is reported at
+ * the next synchronising call.  IAD. */
+int sph_iad(sph_ctx* ctx);
+
+/* Item 8 (MomentumEnergy): a_i, du_i with IAD gradients and Monaghan AV, plus
+ * the local min_i h_i/c_i for item 9.  MOMENTUM_ENERGY. */
+int sph_momentum_energy(sph_ctx* ctx);
+
+/* Item 9: dt = min(C min_i h_i/c_i, growth dt_prev).  Synchronises; *dt may be
+ * NULL.  TIMESTEP. */
+int sph_timestep(sph_ctx* ctx, double* dt);
+
+/* Item 10: kick, drift (+ periodic wrap), AB2 energy update, h update; advances
+ * t and dt_prev.  UPDATE. */
+int sph_update(sph_ctx* ctx);
+
+/* Items 1-10 in order; legal whenever particles are set.  Synchronises once at
+ * the end (plus at every phase edge with PHASE accounting). */
+int sph_step(sph_ctx* ctx, sph_step_info* info);
+
+/* --- energy and clocks ------------------------------------------- */
+
+/* Clock policy: DEFAULT, STATIC (mhz[0] for every phase) or PER_PHASE (mhz[p]
+ * set before phase p, skipped when unchanged; 0 = leave the clock as is).
+ * Requests snap to the nearest supported graphics clock.  Uses
+ * nvmlDeviceSetGpuLockedClocks; this needs root and is disabled unless the
+ * environment sets SPH_ALLOW_CLOCK_CONTROL=1 (shared hosts forbid clock changes)
+ * -> SPH_ERR_NO_PERMISSION / SPH_ERR_NOT_SUPPORTED leave the policy DEFAULT. */
+int sph_set_clock_policy(sph_ctx* ctx, int mode, const uint32_t mhz[SPH_NPHASES]);
+
+/* One row per phase (cap >= SPH_NPHASES).  Time is always filled; joules only
+ * with PHASE accounting and a working NVML energy counter. */
+int sph_energy_report(sph_ctx* ctx, sph_energy_row* rows, int cap, int* n_rows);
+int sph_energy_reset(sph_ctx* ctx);
+
+/* Total-energy counter of the device in mJ (NVML), for whole-run deltas. */
+int sph_energy_counter_mj(sph_ctx* ctx, uint64_t* mj);
+
+/* Switches the accounting mode of an existing context (sph_accounting_mode). */
+int sph_set_accounting(sph_ctx* ctx, int mode);
+
+/* Number of libsph kernels launched by this process so far (all contexts);
+ * for the bench's launch count. */
+int sph_kernel_launches(int64_t* count);
+
+/* Re-runs one pure phase (NEIGHBORS, DENSITY, EOS, IAD, MOMENTUM_ENERGY) reps
+ * times back to back on the same inputs -- the KernelTuner-style isolated
+ * measurement of P:81-87 -- and returns its mean time and energy per call
+ * (joules < 0 when NVML is unavailable).  Synchronises. */
+int sph_repeat_phase(sph_ctx* ctx, int phase, int reps, double* ms_per_call,
+                     double* joules_per_call);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SPH_H */

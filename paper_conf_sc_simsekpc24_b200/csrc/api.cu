@@ -1,0 +1,821 @@
+// api.cu -- the C ABI of include/sph.h: arena sub-allocation, the stage machine,
+// phase wrappers with CUDA-event timing, NVML energy accounting and the
+// per-phase clock policy.  All compute is in the k_*.cu kernels.
+#include <stdarg.h>
+#include <stdio.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <algorithm>
+#include <chrono>
+#include <vector>
+
+#include "nvml_dyn.h"
+#include "sph_internal.cuh"
+
+using namespace sph;
+
+std::atomic<long long> sph::g_launches{0};
+
+namespace {
+
+enum Stage { S_INIT = 0, S_PART, S_TREE, S_NBR, S_DENS, S_EOS, S_IAD, S_MOM, S_DT };
+
+const char* kPhaseNames[SPH_NPHASES] = {"keys",    "sort",    "cells", "neighbors",
+                                        "density", "eos",     "iad",   "momentum_energy",
+                                        "timestep", "update"};
+
+thread_local char g_err[512] = "";
+
+constexpr size_t kAlign = 256;
+inline size_t align_up(size_t v) { return (v + kAlign - 1) / kAlign * kAlign; }
+
+int level_cap_for(const sph_config* c) {
+  int L = std::min(c->max_cell_level, 10);
+  int64_t limit = std::max<int64_t>(8 * c->n_capacity, 512);
+  while (L > 0 && (int64_t(1) << (3 * L)) > limit) --L;
+  return std::max(L, 0);
+}
+
+struct PhaseRow {
+  int64_t calls = 0;
+  double seconds = 0, joules = 0, mhz_sum = 0;
+  int64_t mhz_n = 0;
+  unsigned locked = 0;
+  bool avail = false;
+};
+
+}  // namespace
+
+struct sph_ctx {
+  sph_config cfg;
+  Params P;
+  cudaStream_t st = nullptr;
+  int64_t n = 0;
+  int level_cap = 0;
+  // arena slices
+  double* state[2][kNumStateF];
+  int64_t* ids[2];
+  int cur = 0;
+  uint64_t *keyA, *keyB, *key_sorted;
+  uint32_t *valA, *valB;
+  double *rho, *p, *c, *vol, *prho2, *wq, *wk, *C[6], *ax, *ay, *az, *du;
+  int32_t *nc, *nbr;
+  uint32_t* cell_start;
+  uint32_t *sort_hist, *sort_status;
+  size_t status_bytes;
+  DevScalars* ds;
+  DevScalars h_ds;
+  // state machine / errors
+  int stage = S_INIT;
+  bool poisoned = false;
+  char err[512] = "";
+  // timing / accounting
+  cudaEvent_t ev[SPH_NPHASES][2];
+  bool pending[SPH_NPHASES];
+  double last_ms[SPH_NPHASES];
+  PhaseRow rows[SPH_NPHASES];
+  unsigned long long e0 = 0;
+  bool e0_ok = false;
+  Nvml nvml;
+  int clock_mode = SPH_CLOCK_DEFAULT;
+  unsigned clock_mhz[SPH_NPHASES];
+  unsigned current_lock = 0;
+  bool locked_any = false;
+};
+
+namespace {
+
+int fail(sph_ctx* c, int code, const char* fmt, ...) {
+  char* buf = c ? c->err : g_err;
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, 512, fmt, ap);
+  va_end(ap);
+  return code;
+}
+
+int cuda_check(sph_ctx* c, cudaError_t e, const char* where) {
+  if (e == cudaSuccess) e = cudaGetLastError();
+  if (e != cudaSuccess) {
+    c->poisoned = true;
+    return fail(c, SPH_ERR_CUDA, "%s: %s", where, cudaGetErrorString(e));
+  }
+  return SPH_OK;
+}
+
+int check_ready(sph_ctx* c, int min_stage, const char* what) {
+  if (!c) return fail(nullptr, SPH_ERR_ARG, "%s: null context", what);
+  if (c->poisoned) return fail(c, SPH_ERR_STATE, "%s: context poisoned by an earlier CUDA error", what);
+  if (c->stage < min_stage) return fail(c, SPH_ERR_STATE, "%s: called out of order (stage %d < %d)", what, c->stage, min_stage);
+  return SPH_OK;
+}
+
+Fields fields(sph_ctx* c) {
+  Fields F;
+  F.n = c->n;
+  F.cap = c->cfg.n_capacity;
+  for (int f = 0; f < kNumStateF; ++f) F.f[f] = c->state[c->cur][f];
+  F.id = c->ids[c->cur];
+  F.key = c->key_sorted;
+  F.rho = c->rho; F.p = c->p; F.c = c->c; F.vol = c->vol; F.prho2 = c->prho2;
+  F.wq = c->wq; F.wk = c->wk;
+  for (int e = 0; e < 6; ++e) F.C[e] = c->C[e];
+  F.ax = c->ax; F.ay = c->ay; F.az = c->az; F.du = c->du;
+  F.nc = c->nc; F.nbr = c->nbr; F.ngmax = c->cfg.ngmax;
+  F.cell_start = c->cell_start;
+  F.ds = c->ds;
+  return F;
+}
+
+void collect_phase(sph_ctx* c, int p) {
+  if (!c->pending[p]) return;
+  float ms = 0.f;
+  if (cudaEventElapsedTime(&ms, c->ev[p][0], c->ev[p][1]) == cudaSuccess) {
+    c->rows[p].seconds += ms * 1e-3;
+    c->last_ms[p] = ms;
+  } else {
+    cudaGetLastError();
+  }
+  c->pending[p] = false;
+}
+
+void collect_all(sph_ctx* c) {
+  for (int p = 0; p < SPH_NPHASES; ++p) collect_phase(c, p);
+}
+
+void apply_clock(sph_ctx* c, int p) {
+  if (c->clock_mode == SPH_CLOCK_DEFAULT) return;
+  unsigned want = c->clock_mhz[p];
+  if (want == 0 || want == c->current_lock) return;
+  if (c->nvml.lock_sm_clock(want) == 0) {
+    c->current_lock = want;
+    c->locked_any = true;
+  }
+}
+
+int phase_begin(sph_ctx* c, int p) {
+  if (c->pending[p]) {
+    cudaEventSynchronize(c->ev[p][1]);
+    collect_phase(c, p);
+  }
+  apply_clock(c, p);
+  c->rows[p].locked = c->current_lock;
+  if (c->cfg.accounting == SPH_ACCOUNTING_PHASE) {
+    int rc = cuda_check(c, cudaStreamSynchronize(c->st), "phase sync");
+    if (rc) return rc;
+    c->e0_ok = c->nvml.energy_mj(&c->e0);
+  }
+  return cuda_check(c, cudaEventRecord(c->ev[p][0], c->st), "cudaEventRecord");
+}
+
+int phase_end(sph_ctx* c, int p) {
+  int rc = cuda_check(c, cudaEventRecord(c->ev[p][1], c->st), "phase kernels");
+  if (rc) return rc;
+  c->pending[p] = true;
+  c->rows[p].calls++;
+  if (c->cfg.accounting == SPH_ACCOUNTING_PHASE) {
+    rc = cuda_check(c, cudaStreamSynchronize(c->st), "phase sync");
+    if (rc) return rc;
+    unsigned long long e1;
+    if (c->e0_ok && c->nvml.energy_mj(&e1)) {
+      c->rows[p].joules += (double)(e1 - c->e0) * 1e-3;
+      c->rows[p].avail = true;
+    }
+    unsigned mhz;
+    if (c->nvml.sm_clock_mhz(&mhz)) {
+      c->rows[p].mhz_sum += mhz;
+      c->rows[p].mhz_n++;
+    }
+  }
+  return SPH_OK;
+}
+
+// Reads the device scalars (synchronises) and maps device status bits to codes.
+int sync_scalars(sph_ctx* c) {
+  int rc = cuda_check(c, cudaMemcpyAsync(&c->h_ds, c->ds, sizeof(DevScalars), cudaMemcpyDeviceToHost, c->st), "scalar copy");
+  if (rc) return rc;
+  rc = cuda_check(c, cudaStreamSynchronize(c->st), "stream sync");
+  if (rc) return rc;
+  collect_all(c);
+  int s = c->h_ds.status;
+  if (s & ST_BOX) return fail(c, SPH_ERR_BOX, "degenerate open-axis box (max == min)");
+  if (s & ST_CAPACITY)
+    return fail(c, SPH_ERR_CAPACITY, "neighbour count %d exceeds ngmax %d", c->h_ds.max_nc, c->cfg.ngmax);
+  if (s & ST_SINGULAR) return fail(c, SPH_ERR_SINGULAR, "singular IAD matrix (det <= 0 or non-finite)");
+  return SPH_OK;
+}
+
+void fill_stats(sph_ctx* c, sph_nbr_stats* s) {
+  if (!s) return;
+  s->min_nc = c->n ? c->h_ds.min_nc : 0;
+  s->max_nc = c->h_ds.max_nc;
+  s->total = (int64_t)c->h_ds.total_nc;
+  s->mean_nc = c->n ? (double)c->h_ds.total_nc / (double)c->n : 0.0;
+}
+
+__global__ void set_time_kernel(DevScalars* ds, double t, double dt_prev, int first) {
+  ds->t = t;
+  ds->dt_prev = dt_prev;
+  ds->dt = 0.0;
+  ds->first = first;
+}
+
+__global__ void iota_kernel(int64_t* id, int64_t n) {
+  int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i < n) id[i] = i;
+}
+
+__global__ void reset_nbr_stats_kernel(DevScalars* ds) {
+  ds->max_nc = 0;
+  ds->min_nc = 0x7fffffff;
+  ds->total_nc = 0ull;
+  ds->status &= ~ST_CAPACITY;
+}
+
+// ---- phase bodies (enqueue only) ----
+int body_tree(sph_ctx* c) {
+  int rc;
+  if ((rc = phase_begin(c, SPH_PHASE_KEYS))) return rc;
+  launch_reset_scalars(c->ds, c->P, c->st);
+  c->key_sorted = c->keyA;
+  Fields F = fields(c);
+  F.key = c->keyA;
+  launch_box_keys(F, c->P, c->st);
+  if ((rc = phase_end(c, SPH_PHASE_KEYS))) return rc;
+
+  if ((rc = phase_begin(c, SPH_PHASE_SORT))) return rc;
+  uint32_t* perm = nullptr;
+  uint64_t* ksorted = nullptr;
+  cudaError_t e = launch_sort(F, c->keyA, c->keyB, c->valA, c->valB, c->sort_hist, c->sort_status,
+                              c->status_bytes, &perm, &ksorted, c->st);
+  if ((rc = cuda_check(c, e, "sort"))) return rc;
+  const int nxt = c->cur ^ 1;
+  launch_permute(c->n, perm, c->state[c->cur], c->state[nxt], c->ids[c->cur], c->ids[nxt], c->st);
+  c->cur = nxt;
+  c->key_sorted = ksorted;
+  if ((rc = phase_end(c, SPH_PHASE_SORT))) return rc;
+
+  if ((rc = phase_begin(c, SPH_PHASE_CELLS))) return rc;
+  launch_cells(fields(c), c->P, c->level_cap, c->st);
+  if ((rc = phase_end(c, SPH_PHASE_CELLS))) return rc;
+  c->stage = S_TREE;
+  return SPH_OK;
+}
+
+int body_neighbors(sph_ctx* c) {
+  int rc;
+  if ((rc = phase_begin(c, SPH_PHASE_NEIGHBORS))) return rc;
+  reset_nbr_stats_kernel<<<1, 1, 0, c->st>>>(c->ds); note_launch();
+  launch_neighbors(fields(c), c->P, c->st);
+  if ((rc = phase_end(c, SPH_PHASE_NEIGHBORS))) return rc;
+  c->stage = S_NBR;
+  return SPH_OK;
+}
+
+int body_simple(sph_ctx* c, int phase, int next_stage) {
+  int rc;
+  if ((rc = phase_begin(c, phase))) return rc;
+  Fields F = fields(c);
+  switch (phase) {
+    case SPH_PHASE_DENSITY: launch_density(F, c->P, c->st); break;
+    case SPH_PHASE_EOS: launch_eos(F, c->P, c->st); break;
+    case SPH_PHASE_IAD: launch_iad(F, c->P, c->st); break;
+    case SPH_PHASE_MOMENTUM_ENERGY:
+      cudaMemsetAsync(&c->ds->minhc_ord, 0xff, sizeof(unsigned long long), c->st);
+      launch_momentum_energy(F, c->P, c->st);
+      break;
+    case SPH_PHASE_TIMESTEP: launch_timestep(F, c->P, c->st); break;
+    case SPH_PHASE_UPDATE:
+      launch_update(F, c->P, c->st);
+      launch_advance_time(F, c->st);
+      break;
+  }
+  if ((rc = phase_end(c, phase))) return rc;
+  c->stage = next_stage;
+  return SPH_OK;
+}
+
+}  // namespace
+
+// =========================================================================== ABI
+
+extern "C" {
+
+int sph_config_default(sph_config* cfg) {
+  if (!cfg) return fail(nullptr, SPH_ERR_ARG, "null config");
+  memset(cfg, 0, sizeof(*cfg));
+  cfg->n_capacity = 1 << 20;
+  for (int a = 0; a < 3; ++a) {
+    cfg->box_min[a] = -0.5;
+    cfg->box_max[a] = 0.5;
+    cfg->periodic[a] = 1;
+  }
+  cfg->eos = SPH_EOS_IDEAL;
+  cfg->gamma = 5.0 / 3.0;
+  cfg->cs0 = 1.0;
+  cfg->K = 0.79044958943230290;
+  cfg->ng0 = 100.0;
+  cfg->ngmax = 150;
+  cfg->max_cell_level = 8;
+  cfg->h_cap = 0.25;
+  cfg->k_cour = 0.2;
+  cfg->dt_max_growth = 1.1;
+  cfg->dt_first = 1e-6;
+  cfg->av_alpha = 1.0;
+  cfg->av_beta = 2.0;
+  cfg->av_eps = 0.01;
+  cfg->device = 0;
+  cfg->accounting = SPH_ACCOUNTING_OFF;
+  cfg->rank = 0;
+  cfg->nranks = 1;
+  return SPH_OK;
+}
+
+static int validate(const sph_config* c) {
+  if (!c) return fail(nullptr, SPH_ERR_ARG, "null config");
+  if (c->n_capacity < 1 || c->n_capacity >= (int64_t(1) << 30))
+    return fail(nullptr, SPH_ERR_ARG, "n_capacity must be in [1, 2^30)");
+  if (c->ngmax < 1 || c->ngmax > 4096) return fail(nullptr, SPH_ERR_ARG, "ngmax must be in [1, 4096]");
+  if (c->max_cell_level < 0 || c->max_cell_level > 10) return fail(nullptr, SPH_ERR_ARG, "max_cell_level must be in [0, 10]");
+  for (int a = 0; a < 3; ++a)
+    if (c->periodic[a] && !(c->box_max[a] > c->box_min[a])) return fail(nullptr, SPH_ERR_ARG, "periodic axis %d: box_max <= box_min", a);
+  if (c->eos != SPH_EOS_IDEAL && c->eos != SPH_EOS_ISOTHERMAL) return fail(nullptr, SPH_ERR_ARG, "unknown eos %d", c->eos);
+  if (!(c->K > 0) || !(c->dt_first > 0) || !(c->h_cap > 0)) return fail(nullptr, SPH_ERR_ARG, "K, dt_first and h_cap must be > 0");
+  if (c->nranks != 1) return fail(nullptr, SPH_ERR_NOT_SUPPORTED, "nranks > 1 is not built into this library version");
+  return SPH_OK;
+}
+
+// Computes the arena layout; with ctx != NULL also assigns the slices.
+static size_t layout(const sph_config* cfg, char* base, sph_ctx* c) {
+  const size_t cap = (size_t)cfg->n_capacity;
+  size_t o = 0;
+  auto take = [&](size_t bytes) -> char* {
+    char* r = base ? base + o : nullptr;
+    o += align_up(bytes);
+    return r;
+  };
+  const size_t D = sizeof(double) * cap;
+  for (int b = 0; b < 2; ++b) {
+    for (int f = 0; f < kNumStateF; ++f) {
+      char* p = take(D);
+      if (c) c->state[b][f] = (double*)p;
+    }
+    char* p = take(sizeof(int64_t) * cap);
+    if (c) c->ids[b] = (int64_t*)p;
+  }
+  char* kA = take(sizeof(uint64_t) * cap);
+  char* kB = take(sizeof(uint64_t) * cap);
+  char* vA = take(sizeof(uint32_t) * cap);
+  char* vB = take(sizeof(uint32_t) * cap);
+  double** dst[] = {c ? &c->rho : nullptr, c ? &c->p : nullptr, c ? &c->c : nullptr,
+                    c ? &c->vol : nullptr, c ? &c->prho2 : nullptr, c ? &c->wq : nullptr,
+                    c ? &c->wk : nullptr, c ? &c->ax : nullptr, c ? &c->ay : nullptr,
+                    c ? &c->az : nullptr, c ? &c->du : nullptr};
+  for (double** d : dst) {
+    char* p = take(D);
+    if (c) *d = (double*)p;
+  }
+  for (int e = 0; e < 6; ++e) {
+    char* p = take(D);
+    if (c) c->C[e] = (double*)p;
+  }
+  char* ncp = take(sizeof(int32_t) * cap);
+  char* nbp = take(sizeof(int32_t) * cap * (size_t)cfg->ngmax);
+  const int Lc = level_cap_for(cfg);
+  char* cs = take(sizeof(uint32_t) * ((size_t(1) << (3 * Lc)) + 1));
+  size_t hb, sb;
+  sort_workspace(cfg->n_capacity, &hb, &sb);
+  char* hp = take(hb);
+  char* sp = take(sb);
+  char* dsp = take(sizeof(DevScalars));
+  if (c) {
+    c->keyA = (uint64_t*)kA; c->keyB = (uint64_t*)kB;
+    c->valA = (uint32_t*)vA; c->valB = (uint32_t*)vB;
+    c->nc = (int32_t*)ncp; c->nbr = (int32_t*)nbp;
+    c->cell_start = (uint32_t*)cs;
+    c->level_cap = Lc;
+    c->sort_hist = (uint32_t*)hp; c->sort_status = (uint32_t*)sp; c->status_bytes = sb;
+    c->ds = (DevScalars*)dsp;
+    c->key_sorted = c->keyA;
+  }
+  return o;
+}
+
+int sph_workspace_size(const sph_config* cfg, size_t* bytes) {
+  int rc = validate(cfg);
+  if (rc) return rc;
+  if (!bytes) return fail(nullptr, SPH_ERR_ARG, "null bytes");
+  *bytes = layout(cfg, nullptr, nullptr);
+  return SPH_OK;
+}
+
+int sph_init(const sph_config* cfg, void* arena, size_t arena_bytes, void* stream, sph_ctx** out) {
+  int rc = validate(cfg);
+  if (rc) return rc;
+  if (!out) return fail(nullptr, SPH_ERR_ARG, "null out");
+  *out = nullptr;
+  size_t need = layout(cfg, nullptr, nullptr);
+  if (!arena || arena_bytes < need)
+    return fail(nullptr, SPH_ERR_ARG, "arena too small: %zu < %zu bytes", arena_bytes, need);
+  if (((uintptr_t)arena) % kAlign) return fail(nullptr, SPH_ERR_ARG, "arena not 256-byte aligned");
+  cudaError_t e = cudaSetDevice(cfg->device);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return fail(nullptr, SPH_ERR_CUDA, "cudaSetDevice(%d): %s", cfg->device, cudaGetErrorString(e));
+  }
+  sph_ctx* c = new (std::nothrow) sph_ctx();
+  if (!c) return fail(nullptr, SPH_ERR_ARG, "out of host memory");
+  c->cfg = *cfg;
+  c->st = (cudaStream_t)stream;
+  for (int a = 0; a < 3; ++a) {
+    c->P.box_min[a] = cfg->box_min[a];
+    c->P.box_max[a] = cfg->box_max[a];
+    c->P.periodic[a] = cfg->periodic[a];
+  }
+  c->P.eos = cfg->eos; c->P.gamma = cfg->gamma; c->P.cs0 = cfg->cs0; c->P.K = cfg->K;
+  c->P.ng0 = cfg->ng0; c->P.h_cap = cfg->h_cap; c->P.k_cour = cfg->k_cour;
+  c->P.dt_max_growth = cfg->dt_max_growth; c->P.av_alpha = cfg->av_alpha;
+  c->P.av_beta = cfg->av_beta; c->P.av_eps = cfg->av_eps; c->P.max_cell_level = cfg->max_cell_level;
+  layout(cfg, (char*)arena, c);
+  for (int p = 0; p < SPH_NPHASES; ++p) {
+    c->pending[p] = false;
+    c->last_ms[p] = 0;
+    c->clock_mhz[p] = 0;
+    for (int k = 0; k < 2; ++k) {
+      e = cudaEventCreate(&c->ev[p][k]);
+      if (e != cudaSuccess) {
+        cudaGetLastError();
+        delete c;
+        return fail(nullptr, SPH_ERR_CUDA, "cudaEventCreate: %s", cudaGetErrorString(e));
+      }
+    }
+  }
+  launch_reset_scalars(c->ds, c->P, c->st);
+  set_time_kernel<<<1, 1, 0, c->st>>>(c->ds, 0.0, cfg->dt_first, 1); note_launch();
+  e = cudaStreamSynchronize(c->st);
+  if (e == cudaSuccess) e = cudaGetLastError();
+  if (e != cudaSuccess) {
+    fail(nullptr, SPH_ERR_CUDA, "init kernels: %s", cudaGetErrorString(e));
+    delete c;
+    return SPH_ERR_CUDA;
+  }
+  c->nvml.init(cfg->device);  // failure only disables energy/clock features
+  c->stage = S_INIT;
+  *out = c;
+  return SPH_OK;
+}
+
+void sph_finalize(sph_ctx* c) {
+  if (!c) return;
+  if (c->locked_any) c->nvml.reset_sm_clock();
+  c->nvml.shutdown();
+  if (!c->poisoned) cudaStreamSynchronize(c->st);
+  for (int p = 0; p < SPH_NPHASES; ++p)
+    for (int k = 0; k < 2; ++k) cudaEventDestroy(c->ev[p][k]);
+  cudaGetLastError();
+  delete c;
+}
+
+const char* sph_last_error(const sph_ctx* c) { return c ? c->err : g_err; }
+
+const char* sph_phase_name(int p) {
+  return (p >= 0 && p < SPH_NPHASES) ? kPhaseNames[p] : "unknown";
+}
+
+int sph_set_particles(sph_ctx* c, int64_t n, const double* x, const double* y, const double* z,
+                      const double* vx, const double* vy, const double* vz, const double* h,
+                      const double* m, const double* u, const double* du_m1, const int64_t* id,
+                      int mem) {
+  int rc = check_ready(c, S_INIT, "sph_set_particles");
+  if (rc) return rc;
+  if (n < 0) return fail(c, SPH_ERR_ARG, "n < 0");
+  if (n > c->cfg.n_capacity) return fail(c, SPH_ERR_CAPACITY, "n = %lld exceeds n_capacity %lld", (long long)n, (long long)c->cfg.n_capacity);
+  if (mem != SPH_MEM_HOST && mem != SPH_MEM_DEVICE) return fail(c, SPH_ERR_ARG, "mem must be HOST or DEVICE");
+  const double* src[kNumStateF] = {x, y, z, vx, vy, vz, h, m, u, du_m1};
+  for (int f = 0; f < kNumStateF - 1; ++f)
+    if (n > 0 && !src[f]) return fail(c, SPH_ERR_ARG, "null particle array %d", f);
+  const cudaMemcpyKind kind = mem == SPH_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
+  c->n = n;
+  if (n > 0) {
+    for (int f = 0; f < kNumStateF; ++f) {
+      if (src[f]) rc = cuda_check(c, cudaMemcpyAsync(c->state[c->cur][f], src[f], sizeof(double) * n, kind, c->st), "particle copy");
+      else rc = cuda_check(c, cudaMemsetAsync(c->state[c->cur][f], 0, sizeof(double) * n, c->st), "memset");
+      if (rc) return rc;
+    }
+    if (id) rc = cuda_check(c, cudaMemcpyAsync(c->ids[c->cur], id, sizeof(int64_t) * n, kind, c->st), "id copy");
+    else {
+      iota_kernel<<<(unsigned)div_up(n, 256), 256, 0, c->st>>>(c->ids[c->cur], n); note_launch();
+      rc = cuda_check(c, cudaSuccess, "iota");
+    }
+    if (rc) return rc;
+  }
+  c->stage = S_PART;
+  return SPH_OK;
+}
+
+int sph_set_time(sph_ctx* c, double t, double dt_prev, int first_step) {
+  int rc = check_ready(c, S_INIT, "sph_set_time");
+  if (rc) return rc;
+  if (!(dt_prev > 0)) return fail(c, SPH_ERR_ARG, "dt_prev must be > 0");
+  set_time_kernel<<<1, 1, 0, c->st>>>(c->ds, t, dt_prev, first_step ? 1 : 0); note_launch();
+  return cuda_check(c, cudaSuccess, "set_time");
+}
+
+int sph_get_time(sph_ctx* c, double* t, double* dt_prev, int* first_step) {
+  int rc = check_ready(c, S_INIT, "sph_get_time");
+  if (rc) return rc;
+  rc = cuda_check(c, cudaMemcpyAsync(&c->h_ds, c->ds, sizeof(DevScalars), cudaMemcpyDeviceToHost, c->st), "copy");
+  if (!rc) rc = cuda_check(c, cudaStreamSynchronize(c->st), "sync");
+  if (rc) return rc;
+  if (t) *t = c->h_ds.t;
+  if (dt_prev) *dt_prev = c->h_ds.dt_prev;
+  if (first_step) *first_step = c->h_ds.first;
+  return SPH_OK;
+}
+
+int sph_get_n(const sph_ctx* c, int64_t* n) {
+  if (!c || !n) return fail(nullptr, SPH_ERR_ARG, "null argument");
+  *n = c->n;
+  return SPH_OK;
+}
+
+int sph_get_field(sph_ctx* c, int field, void* dst, int mem) {
+  int rc = check_ready(c, S_INIT, "sph_get_field");
+  if (rc) return rc;
+  if (!dst && c->n > 0) return fail(c, SPH_ERR_ARG, "null dst");
+  if (mem != SPH_MEM_HOST && mem != SPH_MEM_DEVICE) return fail(c, SPH_ERR_ARG, "mem must be HOST or DEVICE");
+  const void* src = nullptr;
+  size_t esz = sizeof(double);
+  if (field >= SPH_F_X && field <= SPH_F_DU_M1) src = c->state[c->cur][field - SPH_F_X];
+  else if (field == SPH_F_ID) { src = c->ids[c->cur]; esz = 8; }
+  else if (field == SPH_F_KEY) { src = c->key_sorted; esz = 8; }
+  else if (field == SPH_F_NC) { src = c->nc; esz = 4; }
+  else if (field == SPH_F_RHO) src = c->rho;
+  else if (field == SPH_F_P) src = c->p;
+  else if (field == SPH_F_C) src = c->c;
+  else if (field >= SPH_F_C11 && field <= SPH_F_C33) src = c->C[field - SPH_F_C11];
+  else if (field == SPH_F_AX) src = c->ax;
+  else if (field == SPH_F_AY) src = c->ay;
+  else if (field == SPH_F_AZ) src = c->az;
+  else if (field == SPH_F_DU) src = c->du;
+  else return fail(c, SPH_ERR_ARG, "unknown field %d", field);
+  if (c->n == 0) return SPH_OK;
+  const cudaMemcpyKind kind = mem == SPH_MEM_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
+  rc = cuda_check(c, cudaMemcpyAsync(dst, src, esz * c->n, kind, c->st), "field copy");
+  if (rc) return rc;
+  rc = cuda_check(c, cudaStreamSynchronize(c->st), "sync");
+  if (!rc) collect_all(c);
+  return rc;
+}
+
+int sph_build_tree(sph_ctx* c) {
+  int rc = check_ready(c, S_PART, "sph_build_tree");
+  if (rc) return rc;
+  return body_tree(c);
+}
+
+int sph_find_neighbors(sph_ctx* c, sph_nbr_stats* stats) {
+  int rc = check_ready(c, S_TREE, "sph_find_neighbors");
+  if (rc) return rc;
+  if ((rc = body_neighbors(c))) return rc;
+  if (!stats) return SPH_OK;
+  rc = sync_scalars(c);
+  fill_stats(c, stats);
+  return rc;
+}
+
+int sph_get_neighbors(sph_ctx* c, int64_t* offsets, int32_t* idx, int64_t idx_cap) {
+  int rc = check_ready(c, S_NBR, "sph_get_neighbors");
+  if (rc) return rc;
+  if (!offsets) return fail(c, SPH_ERR_ARG, "null offsets");
+  const int64_t n = c->n;
+  std::vector<int32_t> nc((size_t)n);
+  if (n) {
+    rc = cuda_check(c, cudaMemcpyAsync(nc.data(), c->nc, 4 * n, cudaMemcpyDeviceToHost, c->st), "nc copy");
+    if (!rc) rc = cuda_check(c, cudaStreamSynchronize(c->st), "sync");
+    if (rc) return rc;
+  }
+  offsets[0] = 0;
+  int maxnc = 0;
+  for (int64_t i = 0; i < n; ++i) {
+    int k = std::min(nc[i], c->cfg.ngmax);
+    maxnc = std::max(maxnc, k);
+    offsets[i + 1] = offsets[i] + k;
+  }
+  if (offsets[n] > idx_cap || (!idx && offsets[n] > 0))
+    return fail(c, SPH_ERR_CAPACITY, "idx_cap %lld < %lld neighbours", (long long)idx_cap, (long long)offsets[n]);
+  if (maxnc == 0) return SPH_OK;
+  std::vector<int32_t> rows((size_t)maxnc * n);
+  rc = cuda_check(c, cudaMemcpy2DAsync(rows.data(), 4 * n, c->nbr, 4 * c->cfg.n_capacity, 4 * n, maxnc, cudaMemcpyDeviceToHost, c->st), "list copy");
+  if (!rc) rc = cuda_check(c, cudaStreamSynchronize(c->st), "sync");
+  if (rc) return rc;
+  for (int64_t i = 0; i < n; ++i)
+    for (int64_t k = 0; k < offsets[i + 1] - offsets[i]; ++k) idx[offsets[i] + k] = rows[(size_t)k * n + i];
+  return SPH_OK;
+}
+
+int sph_density(sph_ctx* c) {
+  int rc = check_ready(c, S_NBR, "sph_density");
+  return rc ? rc : body_simple(c, SPH_PHASE_DENSITY, S_DENS);
+}
+
+int sph_eos(sph_ctx* c) {
+  int rc = check_ready(c, S_DENS, "sph_eos");
+  return rc ? rc : body_simple(c, SPH_PHASE_EOS, S_EOS);
+}
+
+int sph_iad(sph_ctx* c) {
+  int rc = check_ready(c, S_EOS, "sph_iad");
+  return rc ? rc : body_simple(c, SPH_PHASE_IAD, S_IAD);
+}
+
+int sph_momentum_energy(sph_ctx* c) {
+  int rc = check_ready(c, S_IAD, "sph_momentum_energy");
+  return rc ? rc : body_simple(c, SPH_PHASE_MOMENTUM_ENERGY, S_MOM);
+}
+
+int sph_timestep(sph_ctx* c, double* dt) {
+  int rc = check_ready(c, S_MOM, "sph_timestep");
+  if (rc) return rc;
+  if ((rc = body_simple(c, SPH_PHASE_TIMESTEP, S_DT))) return rc;
+  rc = sync_scalars(c);
+  if (dt) *dt = c->h_ds.dt;
+  return rc;
+}
+
+int sph_update(sph_ctx* c) {
+  int rc = check_ready(c, S_DT, "sph_update");
+  return rc ? rc : body_simple(c, SPH_PHASE_UPDATE, S_PART);
+}
+
+int sph_step(sph_ctx* c, sph_step_info* info) {
+  int rc = check_ready(c, S_PART, "sph_step");
+  if (rc) return rc;
+  if ((rc = body_tree(c))) return rc;
+  if ((rc = body_neighbors(c))) return rc;
+  if ((rc = body_simple(c, SPH_PHASE_DENSITY, S_DENS))) return rc;
+  if ((rc = body_simple(c, SPH_PHASE_EOS, S_EOS))) return rc;
+  if ((rc = body_simple(c, SPH_PHASE_IAD, S_IAD))) return rc;
+  if ((rc = body_simple(c, SPH_PHASE_MOMENTUM_ENERGY, S_MOM))) return rc;
+  if ((rc = body_simple(c, SPH_PHASE_TIMESTEP, S_DT))) return rc;
+  // A data error (capacity, singular, box) makes the update meaningless: check
+  // the device status after the update is enqueued (one sync per step).
+  if ((rc = body_simple(c, SPH_PHASE_UPDATE, S_PART))) return rc;
+  rc = sync_scalars(c);
+  if (info) {
+    info->t = c->h_ds.t;
+    info->dt = c->h_ds.dt;
+    fill_stats(c, &info->nbr);
+    info->cell_level = c->h_ds.cell_level;
+    for (int p = 0; p < SPH_NPHASES; ++p) info->phase_ms[p] = c->last_ms[p];
+  }
+  return rc;
+}
+
+int sph_set_clock_policy(sph_ctx* c, int mode, const uint32_t mhz[SPH_NPHASES]) {
+  int rc = check_ready(c, S_INIT, "sph_set_clock_policy");
+  if (rc) return rc;
+  if (mode == SPH_CLOCK_DEFAULT) {
+    if (c->locked_any) c->nvml.reset_sm_clock();
+    c->locked_any = false;
+    c->current_lock = 0;
+    c->clock_mode = SPH_CLOCK_DEFAULT;
+    for (int p = 0; p < SPH_NPHASES; ++p) c->clock_mhz[p] = 0;
+    return SPH_OK;
+  }
+  if (mode != SPH_CLOCK_STATIC && mode != SPH_CLOCK_PER_PHASE) return fail(c, SPH_ERR_ARG, "unknown clock mode %d", mode);
+  if (!mhz) return fail(c, SPH_ERR_ARG, "null mhz");
+  const char* allow = getenv("SPH_ALLOW_CLOCK_CONTROL");
+  if (!allow || strcmp(allow, "1") != 0)
+    return fail(c, SPH_ERR_NO_PERMISSION, "clock control disabled: this host forbids clock changes (set SPH_ALLOW_CLOCK_CONTROL=1 where locking SM clocks is permitted)");
+  if (!c->nvml.ok) return fail(c, SPH_ERR_NOT_SUPPORTED, "NVML unavailable: %s", c->nvml.err);
+  unsigned sup[512];
+  int ns = c->nvml.supported_sm_clocks(sup, 512);
+  if (ns <= 0) return fail(c, SPH_ERR_NOT_SUPPORTED, "no supported graphics clocks reported");
+  unsigned want[SPH_NPHASES];
+  for (int p = 0; p < SPH_NPHASES; ++p) {
+    unsigned r = mode == SPH_CLOCK_STATIC ? mhz[0] : mhz[p];
+    if (r == 0) { want[p] = 0; continue; }
+    unsigned best = sup[0];
+    for (int k = 1; k < ns; ++k)
+      if ((sup[k] > r ? sup[k] - r : r - sup[k]) < (best > r ? best - r : r - best)) best = sup[k];
+    want[p] = best;
+  }
+  unsigned probe = 0;
+  for (int p = 0; p < SPH_NPHASES; ++p) if (want[p]) { probe = want[p]; break; }
+  if (probe) {
+    int lrc = c->nvml.lock_sm_clock(probe);
+    if (lrc == 4) return fail(c, SPH_ERR_NO_PERMISSION, "nvmlDeviceSetGpuLockedClocks: no permission");
+    if (lrc != 0) return fail(c, SPH_ERR_NOT_SUPPORTED, "nvmlDeviceSetGpuLockedClocks: %s", c->nvml.error_string(lrc));
+    c->locked_any = true;
+    c->current_lock = probe;
+  }
+  for (int p = 0; p < SPH_NPHASES; ++p) c->clock_mhz[p] = want[p];
+  c->clock_mode = mode;
+  return SPH_OK;
+}
+
+int sph_energy_report(sph_ctx* c, sph_energy_row* rows, int cap, int* n_rows) {
+  int rc = check_ready(c, S_INIT, "sph_energy_report");
+  if (rc) return rc;
+  if (!rows || cap < SPH_NPHASES) return fail(c, SPH_ERR_ARG, "need room for %d rows", SPH_NPHASES);
+  if (!c->poisoned) {
+    rc = cuda_check(c, cudaStreamSynchronize(c->st), "sync");
+    if (rc) return rc;
+    collect_all(c);
+  }
+  for (int p = 0; p < SPH_NPHASES; ++p) {
+    sph_energy_row& r = rows[p];
+    memset(&r, 0, sizeof(r));
+    r.phase = p;
+    snprintf(r.name, sizeof(r.name), "%s", kPhaseNames[p]);
+    r.calls = c->rows[p].calls;
+    r.seconds = c->rows[p].seconds;
+    r.joules = c->rows[p].joules;
+    r.mean_sm_mhz = c->rows[p].mhz_n ? c->rows[p].mhz_sum / c->rows[p].mhz_n : 0.0;
+    r.locked_mhz = c->rows[p].locked;
+    r.available = c->rows[p].avail ? 1 : 0;
+  }
+  if (n_rows) *n_rows = SPH_NPHASES;
+  return SPH_OK;
+}
+
+int sph_energy_reset(sph_ctx* c) {
+  int rc = check_ready(c, S_INIT, "sph_energy_reset");
+  if (rc) return rc;
+  cudaStreamSynchronize(c->st);
+  collect_all(c);
+  for (int p = 0; p < SPH_NPHASES; ++p) c->rows[p] = PhaseRow();
+  return SPH_OK;
+}
+
+int sph_energy_counter_mj(sph_ctx* c, uint64_t* mj) {
+  if (!c || !mj) return fail(nullptr, SPH_ERR_ARG, "null argument");
+  unsigned long long v;
+  if (!c->nvml.energy_mj(&v)) return fail(c, SPH_ERR_NVML, "NVML energy counter unavailable: %s", c->nvml.err);
+  *mj = v;
+  return SPH_OK;
+}
+
+int sph_set_accounting(sph_ctx* c, int mode) {
+  int rc = check_ready(c, S_INIT, "sph_set_accounting");
+  if (rc) return rc;
+  if (mode != SPH_ACCOUNTING_OFF && mode != SPH_ACCOUNTING_PHASE) return fail(c, SPH_ERR_ARG, "unknown accounting mode %d", mode);
+  c->cfg.accounting = mode;
+  return SPH_OK;
+}
+
+int sph_kernel_launches(int64_t* count) {
+  if (!count) return fail(nullptr, SPH_ERR_ARG, "null count");
+  *count = (int64_t)g_launches.load();
+  return SPH_OK;
+}
+
+int sph_repeat_phase(sph_ctx* c, int phase, int reps, double* ms_per_call, double* joules_per_call) {
+  int need;
+  switch (phase) {
+    case SPH_PHASE_NEIGHBORS: need = S_TREE; break;
+    case SPH_PHASE_DENSITY: need = S_NBR; break;
+    case SPH_PHASE_EOS: need = S_DENS; break;
+    case SPH_PHASE_IAD: need = S_EOS; break;
+    case SPH_PHASE_MOMENTUM_ENERGY: need = S_IAD; break;
+    default: return fail(c, SPH_ERR_ARG, "phase %d is not a pure phase", phase);
+  }
+  int rc = check_ready(c, need, "sph_repeat_phase");
+  if (rc) return rc;
+  if (reps < 1) return fail(c, SPH_ERR_ARG, "reps < 1");
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  rc = cuda_check(c, cudaStreamSynchronize(c->st), "sync");
+  if (rc) return rc;
+  apply_clock(c, phase);
+  unsigned long long e0 = 0, e1 = 0;
+  bool eok = c->nvml.energy_mj(&e0);
+  cudaEventRecord(a, c->st);
+  Fields F = fields(c);
+  for (int r = 0; r < reps; ++r) {
+    switch (phase) {
+      case SPH_PHASE_NEIGHBORS: launch_neighbors(F, c->P, c->st); break;
+      case SPH_PHASE_DENSITY: launch_density(F, c->P, c->st); break;
+      case SPH_PHASE_EOS: launch_eos(F, c->P, c->st); break;
+      case SPH_PHASE_IAD: launch_iad(F, c->P, c->st); break;
+      case SPH_PHASE_MOMENTUM_ENERGY: launch_momentum_energy(F, c->P, c->st); break;
+    }
+  }
+  cudaEventRecord(b, c->st);
+  rc = cuda_check(c, cudaEventSynchronize(b), "repeat");
+  if (!rc) {
+    eok = eok && c->nvml.energy_mj(&e1);
+    float ms = 0;
+    cudaEventElapsedTime(&ms, a, b);
+    if (ms_per_call) *ms_per_call = ms / reps;
+    if (joules_per_call) *joules_per_call = eok ? (double)(e1 - e0) * 1e-3 / reps : -1.0;
+  }
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  return rc;
+}
+
+}  // extern "C"

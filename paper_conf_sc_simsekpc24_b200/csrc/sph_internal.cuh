@@ -1,0 +1,174 @@
+// sph_internal.cuh -- private types and device helpers of libsph.
+//
+// Layout of the data in HBM: every per-particle field is
+// a separate fp64 (or int) array of n_capacity entries inside the caller's arena
+// (structure of arrays, coalesced per field).  Persistent particle state is
+// double-buffered so that the sort's permutation gathers from one buffer into
+// the other.  Neighbour lists are stored column-major, nbr[k * cap + i], so that
+// a warp of 32 consecutive targets reads its k-th neighbours in one 128-B line.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+
+#include "../../include/sph.h"
+
+namespace sph {
+
+constexpr int kNumStateF = 10;  // x y z vx vy vz h m u du_m1 (fp64) + id (int64)
+enum StateField { FX = 0, FY, FZ, FVX, FVY, FVZ, FH, FM, FU, FDUM1 };
+
+// Onesweep radix sort geometry (k_sort.cu).
+constexpr int kSortThreads = 256;
+constexpr int kSortKPT = 16;
+constexpr int kSortTile = kSortThreads * kSortKPT;  // 4096 keys per tile
+constexpr int kRadixBits = 8;
+constexpr int kRadix = 256;
+constexpr int kSortPasses = 8;  // 8 x 8 bits >= 63-bit keys
+
+// Device status bits (reported at the next synchronising call).
+enum DevStatus : int { ST_BOX = 1, ST_CAPACITY = 2, ST_SINGULAR = 4 };
+
+// Small block of device scalars: reductions, the integrator clock and status.
+struct DevScalars {
+  unsigned long long box_min_ord[3];  // order-preserving encodings (open axes)
+  unsigned long long box_max_ord[3];
+  double box_min[3], box_max[3];      // the box used by this step
+  unsigned long long hmax_ord;        // max h (cell level)
+  unsigned long long minhc_ord;       // min h/c (time step)
+  int cell_level;
+  int status;
+  int max_nc, min_nc;
+  unsigned long long total_nc;
+  double t, dt, dt_prev;
+  int first;
+  int pad;
+};
+
+// Everything the kernels need, passed by value.
+struct Fields {
+  int64_t n, cap;
+  double* f[kNumStateF];  // current buffer
+  int64_t* id;
+  uint64_t* key;          // sorted keys (valid after the sort)
+  double *rho, *p, *c, *vol, *prho2;
+  double *wq, *wk;        // per-particle kernel factors (pi/2h)^2 and K/h^3
+  double* C[6];           // 11 12 13 22 23 33
+  double *ax, *ay, *az, *du;
+  int32_t* nc;
+  int32_t* nbr;           // [ngmax][cap]
+  int32_t ngmax;
+  uint32_t* cell_start;   // [8^L + 1]
+  DevScalars* ds;
+};
+
+struct Params {
+  double box_min[3], box_max[3];
+  int periodic[3];
+  int eos;
+  double gamma, cs0, K, ng0, h_cap, k_cour, dt_max_growth;
+  double av_alpha, av_beta, av_eps;
+  int max_cell_level;
+};
+
+// Process-wide count of libsph kernel launches (sph_kernel_launches).
+extern std::atomic<long long> g_launches;
+inline void note_launch(int k = 1) { g_launches.fetch_add(k, std::memory_order_relaxed); }
+
+// ---------------------------------------------------------------- helpers
+__host__ __device__ inline int64_t div_up(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+__device__ __forceinline__ unsigned long long ord_of(double v) {
+  unsigned long long b = (unsigned long long)__double_as_longlong(v);
+  return (b >> 63) ? ~b : (b | 0x8000000000000000ull);
+}
+__device__ __forceinline__ double unord(unsigned long long o) {
+  unsigned long long b = (o >> 63) ? (o & 0x7fffffffffffffffull) : ~o;
+  return __longlong_as_double((long long)b);
+}
+
+// 21-bit Morton spread / compact (x most significant in each triplet).
+__device__ __forceinline__ uint64_t spread3(uint64_t v) {
+  v &= 0x1fffffull;
+  v = (v | v << 32) & 0x1f00000000ffffull;
+  v = (v | v << 16) & 0x1f0000ff0000ffull;
+  v = (v | v << 8) & 0x100f00f00f00f00full;
+  v = (v | v << 4) & 0x10c30c30c30c30c3ull;
+  v = (v | v << 2) & 0x1249249249249249ull;
+  return v;
+}
+__device__ __forceinline__ uint32_t compact3(uint64_t v) {
+  v &= 0x1249249249249249ull;
+  v = (v ^ (v >> 2)) & 0x10c30c30c30c30c3ull;
+  v = (v ^ (v >> 4)) & 0x100f00f00f00f00full;
+  v = (v ^ (v >> 8)) & 0x1f0000ff0000ffull;
+  v = (v ^ (v >> 16)) & 0x1f00000000ffffull;
+  v = (v ^ (v >> 32)) & 0x1fffffull;
+  return (uint32_t)v;
+}
+__device__ __forceinline__ uint64_t morton3(uint32_t ix, uint32_t iy, uint32_t iz) {
+  return (spread3(ix) << 2) | (spread3(iy) << 1) | spread3(iz);
+}
+
+// Minimum image of one raw difference, exactly as the reading of item 4:
+// raw difference first, then one conditional +-L (no FMA anywhere).
+__device__ __forceinline__ double min_image(double dx, double L, double halfL, bool periodic) {
+  if (periodic) {
+    if (dx > halfL) dx = __dsub_rn(dx, L);
+    else if (dx < -halfL) dx = __dadd_rn(dx, L);
+  }
+  return dx;
+}
+
+// sinc(x) for x^2 = t in [0, pi^2]: Taylor series in t to x^26 (14 terms, 13
+// Horner FMAs; coefficients (-1)^k/(2k+1)! rounded to double).  Max abs error
+// 2.9e-16 on [0, pi]; no sqrt/sin per pair.
+__device__ __forceinline__ double sinc_t(double t) {
+  double s = -9.183689863795546e-29;
+  s = fma(s, t, 6.446950284384474e-26);
+  s = fma(s, t, -3.868170170630684e-23);
+  s = fma(s, t, 1.9572941063391263e-20);
+  s = fma(s, t, -8.22063524662433e-18);
+  s = fma(s, t, 2.8114572543455206e-15);
+  s = fma(s, t, -7.647163731819816e-13);
+  s = fma(s, t, 1.6059043836821613e-10);
+  s = fma(s, t, -2.505210838544172e-08);
+  s = fma(s, t, 2.7557319223985893e-06);
+  s = fma(s, t, -0.0001984126984126984);
+  s = fma(s, t, 0.008333333333333333);
+  s = fma(s, t, -0.16666666666666666);
+  s = fma(s, t, 1.0);
+  return s;
+}
+
+// S^6 for the kernel: W = (K/h^3) * S(pi r / 2h)^6, t = r^2 * (pi/2h)^2.
+__device__ __forceinline__ double sinc6_t(double t) {
+  double s = sinc_t(t);
+  double s2 = s * s;
+  return s2 * s2 * s2;
+}
+
+}  // namespace sph
+
+// ---------------------------------------------------------------- launchers
+// (defined in the k_*.cu files; all enqueue on `st`)
+namespace sph {
+void launch_reset_scalars(DevScalars* ds, const Params& P, cudaStream_t st);
+void launch_box_keys(const Fields& F, const Params& P, cudaStream_t st);
+void sort_workspace(int64_t cap, size_t* hist_bytes, size_t* status_bytes);
+cudaError_t launch_sort(const Fields& F, uint64_t* key_in, uint64_t* key_tmp, uint32_t* val_a,
+                        uint32_t* val_b, uint32_t* hist, uint32_t* status, size_t status_bytes,
+                        uint32_t** perm_out, uint64_t** key_out, cudaStream_t st);
+void launch_permute(int64_t n, const uint32_t* perm, double* const* src, double* const* dst,
+                    const int64_t* id_src, int64_t* id_dst, cudaStream_t st);
+void launch_cells(const Fields& F, const Params& P, int level_cap, cudaStream_t st);
+void launch_neighbors(const Fields& F, const Params& P, cudaStream_t st);
+void launch_density(const Fields& F, const Params& P, cudaStream_t st);
+void launch_eos(const Fields& F, const Params& P, cudaStream_t st);
+void launch_iad(const Fields& F, const Params& P, cudaStream_t st);
+void launch_momentum_energy(const Fields& F, const Params& P, cudaStream_t st);
+void launch_timestep(const Fields& F, const Params& P, cudaStream_t st);
+void launch_update(const Fields& F, const Params& P, cudaStream_t st);
+void launch_advance_time(const Fields& F, cudaStream_t st);
+}  // namespace sph

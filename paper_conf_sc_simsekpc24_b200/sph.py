@@ -1,0 +1,331 @@
+"""Thin ctypes binding of libsph (include/sph.h): argument marshalling only.
+
+Every step of the SPH path runs in libsph's CUDA kernels.  PyTorch provides the
+device arena (one uint8 tensor), the CUDA stream and, for multi-GPU runs, the
+process group.  There is no CPU fallback: if libsph.so cannot be loaded, or no
+CUDA device is present, constructing a :class:`Simulation` raises.
+
+Names follow the C ABI: ``Simulation.build_tree`` calls ``sph_build_tree`` etc.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+from . import _build
+
+SPH_OK = 0
+STATUS = {0: "OK", 1: "ERR_ARG", 2: "ERR_STATE", 3: "ERR_CUDA", 4: "ERR_NCCL", 5: "ERR_NVML",
+          6: "ERR_NO_PERMISSION", 7: "ERR_NOT_SUPPORTED", 8: "ERR_CAPACITY", 9: "ERR_HCAP",
+          10: "ERR_SINGULAR", 11: "ERR_BOX"}
+PHASES = ("keys", "sort", "cells", "neighbors", "density", "eos", "iad", "momentum_energy",
+          "timestep", "update")
+NPHASES = len(PHASES)
+FIELDS = ("x", "y", "z", "vx", "vy", "vz", "h", "m", "u", "du_m1", "id", "key", "nc", "rho", "p",
+          "c", "c11", "c12", "c13", "c22", "c23", "c33", "ax", "ay", "az", "du")
+FIELD_ID = {name: k for k, name in enumerate(FIELDS)}
+FIELD_DTYPE = {"id": np.int64, "key": np.uint64, "nc": np.int32}
+MEM_HOST, MEM_DEVICE = 0, 1
+ACCOUNTING_OFF, ACCOUNTING_PHASE = 0, 1
+CLOCK_DEFAULT, CLOCK_STATIC, CLOCK_PER_PHASE = 0, 1, 2
+
+
+class SphError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"{STATUS.get(code, code)}: {msg}")
+        self.code = code
+        self.name = STATUS.get(code, str(code))
+
+
+class Config(C.Structure):
+    _fields_ = [
+        ("n_capacity", C.c_int64), ("box_min", C.c_double * 3), ("box_max", C.c_double * 3),
+        ("periodic", C.c_int32 * 3), ("eos", C.c_int32), ("gamma", C.c_double),
+        ("cs0", C.c_double), ("K", C.c_double), ("ng0", C.c_double), ("ngmax", C.c_int32),
+        ("max_cell_level", C.c_int32), ("h_cap", C.c_double), ("k_cour", C.c_double),
+        ("dt_max_growth", C.c_double), ("dt_first", C.c_double), ("av_alpha", C.c_double),
+        ("av_beta", C.c_double), ("av_eps", C.c_double), ("device", C.c_int32),
+        ("accounting", C.c_int32), ("rank", C.c_int32), ("nranks", C.c_int32),
+        ("reserved", C.c_int32 * 16),
+    ]
+
+
+class NbrStats(C.Structure):
+    _fields_ = [("min_nc", C.c_int32), ("max_nc", C.c_int32), ("mean_nc", C.c_double),
+                ("total", C.c_int64)]
+
+
+class StepInfo(C.Structure):
+    _fields_ = [("t", C.c_double), ("dt", C.c_double), ("nbr", NbrStats),
+                ("cell_level", C.c_int32), ("reserved", C.c_int32),
+                ("phase_ms", C.c_double * NPHASES)]
+
+
+class EnergyRow(C.Structure):
+    _fields_ = [("phase", C.c_int32), ("name", C.c_char * 32), ("calls", C.c_int64),
+                ("seconds", C.c_double), ("joules", C.c_double), ("mean_sm_mhz", C.c_double),
+                ("locked_mhz", C.c_uint32), ("available", C.c_int32)]
+
+
+# Every symbol include/sph.h declares (checked by tests/test_abi.py).
+EXPORTS = ("sph_config_default", "sph_workspace_size", "sph_init", "sph_finalize",
+           "sph_last_error", "sph_phase_name", "sph_set_particles", "sph_set_time",
+           "sph_get_time", "sph_get_n", "sph_get_field", "sph_build_tree", "sph_find_neighbors",
+           "sph_get_neighbors", "sph_density", "sph_eos", "sph_iad", "sph_momentum_energy",
+           "sph_timestep", "sph_update", "sph_step", "sph_set_clock_policy",
+           "sph_energy_report", "sph_energy_reset", "sph_energy_counter_mj", "sph_repeat_phase",
+           "sph_set_accounting", "sph_kernel_launches")
+
+_lib = None
+
+
+def load(build_if_missing: bool = True):
+    """Loads libsph.so (building it in-tree first when missing/stale and nvcc exists)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    path = _build.LIB
+    if build_if_missing and (not os.path.exists(path) or _build.stale()):
+        if os.path.exists(_build.NVCC):
+            _build.build()
+    if not os.path.exists(path):
+        raise RuntimeError(f"libsph.so not found at {path}; run __graft_entry__.build()")
+    L = C.CDLL(path)
+    P, I, I64, D, V = C.c_void_p, C.c_int, C.c_int64, C.c_double, C.c_void_p
+    L.sph_last_error.restype = C.c_char_p
+    L.sph_last_error.argtypes = [P]
+    L.sph_phase_name.restype = C.c_char_p
+    L.sph_phase_name.argtypes = [I]
+    L.sph_config_default.argtypes = [C.POINTER(Config)]
+    L.sph_workspace_size.argtypes = [C.POINTER(Config), C.POINTER(C.c_size_t)]
+    L.sph_init.argtypes = [C.POINTER(Config), V, C.c_size_t, V, C.POINTER(P)]
+    L.sph_finalize.argtypes = [P]
+    L.sph_finalize.restype = None
+    L.sph_set_particles.argtypes = [P, I64] + [V] * 11 + [I]
+    L.sph_set_time.argtypes = [P, D, D, I]
+    L.sph_get_time.argtypes = [P, C.POINTER(D), C.POINTER(D), C.POINTER(I)]
+    L.sph_get_n.argtypes = [P, C.POINTER(I64)]
+    L.sph_get_field.argtypes = [P, I, V, I]
+    for f in ("sph_build_tree", "sph_density", "sph_eos", "sph_iad", "sph_momentum_energy",
+              "sph_update", "sph_energy_reset"):
+        getattr(L, f).argtypes = [P]
+    L.sph_find_neighbors.argtypes = [P, C.POINTER(NbrStats)]
+    L.sph_get_neighbors.argtypes = [P, V, V, I64]
+    L.sph_timestep.argtypes = [P, C.POINTER(D)]
+    L.sph_step.argtypes = [P, C.POINTER(StepInfo)]
+    L.sph_set_clock_policy.argtypes = [P, I, C.POINTER(C.c_uint32)]
+    L.sph_energy_report.argtypes = [P, C.POINTER(EnergyRow), I, C.POINTER(I)]
+    L.sph_energy_counter_mj.argtypes = [P, C.POINTER(C.c_uint64)]
+    L.sph_repeat_phase.argtypes = [P, I, I, C.POINTER(D), C.POINTER(D)]
+    L.sph_set_accounting.argtypes = [P, I]
+    L.sph_kernel_launches.argtypes = [C.POINTER(I64)]
+    _lib = L
+    return L
+
+
+def kernel_launches() -> int:
+    """libsph kernels launched so far by this process (sph_kernel_launches)."""
+    v = C.c_int64()
+    _check(load().sph_kernel_launches(C.byref(v)), None)
+    return int(v.value)
+
+
+def config_from_params(params, n_capacity: int, device: int = 0, accounting: int = 0,
+                       max_cell_level: int = 8) -> Config:
+    """sph_config from the StepParams preset of paper_conf_sc_simsekpc24_b200.ics."""
+    L = load()
+    c = Config()
+    _check(L.sph_config_default(C.byref(c)), None)
+    c.n_capacity = int(n_capacity)
+    c.box_min[:] = [float(v) for v in params.box_min]
+    c.box_max[:] = [float(v) for v in params.box_max]
+    c.periodic[:] = [int(v) for v in params.periodic]
+    c.eos = int(params.eos)
+    for k in ("gamma", "cs0", "K", "ng0", "h_cap", "k_cour", "dt_max_growth", "dt_first",
+              "av_alpha", "av_beta", "av_eps"):
+        setattr(c, k, float(getattr(params, k)))
+    c.ngmax = int(params.ngmax)
+    c.max_cell_level = int(max_cell_level)
+    c.device = int(device)
+    c.accounting = int(accounting)
+    return c
+
+
+def _check(rc, ctx):
+    if rc != SPH_OK:
+        L = load()
+        msg = L.sph_last_error(ctx)
+        raise SphError(rc, msg.decode() if msg else "")
+
+
+def _ptr(a):
+    """Pointer + memory kind of a numpy array (host) or torch tensor (host/device)."""
+    if a is None:
+        return None, MEM_HOST
+    if isinstance(a, np.ndarray):
+        assert a.flags.c_contiguous
+        return a.ctypes.data, MEM_HOST
+    import torch
+    assert isinstance(a, torch.Tensor) and a.is_contiguous()
+    return a.data_ptr(), (MEM_DEVICE if a.is_cuda else MEM_HOST)
+
+
+class Simulation:
+    """One libsph context on one CUDA device (arena + stream owned by torch)."""
+
+    def __init__(self, params, n_capacity: int, device: int = 0, accounting: int = ACCOUNTING_OFF,
+                 stream=None, max_cell_level: int = 8):
+        import torch
+        if not torch.cuda.is_available():
+            raise RuntimeError("libsph needs a CUDA device (no CPU fallback)")
+        self.L = load()
+        self.torch = torch
+        self.device = torch.device("cuda", device)
+        self.cfg = config_from_params(params, n_capacity, device, accounting, max_cell_level)
+        nbytes = C.c_size_t(0)
+        _check(self.L.sph_workspace_size(C.byref(self.cfg), C.byref(nbytes)), None)
+        self.arena_bytes = int(nbytes.value)
+        self.arena = torch.empty(self.arena_bytes + 256, dtype=torch.uint8, device=self.device)
+        base = self.arena.data_ptr()
+        self._base = (base + 255) // 256 * 256
+        self.stream = stream if stream is not None else torch.cuda.Stream(device=self.device)
+        self.ctx = C.c_void_p()
+        _check(self.L.sph_init(C.byref(self.cfg), C.c_void_p(self._base), C.c_size_t(self.arena_bytes),
+                               C.c_void_p(self.stream.cuda_stream), C.byref(self.ctx)), None)
+        self.n = 0
+
+    # ---------------------------------------------------------------- lifetime
+    def finalize(self):
+        if self.ctx:
+            self.L.sph_finalize(self.ctx)
+            self.ctx = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.finalize()
+        except Exception:
+            pass
+
+    def _ok(self, rc):
+        _check(rc, self.ctx)
+
+    # ---------------------------------------------------------------- I/O
+    def set_particles(self, state: dict):
+        """state: x y z vx vy vz h m u [du_m1] [id] as numpy (host) or torch (cuda) arrays."""
+        n = int(len(state["x"]))
+        ptrs = []
+        mem = None
+        for k in ("x", "y", "z", "vx", "vy", "vz", "h", "m", "u", "du_m1", "id"):
+            a = state.get(k)
+            if isinstance(a, np.ndarray):
+                want = np.int64 if k == "id" else np.float64
+                if a.dtype != want or not a.flags.c_contiguous:
+                    a = np.ascontiguousarray(a, dtype=want)
+                    state = dict(state)
+                    state[k] = a
+            p, m = _ptr(a)
+            if a is not None:
+                if mem is None:
+                    mem = m
+                elif mem != m:
+                    raise ValueError("all arrays must live in the same memory kind")
+            ptrs.append(C.c_void_p(p) if p is not None else None)
+        self._keep = state  # host buffers must outlive the async copies
+        self._ok(self.L.sph_set_particles(self.ctx, n, *ptrs, mem if mem is not None else MEM_HOST))
+        self.n = n
+
+    def set_time(self, t: float, dt_prev: float, first_step: bool):
+        self._ok(self.L.sph_set_time(self.ctx, t, dt_prev, 1 if first_step else 0))
+
+    def get_time(self):
+        t, d, f = C.c_double(), C.c_double(), C.c_int()
+        self._ok(self.L.sph_get_time(self.ctx, C.byref(t), C.byref(d), C.byref(f)))
+        return t.value, d.value, bool(f.value)
+
+    def get_field(self, name: str, out=None):
+        dt = FIELD_DTYPE.get(name, np.float64)
+        if out is None:
+            out = np.empty(self.n, dtype=dt)
+        p, mem = _ptr(out)
+        self._ok(self.L.sph_get_field(self.ctx, FIELD_ID[name], C.c_void_p(p), mem))
+        return out
+
+    def get_state(self):
+        return {k: self.get_field(k) for k in ("x", "y", "z", "vx", "vy", "vz", "h", "m", "u",
+                                               "du_m1", "id")}
+
+    # ---------------------------------------------------------------- hot path
+    def build_tree(self):
+        self._ok(self.L.sph_build_tree(self.ctx))
+
+    def find_neighbors(self, stats: bool = True):
+        s = NbrStats()
+        self._ok(self.L.sph_find_neighbors(self.ctx, C.byref(s) if stats else None))
+        return {"min_nc": s.min_nc, "max_nc": s.max_nc, "mean_nc": s.mean_nc, "total": s.total}
+
+    def get_neighbors(self):
+        off = np.zeros(self.n + 1, dtype=np.int64)
+        nc = self.get_field("nc")
+        total = int(np.minimum(nc, self.cfg.ngmax).sum())
+        idx = np.zeros(max(total, 1), dtype=np.int32)
+        self._ok(self.L.sph_get_neighbors(self.ctx, C.c_void_p(off.ctypes.data),
+                                          C.c_void_p(idx.ctypes.data), total))
+        return off, idx[:total]
+
+    def density(self):
+        self._ok(self.L.sph_density(self.ctx))
+
+    def eos(self):
+        self._ok(self.L.sph_eos(self.ctx))
+
+    def iad(self):
+        self._ok(self.L.sph_iad(self.ctx))
+
+    def momentum_energy(self):
+        self._ok(self.L.sph_momentum_energy(self.ctx))
+
+    def timestep(self) -> float:
+        d = C.c_double()
+        self._ok(self.L.sph_timestep(self.ctx, C.byref(d)))
+        return d.value
+
+    def update(self):
+        self._ok(self.L.sph_update(self.ctx))
+
+    def step(self):
+        info = StepInfo()
+        self._ok(self.L.sph_step(self.ctx, C.byref(info)))
+        return {"t": info.t, "dt": info.dt, "min_nc": info.nbr.min_nc, "max_nc": info.nbr.max_nc,
+                "mean_nc": info.nbr.mean_nc, "cell_level": info.cell_level,
+                "phase_ms": {PHASES[p]: info.phase_ms[p] for p in range(NPHASES)}}
+
+    # ---------------------------------------------------------------- energy / clocks
+    def set_clock_policy(self, mode: int, mhz=None):
+        arr = (C.c_uint32 * NPHASES)(*([0] * NPHASES if mhz is None else [int(v) for v in mhz]))
+        self._ok(self.L.sph_set_clock_policy(self.ctx, mode, arr))
+
+    def energy_report(self):
+        rows = (EnergyRow * NPHASES)()
+        n = C.c_int()
+        self._ok(self.L.sph_energy_report(self.ctx, rows, NPHASES, C.byref(n)))
+        return [{"phase": r.phase, "name": r.name.decode(), "calls": r.calls, "seconds": r.seconds,
+                 "joules": r.joules if r.available else None, "mean_sm_mhz": r.mean_sm_mhz,
+                 "locked_mhz": r.locked_mhz} for r in rows[: n.value]]
+
+    def energy_reset(self):
+        self._ok(self.L.sph_energy_reset(self.ctx))
+
+    def energy_counter_mj(self):
+        v = C.c_uint64()
+        rc = self.L.sph_energy_counter_mj(self.ctx, C.byref(v))
+        return int(v.value) if rc == SPH_OK else None
+
+    def set_accounting(self, mode: int):
+        self._ok(self.L.sph_set_accounting(self.ctx, mode))
+
+    def repeat_phase(self, phase: str, reps: int):
+        ms, j = C.c_double(), C.c_double()
+        self._ok(self.L.sph_repeat_phase(self.ctx, PHASES.index(phase), reps, C.byref(ms), C.byref(j)))
+        return ms.value, (j.value if j.value >= 0 else None)

@@ -1,0 +1,188 @@
+"""GPU (libsph through the C ABI) vs the CPU oracle on identical seeded inputs.
+
+Bars (BASELINE.json north_star): Morton order and neighbour lists bit-exact;
+fp64 fields within 1e-10 after one step and 1e-8 after ten, in the metric of
+DESIGN.md section 3 (|err| <= tol * sum_j |term_j| for the neighbour sums)."""
+import hashlib
+
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_sc_simsekpc24_b200 import ics
+from parity import (TOL_1STEP, TOL_10STEP, compare_state, compare_sums, gpu_pipeline, new_sim)
+
+pytestmark = pytest.mark.gpu
+
+
+def _workloads():
+    w_open = ics.random_box(3001, seed=7, periodic=False)
+    w_rand = ics.random_box(5003, seed=8, periodic=True)   # ragged: not a multiple of any tile
+    w_turb = ics.turbulence(20)
+    w_sedov = ics.sedov(16)
+    w_noh = ics.noh(14)
+    return {"sedov16": w_sedov, "turbulence20": w_turb, "random_periodic": w_rand,
+            "random_open": w_open, "noh14": w_noh}
+
+
+WORKLOADS = _workloads()
+
+
+@pytest.fixture(scope="module", params=list(WORKLOADS))
+def case(request):
+    w = WORKLOADS[request.param]
+    st, o = oracle.step({k: v.copy() for k, v in w.state.items()}, w.params, w.params.dt_first, True)
+    sim = new_sim(w)
+    g = gpu_pipeline(sim)
+    return request.param, w, sim, g, st, o
+
+
+def test_morton_order_bit_exact(case):
+    name, w, sim, g, st, o = case
+    assert np.array_equal(g["key"], o["keys"]), "sorted Morton keys"
+    assert np.array_equal(g["id"], o["pre"]["id"]), "Morton order (id sequence)"
+    for k in ("x", "y", "z", "h", "m", "u"):
+        assert np.array_equal(g[k], o["pre"][k]), f"permuted {k}"
+
+
+def test_neighbour_lists_bit_exact(case):
+    name, w, sim, g, st, o = case
+    nb = o["nb"]
+    assert np.array_equal(g["nc"], nb.nc)
+    off, idx = sim.get_neighbors()
+    assert np.array_equal(off, nb.offsets)
+    assert np.array_equal(idx.astype(np.int64), nb.idx)
+    s = g["stats"]
+    assert s["max_nc"] == nb.nc.max() and s["min_nc"] == nb.nc.min() and s["total"] == nb.nc.sum()
+
+
+def test_neighbour_sums_within_tolerance(case):
+    name, w, sim, g, st, o = case
+    compare_sums(g, o, TOL_1STEP)
+
+
+def test_step_parity_one_step(case):
+    name, w, sim, g, st, o = case
+    dt = sim.timestep()
+    assert dt == o["dt"], "dt is bit-exact (min of IEEE h/c, same operations)"
+    sim.update()
+    t, dtp, first = sim.get_time()
+    assert t == dt and dtp == dt and not first
+    gs = sim.get_state()
+    assert np.array_equal(gs["id"], st["id"])
+    L = float(np.max(np.array(o["bmax"]) - np.array(o["bmin"])))
+    compare_state(gs, st, L, TOL_1STEP)
+
+
+def test_ten_steps_sedov16():
+    w = ics.sedov(16)
+    s = {k: v.copy() for k, v in w.state.items()}
+    dt = w.params.dt_first
+    sim = new_sim(w)
+    for k in range(10):
+        s, out = oracle.step(s, w.params, dt, k == 0)
+        dt = out["dt"]
+        info = sim.step()
+        assert info["dt"] == pytest.approx(dt, rel=1e-12)
+    gs = sim.get_state()
+    assert np.array_equal(gs["id"], s["id"])
+    compare_state(gs, s, 1.0, TOL_10STEP, "10 steps: ")
+
+
+def test_ten_steps_turbulence():
+    w = ics.turbulence(14)
+    s = {k: v.copy() for k, v in w.state.items()}
+    dt = w.params.dt_first
+    sim = new_sim(w)
+    for k in range(10):
+        s, out = oracle.step(s, w.params, dt, k == 0)
+        dt = out["dt"]
+        sim.step()
+    gs = sim.get_state()
+    assert np.array_equal(gs["id"], s["id"])
+    compare_state(gs, s, 1.0, TOL_10STEP, "10 steps: ")
+
+
+def test_deterministic_bitwise():
+    w = ics.turbulence(16)
+    hashes = set()
+    for _ in range(3):
+        sim = new_sim(w)
+        for _ in range(2):
+            sim.step()
+        h = hashlib.sha256()
+        for k, v in sim.get_state().items():
+            h.update(v.tobytes())
+        hashes.add(h.hexdigest())
+        sim.finalize()
+    assert len(hashes) == 1
+
+
+def test_empty_input():
+    w = ics.sedov(4)
+    from paper_conf_sc_simsekpc24_b200 import sph
+    sim = sph.Simulation(w.params, n_capacity=64)
+    sim.set_particles({k: v[:0] for k, v in w.state.items()})
+    sim.set_time(0.0, 1e-3, True)
+    info = sim.step()
+    assert info["dt"] == pytest.approx(1.1e-3, rel=1e-15)
+
+
+def test_lone_particle_is_singular():
+    from paper_conf_sc_simsekpc24_b200 import sph
+    w = ics.random_box(1, seed=3)
+    sim = new_sim(w, cap=16)
+    with pytest.raises(sph.SphError) as e:
+        sim.step()
+    assert e.value.name == "ERR_SINGULAR"
+
+
+def test_capacity_error_reports_needed_size():
+    from paper_conf_sc_simsekpc24_b200 import sph
+    w = ics.sedov(10)
+    w.params.ngmax = 50
+    sim = new_sim(w)
+    sim.build_tree()
+    with pytest.raises(sph.SphError) as e:
+        sim.find_neighbors()
+    assert e.value.name == "ERR_CAPACITY" and "92" in str(e.value)
+
+
+def test_degenerate_open_box():
+    from paper_conf_sc_simsekpc24_b200 import sph
+    w = ics.random_box(100, seed=3, periodic=False)
+    w.state["z"][:] = 0.25
+    sim = new_sim(w)
+    sim.build_tree()
+    with pytest.raises(sph.SphError) as e:
+        sim.find_neighbors()
+    assert e.value.name == "ERR_BOX"
+
+
+def test_stage_machine():
+    from paper_conf_sc_simsekpc24_b200 import sph
+    w = ics.sedov(8)
+    sim = new_sim(w)
+    with pytest.raises(sph.SphError) as e:
+        sim.density()
+    assert e.value.name == "ERR_STATE"
+    sim.build_tree()
+    with pytest.raises(sph.SphError):
+        sim.iad()
+    with pytest.raises(sph.SphError) as e:
+        sim.set_particles({k: v[: 10 ** 6] for k, v in ics.sedov(12).state.items()})
+    assert e.value.name == "ERR_CAPACITY"
+
+
+def test_host_and_device_inputs_agree():
+    import torch
+    w = ics.turbulence(12)
+    a = new_sim(w)
+    a.step()
+    b = new_sim(w)
+    dev = {k: torch.from_numpy(np.ascontiguousarray(v)).cuda() for k, v in w.state.items()}
+    b.set_particles(dev)
+    b.set_time(0.0, w.params.dt_first, True)
+    b.step()
+    for k in ("x", "vx", "u", "h"):
+        assert np.array_equal(a.get_field(k), b.get_field(k))
