@@ -176,7 +176,8 @@ def random_box(n: int, seed: int = 0, periodic: bool = True, h: float | None = N
     x, y, z = (rng.uniform(-0.5, 0.5, n) for _ in range(3))
     vx, vy, vz = (rng.normal(0.0, v_scale, n) for _ in range(3))
     u = rng.uniform(0.5, 1.5, n)
-    p = StepParams(periodic=(1, 1, 1) if periodic else (0, 0, 0), eos=0, dt_first=1e-4,
+    # Poisson positions: nc spreads far wider than on a lattice (max ~ 1.7 x mean)
+    p = StepParams(periodic=(1, 1, 1) if periodic else (0, 0, 0), eos=0, dt_first=1e-4, ngmax=256,
                    h_cap=0.25 if periodic else 1e300)
     hh = h if h is not None else h_initial(n, p.ng0)
     hv = hh * rng.uniform(0.9, 1.1, n)
