@@ -62,6 +62,8 @@ struct sph_ctx {
   double *rho, *p, *c, *vol, *prho2, *wq, *wk, *C[6], *ax, *ay, *az, *du;
   int32_t *nc, *nbr;
   uint32_t* cell_start;
+  float4* pos4;
+  Rec4 *rec_d, *rec_i, *rec_m;
   uint32_t *sort_hist, *sort_status;
   size_t status_bytes;
   DevScalars* ds;
@@ -124,6 +126,10 @@ Fields fields(sph_ctx* c) {
   F.ax = c->ax; F.ay = c->ay; F.az = c->az; F.du = c->du;
   F.nc = c->nc; F.nbr = c->nbr; F.ngmax = c->cfg.ngmax;
   F.cell_start = c->cell_start;
+  F.pos4 = c->pos4;
+  F.rec_d = c->rec_d;
+  F.rec_i = c->rec_i;
+  F.rec_m = c->rec_m;
   F.ds = c->ds;
   return F;
 }
@@ -250,10 +256,10 @@ int body_tree(sph_ctx* c) {
   cudaError_t e = launch_sort(F, c->keyA, c->keyB, c->valA, c->valB, c->sort_hist, c->sort_status,
                               c->status_bytes, &perm, &ksorted, c->st);
   if ((rc = cuda_check(c, e, "sort"))) return rc;
-  const int nxt = c->cur ^ 1;
-  launch_permute(c->n, perm, c->state[c->cur], c->state[nxt], c->ids[c->cur], c->ids[nxt], c->st);
-  c->cur = nxt;
+  const int prv = c->cur;
+  c->cur ^= 1;
   c->key_sorted = ksorted;
+  launch_permute(fields(c), perm, c->state[prv], c->ids[prv], c->st);
   if ((rc = phase_end(c, SPH_PHASE_SORT))) return rc;
 
   if ((rc = phase_begin(c, SPH_PHASE_CELLS))) return rc;
@@ -379,6 +385,16 @@ static size_t layout(const sph_config* cfg, char* base, sph_ctx* c) {
   for (int e = 0; e < 6; ++e) {
     char* p = take(D);
     if (c) c->C[e] = (double*)p;
+  }
+  char* p4 = take(sizeof(float4) * cap);
+  char* rd = take(sizeof(Rec4) * cap);
+  char* ri = take(sizeof(Rec4) * cap);
+  char* rm = take(sizeof(Rec4) * kRecM * cap);
+  if (c) {
+    c->pos4 = (float4*)p4;
+    c->rec_d = (Rec4*)rd;
+    c->rec_i = (Rec4*)ri;
+    c->rec_m = (Rec4*)rm;
   }
   char* ncp = take(sizeof(int32_t) * cap);
   char* nbp = take(sizeof(int32_t) * cap * (size_t)cfg->ngmax);

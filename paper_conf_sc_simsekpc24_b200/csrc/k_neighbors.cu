@@ -1,24 +1,40 @@
 // k_neighbors.cu -- phases CELLS and NEIGHBORS (items 3-4 of DESIGN.md section 3).
 //
-// CELLS: a uniform grid over the box at level L (2^L cells per axis) whose cells
-// are exactly the level-L octree nodes of the Morton curve, so every cell is one
-// contiguous range of the sorted particles: cell_start[c] .. cell_start[c+1] with
-// c = key >> 3(21-L).  L is the finest level <= cap whose cell side is >= 2 h_max
-// on every axis (decided on the device from the exact h_max of phase KEYS, so no
-// host round trip).  HBM-bound: 8 B/particle read (key) + 4 B/cell written.
+// CELLS: a uniform grid whose cells are exactly the level-L octree nodes of the
+// Morton curve, so every cell is one contiguous range of the sorted particles:
+// cell_start[c] .. cell_start[c+1], c = key >> 3(21-L).  Two levels are used: a
+// coarse level Lc (the finest with cell side >= 2 h_max on every axis, so a
+// target's neighbours lie in the 27 coarse cells around it) and the fine table
+// level Lf = Lc + 1 (each coarse cell = 8 consecutive fine cells).  Lc is decided
+// on the device from the exact h_max of phase KEYS (no host round trip).
+// HBM-bound: 8 B/particle read (key) + 4 B/fine cell written.
 //
-// NEIGHBORS: one thread per target i.  The 27 stencil cells around i's cell
-// (periodic wrap or clipped at open faces, duplicates removed when 2^L < 3) are
-// sorted by Morton index with a register bitonic network, so candidates are
-// visited -- and neighbours appended -- in ascending particle index, the
-// oracle's order.  The predicate is the oracle's exactly: raw difference,
-// conditional +-L, d2 = (dx*dx + dy*dy) + dz*dz with every operation rounded
-// (__dmul_rn/__dadd_rn: no FMA contraction), d2 < (2h_i)(2h_i).  Consecutive
-// targets sit in the same few cells, so a warp's candidate loads are mostly
-// broadcasts from L1.  Lists are stored column-major nbr[k*cap + i].
-// Bound: FP64 pipe (the exact predicate costs ~15 DP ops per candidate; ~27 x
-// 30 candidates per target).  Algorithmic bytes: x, y, z, h in (32 B), nc out
-// (4 B) and the list out (4 B per neighbour).
+// NEIGHBORS: warp-cooperative.  A warp takes 32 consecutive (Morton-sorted)
+// targets, which sit in a small region of space, and walks ONE candidate stream
+// for all of them (no per-lane divergence):
+//  1. the coarse cells covering the targets' 2h spheres (<= 128 cells; periodic
+//     wrap, clipped at open faces) are ranked by Morton index, so the stream is in
+//     ascending particle index -- every lane's neighbours come out ascending, the
+//     oracle's order.  A warp whose targets straddle a large Morton jump (box >
+//     128 cells) is split into halves, quarters, ... processed one after another;
+//  2. per coarse cell, the fine children no lane's sphere reaches are culled
+//     (warp OR of per-lane masks); the runs of needed children form a run list
+//     (cell_start loads issued by all lanes in parallel, warp prefix sum);
+//  3. the runs are streamed 32 candidates at a time (one coalesced 128-bit pos4
+//     load per lane, prefetched one chunk ahead, staged in shared memory) and every
+//     lane tests every candidate two at a time with packed f32x2 arithmetic
+//     (FADD2/FFMA2) against an outer and an inner radius that bracket 2h_i by a
+//     rigorous bound on the fp32 rounding (reading 14):
+//     outside -> rejected, inside -> accepted; only the thin shell in between
+//     (~1e-4 of candidates) runs the oracle's exact fp64 predicate (raw
+//     difference, conditional +-L, d2 = (dx*dx + dy*dy) + dz*dz rounded per
+//     operation, d2 < (2h_i)(2h_i)).  Every decision equals the exact predicate's:
+//     the neighbour sets are bit-identical to brute force;
+//  4. hits are appended with predicated stores in candidate order.
+// Lists are stored column-major nbr[k*cap + i].
+// Bound: issue (fp32 + integer work per candidate test, ~880 candidates per
+// warp of 32 targets at 100 neighbours).  Algorithmic bytes: pos4, x, y, z, h in
+// (48 B), nc out (4 B), the list out (4 B per neighbour).
 #include <algorithm>
 
 #include "sph_internal.cuh"
@@ -27,7 +43,7 @@ namespace sph {
 
 __global__ void cell_level_kernel(DevScalars* ds, int level_cap) {
   double hmax = unord(ds->hmax_ord);
-  int L = level_cap;
+  int L = level_cap - 1;  // coarse level; the table is one level finer
   while (L > 0) {
     bool ok = true;
     for (int a = 0; a < 3; ++a) {
@@ -37,7 +53,7 @@ __global__ void cell_level_kernel(DevScalars* ds, int level_cap) {
     if (ok) break;
     --L;
   }
-  ds->cell_level = L;
+  ds->cell_level = L + 1;
 }
 
 __global__ void __launch_bounds__(256) cells_kernel(int64_t n, const uint64_t* __restrict__ key,
@@ -57,108 +73,466 @@ __global__ void __launch_bounds__(256) cells_kernel(int64_t n, const uint64_t* _
 
 void launch_cells(const Fields& F, const Params& P, int level_cap, cudaStream_t st) {
   (void)P;
-  cell_level_kernel<<<1, 1, 0, st>>>(F.ds, level_cap); note_launch();
+  cell_level_kernel<<<1, 1, 0, st>>>(F.ds, level_cap);
+  note_launch();
   if (F.n > 0) {
     cells_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F.n, F.key, F.ds, F.cell_start);
     note_launch();
   }
 }
 
-template <int N>
-__device__ __forceinline__ void bitonic_sort(uint32_t (&a)[N]) {
-#pragma unroll
-  for (int k = 2; k <= N; k <<= 1)
-#pragma unroll
-    for (int j = k >> 1; j > 0; j >>= 1)
-#pragma unroll
-      for (int i = 0; i < N; ++i) {
-        const int l = i ^ j;
-        if (l > i) {
-          uint32_t x = a[i], y = a[l];
-          uint32_t lo = min(x, y), hi = max(x, y);
-          if ((i & k) == 0) {
-            a[i] = lo;
-            a[l] = hi;
-          } else {
-            a[i] = hi;
-            a[l] = lo;
-          }
-        }
-      }
-}
-
 constexpr int kNbrThreads = 128;
+constexpr int kNbrWarps = kNbrThreads / 32;
+constexpr int kMaxWarpCells = 128;
 constexpr uint32_t kNoCell = 0xffffffffu;
 
-__global__ void __launch_bounds__(kNbrThreads) neighbors_kernel(Fields F, Params P) {
-  __shared__ uint32_t s_cells[27][kNbrThreads];
-  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  const bool active = i < F.n;
-  int cnt = 0;
-  if (active) {
-    const DevScalars* ds = F.ds;
-    const int L = ds->cell_level;
-    const int nside = 1 << L;
-    const uint64_t key = F.key[i];
-    const int cx = (int)(compact3(key >> 2) >> (21 - L));
-    const int cy = (int)(compact3(key >> 1) >> (21 - L));
-    const int cz = (int)(compact3(key) >> (21 - L));
-    uint32_t ck[32];
+// Per-target constants of the search.
+struct Target {
+  double x, y, z, r2max;  // fp64 position and (2h)^2 for the exact predicate
+  float m[3];             // fp32 position relative to box_min
+  float r_out2, r_in2;    // fp32 bracket of (2h)^2
+  float rc;               // culling radius
+};
+
+struct Box {
+  double L[3], H[3];
+  float Lf[3], side[3];    // box length, coarse cell side (fp32)
+  bool per[3];
+  int nside;               // coarse cells per axis
+  int Lc;
+};
+
+__device__ __forceinline__ Target make_target(const Fields& F, const Box& B, int64_t i, bool active) {
+  Target t;
+  if (!active) {
+    t.x = t.y = t.z = 0.0;
+    t.r2max = -1.0;
+    t.m[0] = t.m[1] = t.m[2] = 0.f;
+    t.r_out2 = -1.f;  // rejects every candidate
+    t.r_in2 = -1.f;
+    t.rc = -1.f;
+    return t;
+  }
+  t.x = F.f[FX][i];
+  t.y = F.f[FY][i];
+  t.z = F.f[FZ][i];
+  const double h = F.f[FH][i];
+  const double r = 2.0 * h;
+  t.r2max = r * r;
+  const double Lmax = fmax(B.L[0], fmax(B.L[1], B.L[2]));
+  // fp32 rounding bound per axis: pos4 conversion, shift by +-L and the
+  // difference each add <= 2^-24 L  ->  E = 8 * 2^-24 * L (reading 14)
+  const double E = 8.0 * 5.9604644775390625e-08 * Lmax;
+  const double sE = 1.7320508075688772 * E;
+  t.r_out2 = __double2float_ru((r + sE) * (r + sE) * (1.0 + 1e-6));
+  t.r_in2 = r > sE ? __double2float_rd((r - sE) * (r - sE) * (1.0 - 1e-6)) : -1.0f;
+  t.rc = __double2float_ru((r + sE + 4.0 * E) * (1.0 + 1e-6));
+  const float4 me = F.pos4[i];
+  t.m[0] = me.x;
+  t.m[1] = me.y;
+  t.m[2] = me.z;
+  return t;
+}
+
+// The exact predicate of item 4 (only reached for the thin fp32 shell).
+__device__ __forceinline__ bool exact_in(const Fields& F, const Box& B, const Target& t, uint32_t j) {
+  double ex = min_image(__dsub_rn(t.x, F.f[FX][j]), B.L[0], B.H[0], B.per[0]);
+  double ey = min_image(__dsub_rn(t.y, F.f[FY][j]), B.L[1], B.H[1], B.per[1]);
+  double ez = min_image(__dsub_rn(t.z, F.f[FZ][j]), B.L[2], B.H[2], B.per[2]);
+  return __dadd_rn(__dadd_rn(__dmul_rn(ex, ex), __dmul_rn(ey, ey)), __dmul_rn(ez, ez)) < t.r2max;
+}
+
+// Per-axis squared distances from the target to the lower/upper child slab of
+// the coarse cell at unwrapped coordinate u (0 when the axis is "full": the
+// warp's range covers the whole periodic axis and the image is resolved per
+// candidate).
+__device__ __forceinline__ void slab_d2(const Box& B, const Target& t, int a, int u, bool full,
+                                        float& d0, float& d1) {
+  if (full) {
+    d0 = d1 = 0.f;
+    return;
+  }
+  const float lo = (float)u * B.side[a];
+  const float half = 0.5f * B.side[a];
+  const float m = t.m[a];
+  float a0 = fmaxf(fmaxf(lo - m, m - (lo + half)), 0.f);
+  float a1 = fmaxf(fmaxf(lo + half - m, m - (lo + B.side[a])), 0.f);
+  d0 = a0 * a0;
+  d1 = a1 * a1;
+}
+
+// Packed fp32x2 arithmetic (FADD2/FMUL2/FFMA2 on sm_100a): two candidates per
+// instruction in the neighbour test.  Each lane is IEEE round-to-nearest.
+__device__ __forceinline__ unsigned long long pack2(float lo, float hi) {
+  return ((unsigned long long)__float_as_uint(hi) << 32) | (unsigned long long)__float_as_uint(lo);
+}
+__device__ __forceinline__ void unpack2(unsigned long long v, float& lo, float& hi) {
+  lo = __uint_as_float((uint32_t)v);
+  hi = __uint_as_float((uint32_t)(v >> 32));
+}
+__device__ __forceinline__ unsigned long long sub2(unsigned long long a, unsigned long long b) {
+  unsigned long long d;
+  asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+__device__ __forceinline__ unsigned long long mul2(unsigned long long a, unsigned long long b) {
+  unsigned long long d;
+  asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+__device__ __forceinline__ unsigned long long fma2(unsigned long long a, unsigned long long b,
+                                                   unsigned long long c) {
+  unsigned long long d;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
+  return d;
+}
+
+
+constexpr int kMaxRuns = 4 * kMaxWarpCells;  // <= 4 runs of children per cell
+
+struct WarpSmem {
+  uint32_t cell[kMaxWarpCells];   // sorted coarse cell keys
+  uint32_t ucs[kMaxWarpCells];    // their unwrapped coordinates (biased, packed)
+  uint32_t mask[kMaxWarpCells];   // children any lane needs
+  uint32_t run_start[kMaxRuns];   // first particle of each run
+  uint32_t run_pos[kMaxRuns + 1]; // stream position of each run (exclusive prefix)
+  uint32_t run_cell[kMaxRuns];    // index of the run's coarse cell
+  // staged chunk of 32 candidates (image-shifted fp32 position, SoA so that two
+  // consecutive candidates are one 64-bit load for the packed f32x2 math)
+  alignas(16) float cx[32];
+  alignas(16) float cy[32];
+  alignas(16) float cz[32];
+  uint32_t cj[32];
+};
+
+// Butterfly min/max within aligned groups of g lanes (g a power of two).
+__device__ __forceinline__ int group_min(int v, int g) {
+  for (int off = 1; off < g; off <<= 1) v = min(v, __shfl_xor_sync(0xffffffffu, v, off));
+  return v;
+}
+__device__ __forceinline__ int group_max(int v, int g) {
+  for (int off = 1; off < g; off <<= 1) v = max(v, __shfl_xor_sync(0xffffffffu, v, off));
+  return v;
+}
+
+// Coarse-cell box of a group of targets: [lo, lo + ext) per axis; "full" axes
+// cover the whole periodic axis (images then resolved per candidate).
+struct GroupBox {
+  int lo[3], ext[3];
+  bool full[3];
+  int T;
+};
+
+__device__ __forceinline__ GroupBox group_box(const Box& B, const Target& t, bool member, int g) {
+  GroupBox G;
+  G.T = 1;
 #pragma unroll
-    for (int s = 0; s < 32; ++s) {
-      if (s >= 27) {
-        ck[s] = kNoCell;
-        continue;
+  for (int a = 0; a < 3; ++a) {
+    int l = member ? (int)floorf((t.m[a] - t.rc) / B.side[a]) : 0x3fffffff;
+    int h = member ? (int)floorf((t.m[a] + t.rc) / B.side[a]) : -0x3fffffff;
+    l = group_min(l, g);
+    h = group_max(h, g);
+    G.full[a] = false;
+    if (B.per[a]) {
+      if (h - l + 1 >= B.nside) {
+        l = 0;
+        h = B.nside - 1;
+        G.full[a] = true;
       }
-      int o[3] = {s / 9 - 1, (s / 3) % 3 - 1, s % 3 - 1};
-      int c[3] = {cx + o[0], cy + o[1], cz + o[2]};
-      bool ok = true;
+    } else {
+      l = max(l, 0);
+      h = min(h, B.nside - 1);
+    }
+    G.lo[a] = l;
+    G.ext[a] = max(h - l + 1, 0);
+    G.T *= G.ext[a];
+  }
+  return G;
+}
+
+// The group's candidate stream (see the file header, steps 1-4).  Lanes with
+// t.rc < 0 take part in the warp collectives but test nothing.
+template <bool kFull>
+__device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const Target& t, int64_t i,
+                                          const GroupBox& G, WarpSmem& S, int lane, int& cnt) {
+  const int n = B.nside, nm = n - 1;
+  const int T = G.T;
+  const int64_t cap = F.cap;
+  const int ngmax = F.ngmax;
+  const float rc2 = t.rc * t.rc;
+  const bool live = t.rc >= 0.f;
+  // ---- 1. rank the T cells by Morton key (keys are distinct)
+  {
+    uint32_t mykey[kMaxWarpCells / 32], myuc[kMaxWarpCells / 32], rank[kMaxWarpCells / 32];
 #pragma unroll
-      for (int a = 0; a < 3; ++a) {
-        if (c[a] < 0 || c[a] >= nside) {
-          if (P.periodic[a]) c[a] = (c[a] + nside) % nside;
-          else ok = false;
+    for (int r = 0; r < kMaxWarpCells / 32; ++r) {
+      const int tt = r * 32 + lane;
+      mykey[r] = kNoCell;
+      myuc[r] = 0;
+      rank[r] = 0;
+      if (tt < T) {
+        const int q = tt / G.ext[2];
+        const int uc[3] = {G.lo[0] + q / G.ext[1], G.lo[1] + q % G.ext[1], G.lo[2] + tt - q * G.ext[2]};
+        // wrap (n is a power of two; open axes are clipped to [0, n) already)
+        mykey[r] = (uint32_t)morton3((uint32_t)(uc[0] & nm), (uint32_t)(uc[1] & nm), (uint32_t)(uc[2] & nm));
+        // unwrapped coordinates (>= -2), biased by +4, 10 bits each
+        myuc[r] = (uint32_t)(uc[0] + 4) | ((uint32_t)(uc[1] + 4) << 10) | ((uint32_t)(uc[2] + 4) << 20);
+      }
+      S.cell[tt] = mykey[r];
+    }
+    __syncwarp();
+    for (int u = 0; u < T; ++u) {
+      const uint32_t k = S.cell[u];
+#pragma unroll
+      for (int r = 0; r < kMaxWarpCells / 32; ++r) rank[r] += (k < mykey[r]) ? 1u : 0u;
+    }
+    __syncwarp();
+#pragma unroll
+    for (int r = 0; r < kMaxWarpCells / 32; ++r)
+      if (r * 32 + lane < T) {
+        S.cell[rank[r]] = mykey[r];
+        S.ucs[rank[r]] = myuc[r];
+      }
+    __syncwarp();
+  }
+  // ---- 2a. needed children per cell (warp OR)
+  for (int u = 0; u < T; ++u) {
+    const uint32_t pk = S.ucs[u];
+    const int uc[3] = {(int)(pk & 1023u) - 4, (int)((pk >> 10) & 1023u) - 4, (int)(pk >> 20) - 4};
+    float d[3][2];
+#pragma unroll
+    for (int a = 0; a < 3; ++a) slab_d2(B, t, a, uc[a], kFull && G.full[a], d[a][0], d[a][1]);
+    uint32_t mask = 0;
+#pragma unroll
+    for (int b = 0; b < 8; ++b)
+      if (live && d[0][b >> 2] + d[1][(b >> 1) & 1] + d[2][b & 1] <= rc2) mask |= 1u << b;
+    mask = __reduce_or_sync(0xffffffffu, mask);
+    if (lane == 0) S.mask[u] = mask;
+  }
+  __syncwarp();
+  // ---- 2b. runs (one cell per lane), placed by a warp prefix sum in cell order
+  uint32_t nruns = 0, ncand = 0;
+  for (int r0 = 0; r0 < T; r0 += 32) {
+    const int u = r0 + lane;
+    const uint32_t mask = u < T ? S.mask[u] : 0u;
+    uint32_t bnd[9];
+#pragma unroll
+    for (int b = 0; b < 9; ++b) bnd[b] = 0;
+    if (mask) {
+      const uint32_t* cs = F.cell_start + ((size_t)S.cell[u] << 3);
+#pragma unroll
+      for (int b = 0; b < 9; ++b) bnd[b] = cs[b];
+    }
+    uint32_t my_runs = 0, my_cand = 0;
+    uint32_t rs[4], re[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) rs[q] = re[q] = 0;
+    uint32_t m = mask;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (m) {
+        const int b0 = __ffs(m) - 1;
+        const uint32_t run = (~(m >> b0)) & 0xffu;  // first zero bit above the run
+        const int b1 = b0 + (run ? __ffs(run) - 1 : 8 - b0);
+        m &= ~(((1u << b1) - 1u) & ~((1u << b0) - 1u));
+        uint32_t j0 = 0, j1 = 0;
+#pragma unroll
+        for (int b = 0; b < 9; ++b) {
+          j0 = (b == b0) ? bnd[b] : j0;
+          j1 = (b == b1) ? bnd[b] : j1;
+        }
+        if (j1 > j0) {
+          rs[my_runs] = j0;
+          re[my_runs] = j1;
+          my_cand += j1 - j0;
+          ++my_runs;
         }
       }
-      ck[s] = ok ? (uint32_t)morton3((uint32_t)c[0], (uint32_t)c[1], (uint32_t)c[2]) : kNoCell;
     }
-    bitonic_sort<32>(ck);
+    uint32_t sr = my_runs, sc = my_cand;
 #pragma unroll
-    for (int s = 0; s < 27; ++s) s_cells[s][threadIdx.x] = ck[s];
+    for (int off = 1; off < 32; off <<= 1) {
+      const uint32_t a1 = __shfl_up_sync(0xffffffffu, sr, off), a2 = __shfl_up_sync(0xffffffffu, sc, off);
+      if (lane >= off) {
+        sr += a1;
+        sc += a2;
+      }
+    }
+    uint32_t pr = nruns + sr - my_runs, pc = ncand + sc - my_cand;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (q < (int)my_runs) {
+        S.run_start[pr + q] = rs[q];
+        S.run_pos[pr + q] = pc;
+        S.run_cell[pr + q] = (uint32_t)u;
+        pc += re[q] - rs[q];
+      }
+    }
+    nruns += __shfl_sync(0xffffffffu, sr, 31);
+    ncand += __shfl_sync(0xffffffffu, sc, 31);
+  }
+  if (lane == 0) S.run_pos[nruns] = ncand;
+  __syncwarp();
 
-    const double xi = F.f[FX][i], yi = F.f[FY][i], zi = F.f[FZ][i], hi = F.f[FH][i];
-    const double r2max = (2.0 * hi) * (2.0 * hi);
-    double L0 = ds->box_max[0] - ds->box_min[0], L1 = ds->box_max[1] - ds->box_min[1],
-           L2 = ds->box_max[2] - ds->box_min[2];
-    double H0 = 0.5 * L0, H1 = 0.5 * L1, H2 = 0.5 * L2;
-    const bool p0 = P.periodic[0], p1 = P.periodic[1], p2 = P.periodic[2];
-    const double* __restrict__ X = F.f[FX];
-    const double* __restrict__ Y = F.f[FY];
-    const double* __restrict__ Z = F.f[FZ];
-    int32_t* __restrict__ nbr = F.nbr;
-    const int64_t cap = F.cap;
-    const int ngmax = F.ngmax;
-    uint32_t prev = kNoCell;
-    for (int s = 0; s < 27; ++s) {
-      const uint32_t cell = s_cells[s][threadIdx.x];
-      if (cell == kNoCell) break;
-      if (cell == prev) continue;
-      prev = cell;
-      const uint32_t j0 = F.cell_start[cell], j1 = F.cell_start[cell + 1];
-      for (uint32_t j = j0; j < j1; ++j) {
-        if ((int64_t)j == i) continue;
-        double dx = min_image(__dsub_rn(xi, __ldg(X + j)), L0, H0, p0);
-        double dy = min_image(__dsub_rn(yi, __ldg(Y + j)), L1, H1, p1);
-        double dz = min_image(__dsub_rn(zi, __ldg(Z + j)), L2, H2, p2);
-        double d2 = __dadd_rn(__dadd_rn(__dmul_rn(dx, dx), __dmul_rn(dy, dy)), __dmul_rn(dz, dz));
-        if (d2 < r2max) {
-          if (cnt < ngmax) nbr[(int64_t)cnt * cap + i] = (int32_t)j;
+  // ---- where the target itself sits in the stream (always there: its own fine
+  // cell is at distance 0), so that it can be dropped from its hits
+  int c_self = -1, k_self = 0;
+  if (live && nruns > 0) {
+    int lo = 0, hi = (int)nruns - 1;
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if ((int64_t)S.run_start[mid] <= i) lo = mid;
+      else hi = mid - 1;
+    }
+    const int64_t s0 = S.run_start[lo];
+    const int64_t len = (int64_t)S.run_pos[lo + 1] - S.run_pos[lo];
+    if (s0 <= i && i < s0 + len) {
+      const int64_t g = S.run_pos[lo] + (i - s0);
+      c_self = (int)(g >> 5);
+      k_self = (int)(g & 31);
+    }
+  }
+
+  // ---- 3./4. stream, test, append
+  const uint32_t nchunks = (ncand + 31) / 32;
+  uint32_t run = 0;
+  float4 q = make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);  // NaN: fails every test
+  float sx = 0.f, sy = 0.f, sz = 0.f;
+  uint32_t qj = 0;
+  auto load = [&](uint32_t c) {
+    const uint32_t g = c * 32 + (uint32_t)lane;
+    sx = sy = sz = 0.f;
+    if (g >= ncand) {
+      q = make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
+      qj = 0;
+      return;
+    }
+    while (S.run_pos[run + 1] <= g) ++run;
+    qj = S.run_start[run] + (g - S.run_pos[run]);
+    q = F.pos4[qj];
+    // unwrapped position of the candidate = stored + k L (k = -1, 0, 1); the
+    // shift is applied when the chunk is staged (keeps the load latency hidden)
+    const uint32_t pk = S.ucs[S.run_cell[run]];
+    const int uc[3] = {(int)(pk & 1023u) - 4, (int)((pk >> 10) & 1023u) - 4, (int)(pk >> 20) - 4};
+    if (!(kFull && G.full[0])) sx = uc[0] < 0 ? -B.Lf[0] : (uc[0] >= n ? B.Lf[0] : 0.f);
+    if (!(kFull && G.full[1])) sy = uc[1] < 0 ? -B.Lf[1] : (uc[1] >= n ? B.Lf[1] : 0.f);
+    if (!(kFull && G.full[2])) sz = uc[2] < 0 ? -B.Lf[2] : (uc[2] >= n ? B.Lf[2] : 0.f);
+  };
+  const unsigned long long mx2 = pack2(t.m[0], t.m[0]), my2 = pack2(t.m[1], t.m[1]),
+                           mz2 = pack2(t.m[2], t.m[2]);
+  int32_t* wp = F.nbr + (int64_t)cnt * cap + i;
+  if (nchunks) load(0);
+  for (uint32_t c = 0; c < nchunks; ++c) {
+    S.cx[lane] = q.x + sx;
+    S.cy[lane] = q.y + sy;
+    S.cz[lane] = q.z + sz;
+    S.cj[lane] = qj;
+    __syncwarp();
+    if (c + 1 < nchunks) load(c + 1);
+    uint32_t hin = 0, hout = 0;
+#pragma unroll
+    for (int k = 0; k < 32; k += 2) {
+      const unsigned long long px = *reinterpret_cast<const unsigned long long*>(&S.cx[k]);
+      const unsigned long long py = *reinterpret_cast<const unsigned long long*>(&S.cy[k]);
+      const unsigned long long pz = *reinterpret_cast<const unsigned long long*>(&S.cz[k]);
+      unsigned long long dx = sub2(mx2, px), dy = sub2(my2, py), dz = sub2(mz2, pz);
+      if (kFull) {
+        float a0, a1;
+        unpack2(dx, a0, a1);
+        if (G.full[0]) { a0 -= B.Lf[0] * rintf(a0 / B.Lf[0]); a1 -= B.Lf[0] * rintf(a1 / B.Lf[0]); }
+        dx = pack2(a0, a1);
+        unpack2(dy, a0, a1);
+        if (G.full[1]) { a0 -= B.Lf[1] * rintf(a0 / B.Lf[1]); a1 -= B.Lf[1] * rintf(a1 / B.Lf[1]); }
+        dy = pack2(a0, a1);
+        unpack2(dz, a0, a1);
+        if (G.full[2]) { a0 -= B.Lf[2] * rintf(a0 / B.Lf[2]); a1 -= B.Lf[2] * rintf(a1 / B.Lf[2]); }
+        dz = pack2(a0, a1);
+      }
+      const unsigned long long d2 = fma2(dx, dx, fma2(dy, dy, mul2(dz, dz)));
+      float e0, e1;
+      unpack2(d2, e0, e1);
+      hin |= (e0 < t.r_in2 ? 1u : 0u) << k;
+      hin |= (e1 < t.r_in2 ? 1u : 0u) << (k + 1);
+      hout |= (e0 < t.r_out2 ? 1u : 0u) << k;
+      hout |= (e1 < t.r_out2 ? 1u : 0u) << (k + 1);
+    }
+    if (c == (uint32_t)c_self) {  // the target itself is not its own neighbour
+      hin &= ~(1u << k_self);
+      hout &= ~(1u << k_self);
+    }
+    // thin shell: the exact fp64 predicate decides (rare)
+    uint32_t shell = hout & ~hin;
+    if (__any_sync(0xffffffffu, shell != 0)) {
+      while (shell) {
+        const int k = __ffs(shell) - 1;
+        shell &= shell - 1;
+        if (exact_in(F, B, t, S.cj[k])) hin |= 1u << k;
+      }
+    }
+    // append in candidate order (predicated, no per-lane loop imbalance)
+    if (__any_sync(0xffffffffu, hin != 0)) {
+#pragma unroll
+      for (int k = 0; k < 32; ++k) {
+        if (hin & (1u << k)) {
+          if (cnt < ngmax) *wp = (int32_t)S.cj[k];
+          wp += cap;
           ++cnt;
         }
       }
     }
-    F.nc[i] = cnt;
+    __syncwarp();
   }
+}
+
+__global__ void __launch_bounds__(kNbrThreads) neighbors_kernel(Fields F, Params P) {
+  __shared__ WarpSmem s_w[kNbrWarps];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  const bool active = i < F.n;
+  if (!__any_sync(0xffffffffu, active)) return;  // whole warp past the end
+  const DevScalars* ds = F.ds;
+  Box B;
+  B.Lc = ds->cell_level - 1;
+  B.nside = 1 << B.Lc;
+#pragma unroll
+  for (int a = 0; a < 3; ++a) {
+    B.L[a] = ds->box_max[a] - ds->box_min[a];
+    B.H[a] = 0.5 * B.L[a];
+    B.Lf[a] = (float)B.L[a];
+    B.side[a] = (float)(B.L[a] / B.nside);
+    B.per[a] = P.periodic[a] != 0;
+  }
+  const Target t = make_target(F, B, i, active);
+  int cnt = 0;
+
+  // group size: the whole warp unless its box exceeds kMaxWarpCells cells
+  int g = 32;
+  GroupBox mine = group_box(B, t, active, g);
+  while (g > 1 && __reduce_max_sync(0xffffffffu, mine.T) > kMaxWarpCells) {
+    g >>= 1;
+    mine = group_box(B, t, active, g);
+  }
+  for (int gid = 0; gid < 32 / g; ++gid) {
+    const int src = gid * g;
+    GroupBox G;
+#pragma unroll
+    for (int a = 0; a < 3; ++a) {
+      G.lo[a] = __shfl_sync(0xffffffffu, mine.lo[a], src);
+      G.ext[a] = __shfl_sync(0xffffffffu, mine.ext[a], src);
+      G.full[a] = __shfl_sync(0xffffffffu, (int)mine.full[a], src) != 0;
+    }
+    G.T = __shfl_sync(0xffffffffu, mine.T, src);
+    if (G.T == 0) continue;
+    Target tg = t;
+    if (lane / g != gid) tg.r_out2 = tg.r_in2 = tg.rc = -1.f;  // not in this pass
+    if (G.full[0] || G.full[1] || G.full[2])
+      warp_walk<true>(F, B, tg, i, G, s_w[warp], lane, cnt);
+    else
+      warp_walk<false>(F, B, tg, i, G, s_w[warp], lane, cnt);
+    __syncwarp();
+  }
+  if (active) F.nc[i] = cnt;
+
   // nc statistics (min, max, total) and the capacity flag.
   int mn = active ? cnt : 0x7fffffff, mx = active ? cnt : 0;
   unsigned long long tot = active ? (unsigned long long)cnt : 0ull;
@@ -168,7 +542,7 @@ __global__ void __launch_bounds__(kNbrThreads) neighbors_kernel(Fields F, Params
     mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, off));
     tot += __shfl_xor_sync(0xffffffffu, tot, off);
   }
-  if ((threadIdx.x & 31) == 0 && mn != 0x7fffffff) {  // warp had an active lane
+  if (lane == 0) {
     atomicMin(&F.ds->min_nc, mn);
     atomicMax(&F.ds->max_nc, mx);
     atomicAdd(&F.ds->total_nc, tot);
@@ -178,7 +552,8 @@ __global__ void __launch_bounds__(kNbrThreads) neighbors_kernel(Fields F, Params
 
 void launch_neighbors(const Fields& F, const Params& P, cudaStream_t st) {
   if (F.n == 0) return;
-  neighbors_kernel<<<(unsigned)div_up(F.n, kNbrThreads), kNbrThreads, 0, st>>>(F, P); note_launch();
+  neighbors_kernel<<<(unsigned)div_up(F.n, kNbrThreads), kNbrThreads, 0, st>>>(F, P);
+  note_launch();
 }
 
 }  // namespace sph

@@ -5,12 +5,14 @@
 //
 // The three neighbour sums run one thread per target over its stored list in
 // list order (ascending j, the oracle's summation order).  Lists are column-
-// major so the k-th neighbour indices of a warp's 32 consecutive targets are
-// one coalesced 128-B load; the j-side fields are gathers that hit L1/L2
-// because consecutive targets share most neighbours (Morton order).  The sinc
-// kernel is a polynomial in t = r^2 (pi/2h)^2 (no sqrt/sin per pair); the
-// per-particle factors (pi/2h)^2 and K/h^3 are computed once per particle by the
-// density kernel.  All of them are FP64-bound.
+// major so the k-th neighbour indices of a warp's 32 consecutive targets are one
+// coalesced 128-B load.  The j-side data are gathered as packed 32-byte records
+// (one 256-bit load each; see Rec4 in sph_internal.cuh), built by the phase that
+// produces their last field: rec_d by the sort's permutation, rec_i by EOS,
+// rec_m by IAD.  Consecutive targets share most neighbours (Morton order), so the
+// gathers hit L1/L2.  The sinc kernel is a polynomial in t = r^2 (pi/2h)^2 (no
+// sqrt/sin per pair); (pi/2h)^2 and K/h^3 are computed once per particle by the
+// density kernel.  All three sums are FP64-bound.
 #include <algorithm>
 
 #include "sph_internal.cuh"
@@ -37,41 +39,50 @@ __device__ __forceinline__ Geom load_geom(const DevScalars* ds, const Params& P)
   return g;
 }
 
+// d = x_i - x_j, minimum image (the oracle's order: raw difference, then +-L)
+__device__ __forceinline__ void pair_d(const Geom& g, double xi, double yi, double zi, double xj,
+                                       double yj, double zj, double& dx, double& dy, double& dz) {
+  dx = min_image(xi - xj, g.L[0], g.H[0], g.per[0]);
+  dy = min_image(yi - yj, g.L[1], g.H[1], g.per[1]);
+  dz = min_image(zi - zj, g.L[2], g.H[2], g.per[2]);
+}
+
 // ------------------------------------------------------------------ density
 // rho_i = (K/h_i^3) [m_i + sum_j m_j S(pi r_ij / 2h_i)^6]; also writes the
 // per-particle kernel factors wq = (pi/2h)^2 and wk = K/h^3 reused by IAD and
-// momentum-energy.  Per pair: 4 gathered doubles (x, y, z, m), ~27 DP flops.
-__global__ void __launch_bounds__(256) density_kernel(Fields F, Params P, double* __restrict__ wq,
-                                                      double* __restrict__ wk) {
+// momentum-energy.  Per pair: one 32-B record {x, y, z, m}, 40 DP flops.
+__global__ void __launch_bounds__(256) density_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= F.n) return;
   const Geom g = load_geom(F.ds, P);
-  const double* __restrict__ X = F.f[FX];
-  const double* __restrict__ Y = F.f[FY];
-  const double* __restrict__ Z = F.f[FZ];
-  const double* __restrict__ M = F.f[FM];
-  const double xi = X[i], yi = Y[i], zi = Z[i], hi = F.f[FH][i];
+  const Rec4 me = F.rec_d[i];
+  const double hi = F.f[FH][i];
   const double q = kPi2Over4 / (hi * hi);
   const double kh3 = P.K / (hi * hi * hi);
   const int nci = min(F.nc[i], F.ngmax);
-  double sum = M[i];
+  double sum = me.d;
   const int32_t* __restrict__ nb = F.nbr + i;
+  const Rec4* __restrict__ rec = F.rec_d;
+  // software pipeline: neighbour index two ahead, record one ahead
+  int j1 = nci > 1 ? __ldg(nb + F.cap) : 0;
+  Rec4 rn = nci > 0 ? ldg4(rec + __ldg(nb)) : Rec4{0, 0, 0, 0};
   for (int k = 0; k < nci; ++k) {
-    const int j = __ldg(nb + (int64_t)k * F.cap);
-    double dx = min_image(xi - __ldg(X + j), g.L[0], g.H[0], g.per[0]);
-    double dy = min_image(yi - __ldg(Y + j), g.L[1], g.H[1], g.per[1]);
-    double dz = min_image(zi - __ldg(Z + j), g.L[2], g.H[2], g.per[2]);
-    double r2 = dx * dx + dy * dy + dz * dz;
-    sum = fma(__ldg(M + j), sinc6_t(r2 * q), sum);
+    const Rec4 rj = rn;
+    if (k + 1 < nci) rn = ldg4(rec + j1);
+    if (k + 2 < nci) j1 = __ldg(nb + (int64_t)(k + 2) * F.cap);
+    double dx, dy, dz;
+    pair_d(g, me.a, me.b, me.c, rj.a, rj.b, rj.c, dx, dy, dz);
+    const double r2 = dx * dx + dy * dy + dz * dz;
+    sum = fma(rj.d, sinc6_t(r2 * q), sum);
   }
   F.rho[i] = kh3 * sum;
-  wq[i] = q;
-  wk[i] = kh3;
+  F.wq[i] = q;
+  F.wk[i] = kh3;
 }
 
 // ------------------------------------------------------------------ EOS
-// Bit-exact vs the oracle (same operation order, IEEE sqrt/div): p, c, and the
-// derived per-particle V = m/rho and p/rho^2 used by the next two sums.
+// Bit-exact vs the oracle (same operation order, IEEE sqrt/div): p, c; plus the
+// derived V = m/rho, p/rho^2 and the IAD record {x, y, z, V}.
 __global__ void __launch_bounds__(256) eos_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= F.n) return;
@@ -84,38 +95,42 @@ __global__ void __launch_bounds__(256) eos_kernel(Fields F, Params P) {
     p = __dmul_rn(__dmul_rn(P.cs0, P.cs0), rho);
     c = P.cs0;
   }
+  const Rec4 rd = F.rec_d[i];
+  const double V = __ddiv_rn(rd.d, rho);
   F.p[i] = p;
   F.c[i] = c;
-  F.vol[i] = __ddiv_rn(F.f[FM][i], rho);
+  F.vol[i] = V;
   F.prho2[i] = __ddiv_rn(p, __dmul_rn(rho, rho));
+  st4(F.rec_i + i, rd.a, rd.b, rd.c, V);
 }
 
 // ------------------------------------------------------------------ IAD
-// tau_i = sum_j V_j W(r,h_i) Delta Delta^T, C_i = tau_i^{-1} (adjugate / det).
-// Per pair: 4 gathered doubles (x, y, z, V), ~41 DP flops.
-__global__ void __launch_bounds__(256) iad_kernel(Fields F, Params P, const double* __restrict__ wq,
-                                                  const double* __restrict__ wk) {
+// tau_i = sum_j V_j W(r,h_i) Delta Delta^T, C_i = tau_i^{-1} (adjugate / det);
+// epilogue: the momentum record of particle i.  Per pair: one 32-B record
+// {x, y, z, V}, 55 DP flops.
+__global__ void __launch_bounds__(256) iad_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= F.n) return;
   const Geom g = load_geom(F.ds, P);
-  const double* __restrict__ X = F.f[FX];
-  const double* __restrict__ Y = F.f[FY];
-  const double* __restrict__ Z = F.f[FZ];
-  const double* __restrict__ V = F.vol;
-  const double xi = X[i], yi = Y[i], zi = Z[i];
-  const double q = wq[i], kh3 = wk[i];
+  const Rec4 me = F.rec_i[i];
+  const double q = F.wq[i], kh3 = F.wk[i];
   const int nci = min(F.nc[i], F.ngmax);
   double t11 = 0, t12 = 0, t13 = 0, t22 = 0, t23 = 0, t33 = 0;
   const int32_t* __restrict__ nb = F.nbr + i;
+  const Rec4* __restrict__ rec = F.rec_i;
+  // software pipeline: neighbour index two ahead, record one ahead
+  int j1 = nci > 1 ? __ldg(nb + F.cap) : 0;
+  Rec4 rn = nci > 0 ? ldg4(rec + __ldg(nb)) : Rec4{0, 0, 0, 0};
   for (int k = 0; k < nci; ++k) {
-    const int j = __ldg(nb + (int64_t)k * F.cap);
-    double dx = min_image(xi - __ldg(X + j), g.L[0], g.H[0], g.per[0]);
-    double dy = min_image(yi - __ldg(Y + j), g.L[1], g.H[1], g.per[1]);
-    double dz = min_image(zi - __ldg(Z + j), g.L[2], g.H[2], g.per[2]);
-    double r2 = dx * dx + dy * dy + dz * dz;
-    double vw = __ldg(V + j) * (kh3 * sinc6_t(r2 * q));
+    const Rec4 rj = rn;
+    if (k + 1 < nci) rn = ldg4(rec + j1);
+    if (k + 2 < nci) j1 = __ldg(nb + (int64_t)(k + 2) * F.cap);
+    double dx, dy, dz;
+    pair_d(g, me.a, me.b, me.c, rj.a, rj.b, rj.c, dx, dy, dz);
+    const double r2 = dx * dx + dy * dy + dz * dz;
+    const double vw = rj.d * (kh3 * sinc6_t(r2 * q));
     // Delta = -d; the products Delta^a Delta^b equal d^a d^b.
-    double ax = vw * dx, ay = vw * dy, az = vw * dz;
+    const double ax = vw * dx, ay = vw * dy, az = vw * dz;
     t11 = fma(ax, dx, t11);
     t12 = fma(ax, dy, t12);
     t13 = fma(ax, dz, t13);
@@ -126,13 +141,22 @@ __global__ void __launch_bounds__(256) iad_kernel(Fields F, Params P, const doub
   const double det = t11 * (t22 * t33 - t23 * t23) - t12 * (t12 * t33 - t23 * t13) +
                      t13 * (t12 * t23 - t22 * t13);
   const double inv = 1.0 / det;
-  F.C[0][i] = (t22 * t33 - t23 * t23) * inv;
-  F.C[1][i] = (t13 * t23 - t12 * t33) * inv;
-  F.C[2][i] = (t12 * t23 - t13 * t22) * inv;
-  F.C[3][i] = (t11 * t33 - t13 * t13) * inv;
-  F.C[4][i] = (t12 * t13 - t11 * t23) * inv;
-  F.C[5][i] = (t11 * t22 - t12 * t12) * inv;
+  const double c11 = (t22 * t33 - t23 * t23) * inv, c12 = (t13 * t23 - t12 * t33) * inv;
+  const double c13 = (t12 * t23 - t13 * t22) * inv, c22 = (t11 * t33 - t13 * t13) * inv;
+  const double c23 = (t12 * t13 - t11 * t23) * inv, c33 = (t11 * t22 - t12 * t12) * inv;
+  F.C[0][i] = c11;
+  F.C[1][i] = c12;
+  F.C[2][i] = c13;
+  F.C[3][i] = c22;
+  F.C[4][i] = c23;
+  F.C[5][i] = c33;
   if (!(det > 0.0) || !isfinite(det)) atomicOr(&F.ds->status, (int)ST_SINGULAR);
+  Rec4* rm = F.rec_m + (int64_t)kRecM * i;
+  st4(rm + 0, me.a, me.b, me.c, q);
+  st4(rm + 1, c11, c12, c13, kh3);
+  st4(rm + 2, c22, c23, c33, F.f[FM][i]);
+  st4(rm + 3, F.f[FVX][i], F.f[FVY][i], F.f[FVZ][i], F.prho2[i]);
+  st4(rm + 4, F.f[FH][i], F.c[i], F.rho[i], 0.0);
 }
 
 // ------------------------------------------------------------------ momentum-energy
@@ -141,72 +165,68 @@ __global__ void __launch_bounds__(256) iad_kernel(Fields F, Params P, const doub
 // A = C_i Delta W(r,h_i), B = C_j Delta W(r,h_j), G = (A+B)/2, Monaghan Pi.
 // Also the warp-min of h_i/c_i for the time step (exact: integer atomicMin on the
 // order-preserving bit pattern of a positive double).
-// Per pair: 18 gathered doubles, ~150 DP flops (+ 2 divisions when approaching).
-__global__ void __launch_bounds__(128) momentum_energy_kernel(Fields F, Params P,
-                                                              const double* __restrict__ wq,
-                                                              const double* __restrict__ wk) {
+// Per pair: 4 records (128 B) + 1 more (AV) for approaching pairs, 157 DP flops
+// (+ 17 and 2 divisions when approaching).
+__global__ void __launch_bounds__(128) momentum_energy_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   const bool active = i < F.n;
   unsigned long long hc = ~0ull;
   if (active) {
     const Geom g = load_geom(F.ds, P);
-    const double* __restrict__ X = F.f[FX];
-    const double* __restrict__ Y = F.f[FY];
-    const double* __restrict__ Z = F.f[FZ];
-    const double* __restrict__ VX = F.f[FVX];
-    const double* __restrict__ VY = F.f[FVY];
-    const double* __restrict__ VZ = F.f[FVZ];
-    const double* __restrict__ Hh = F.f[FH];
-    const double* __restrict__ M = F.f[FM];
-    const double* __restrict__ RHO = F.rho;
-    const double* __restrict__ PR = F.prho2;
-    const double* __restrict__ CS = F.c;
-    const double* __restrict__ C0 = F.C[0];
-    const double* __restrict__ C1 = F.C[1];
-    const double* __restrict__ C2 = F.C[2];
-    const double* __restrict__ C3 = F.C[3];
-    const double* __restrict__ C4 = F.C[4];
-    const double* __restrict__ C5 = F.C[5];
-    const double xi = X[i], yi = Y[i], zi = Z[i];
-    const double vxi = VX[i], vyi = VY[i], vzi = VZ[i];
-    const double hi = Hh[i], rhoi = RHO[i], pri = PR[i], ci = CS[i];
-    const double ci11 = C0[i], ci12 = C1[i], ci13 = C2[i], ci22 = C3[i], ci23 = C4[i], ci33 = C5[i];
-    const double qi = wq[i], khi = wk[i];
+    const Rec4* __restrict__ rec = F.rec_m;
+    const Rec4* mi = rec + (int64_t)kRecM * i;
+    const Rec4 i0 = mi[0], i1 = mi[1], i2 = mi[2], i3 = mi[3], i4 = mi[4];
+    const double xi = i0.a, yi = i0.b, zi = i0.c, qi = i0.d;
+    const double ci11 = i1.a, ci12 = i1.b, ci13 = i1.c, khi = i1.d;
+    const double ci22 = i2.a, ci23 = i2.b, ci33 = i2.c;
+    const double vxi = i3.a, vyi = i3.b, vzi = i3.c, pri = i3.d;
+    const double hi = i4.a, ci = i4.b, rhoi = i4.c;
     const double alpha = P.av_alpha, beta = P.av_beta, eps = P.av_eps;
     const int nci = min(F.nc[i], F.ngmax);
     double ax = 0, ay = 0, az = 0, de = 0;
     const int32_t* __restrict__ nb = F.nbr + i;
+    // software pipeline: neighbour index two ahead, its 4 record chunks one ahead
+    int jn = nci > 1 ? __ldg(nb + F.cap) : 0;
+    const Rec4* rj = rec + (int64_t)kRecM * (nci > 0 ? __ldg(nb) : 0);
+    Rec4 n0 = ldg4(rj), n1 = ldg4(rj + 1), n2 = ldg4(rj + 2), n3 = ldg4(rj + 3);
     for (int k = 0; k < nci; ++k) {
-      const int j = __ldg(nb + (int64_t)k * F.cap);
-      const double dx = min_image(xi - __ldg(X + j), g.L[0], g.H[0], g.per[0]);
-      const double dy = min_image(yi - __ldg(Y + j), g.L[1], g.H[1], g.per[1]);
-      const double dz = min_image(zi - __ldg(Z + j), g.L[2], g.H[2], g.per[2]);
+      const Rec4 j0 = n0, j1 = n1, j2 = n2, j3 = n3;
+      const Rec4* rcur = rj;
+      if (k + 1 < nci) {
+        rj = rec + (int64_t)kRecM * jn;
+        n0 = ldg4(rj);
+        n1 = ldg4(rj + 1);
+        n2 = ldg4(rj + 2);
+        n3 = ldg4(rj + 3);
+      }
+      if (k + 2 < nci) jn = __ldg(nb + (int64_t)(k + 2) * F.cap);
+      double dx, dy, dz;
+      pair_d(g, xi, yi, zi, j0.a, j0.b, j0.c, dx, dy, dz);
       const double r2 = dx * dx + dy * dy + dz * dz;
       const double wi = khi * sinc6_t(r2 * qi);
-      const double tj = r2 * __ldg(wq + j);
-      const double wj = tj < kPi2 ? __ldg(wk + j) * sinc6_t(tj) : 0.0;
+      const double tj = r2 * j0.d;
+      const double wj = tj < kPi2 ? j1.d * sinc6_t(tj) : 0.0;
       // Delta = -d
       const double Dx = -dx, Dy = -dy, Dz = -dz;
-      const double cj11 = __ldg(C0 + j), cj12 = __ldg(C1 + j), cj13 = __ldg(C2 + j);
-      const double cj22 = __ldg(C3 + j), cj23 = __ldg(C4 + j), cj33 = __ldg(C5 + j);
       const double Ax = (ci11 * Dx + ci12 * Dy + ci13 * Dz) * wi;
       const double Ay = (ci12 * Dx + ci22 * Dy + ci23 * Dz) * wi;
       const double Az = (ci13 * Dx + ci23 * Dy + ci33 * Dz) * wi;
-      const double Bx = (cj11 * Dx + cj12 * Dy + cj13 * Dz) * wj;
-      const double By = (cj12 * Dx + cj22 * Dy + cj23 * Dz) * wj;
-      const double Bz = (cj13 * Dx + cj23 * Dy + cj33 * Dz) * wj;
+      const double Bx = (j1.a * Dx + j1.b * Dy + j1.c * Dz) * wj;
+      const double By = (j1.b * Dx + j2.a * Dy + j2.b * Dz) * wj;
+      const double Bz = (j1.c * Dx + j2.b * Dy + j2.c * Dz) * wj;
       const double Gx = 0.5 * (Ax + Bx), Gy = 0.5 * (Ay + By), Gz = 0.5 * (Az + Bz);
-      const double vx = vxi - __ldg(VX + j), vy = vyi - __ldg(VY + j), vz = vzi - __ldg(VZ + j);
+      const double vx = vxi - j3.a, vy = vyi - j3.b, vz = vzi - j3.c;
       const double rv = dx * vx + dy * vy + dz * vz;
       double Pi = 0.0;
       if (rv < 0.0) {
-        const double hbar = 0.5 * (hi + __ldg(Hh + j));
-        const double cbar = 0.5 * (ci + __ldg(CS + j));
-        const double rhobar = 0.5 * (rhoi + __ldg(RHO + j));
+        const Rec4 j4 = ldg4(rcur + 4);
+        const double hbar = 0.5 * (hi + j4.a);
+        const double cbar = 0.5 * (ci + j4.b);
+        const double rhobar = 0.5 * (rhoi + j4.c);
         const double mu = hbar * rv / (r2 + eps * hbar * hbar);
         Pi = (-alpha * cbar * mu + beta * mu * mu) / rhobar;
       }
-      const double mj = __ldg(M + j), prj = __ldg(PR + j);
+      const double mj = j2.d, prj = j3.d;
       ax -= mj * (pri * Ax + prj * Bx + Pi * Gx);
       ay -= mj * (pri * Ay + prj * By + Pi * Gy);
       az -= mj * (pri * Az + prj * Bz + Pi * Gz);
@@ -235,6 +255,8 @@ __global__ void timestep_kernel(DevScalars* ds, Params P) {
 }
 
 // ------------------------------------------------------------------ update
+// Item 10: kick (v at half steps), drift + periodic wrap, AB2 energy, h update.
+// HBM-bound: 13 doubles + nc read, 9 doubles written per particle.
 __global__ void __launch_bounds__(256) update_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= F.n) return;
@@ -274,27 +296,36 @@ __global__ void advance_time_kernel(DevScalars* ds) {
 // ------------------------------------------------------------------ launchers
 void launch_density(const Fields& F, const Params& P, cudaStream_t st) {
   if (F.n == 0) return;
-  density_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F, P, F.wq, F.wk); note_launch();
+  density_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F, P);
+  note_launch();
 }
 void launch_eos(const Fields& F, const Params& P, cudaStream_t st) {
   if (F.n == 0) return;
-  eos_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F, P); note_launch();
+  eos_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F, P);
+  note_launch();
 }
 void launch_iad(const Fields& F, const Params& P, cudaStream_t st) {
   if (F.n == 0) return;
-  iad_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F, P, F.wq, F.wk); note_launch();
+  iad_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F, P);
+  note_launch();
 }
 void launch_momentum_energy(const Fields& F, const Params& P, cudaStream_t st) {
   if (F.n == 0) return;
-  momentum_energy_kernel<<<(unsigned)div_up(F.n, 128), 128, 0, st>>>(F, P, F.wq, F.wk); note_launch();
+  momentum_energy_kernel<<<(unsigned)div_up(F.n, 128), 128, 0, st>>>(F, P);
+  note_launch();
 }
 void launch_timestep(const Fields& F, const Params& P, cudaStream_t st) {
-  timestep_kernel<<<1, 1, 0, st>>>(F.ds, P); note_launch();
+  timestep_kernel<<<1, 1, 0, st>>>(F.ds, P);
+  note_launch();
 }
 void launch_update(const Fields& F, const Params& P, cudaStream_t st) {
   if (F.n == 0) return;
-  update_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F, P); note_launch();
+  update_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F, P);
+  note_launch();
 }
-void launch_advance_time(const Fields& F, cudaStream_t st) { advance_time_kernel<<<1, 1, 0, st>>>(F.ds); note_launch(); }
+void launch_advance_time(const Fields& F, cudaStream_t st) {
+  advance_time_kernel<<<1, 1, 0, st>>>(F.ds);
+  note_launch();
+}
 
 }  // namespace sph

@@ -241,32 +241,40 @@ cudaError_t launch_sort(const Fields& F, uint64_t* key_in, uint64_t* key_tmp, ui
   return cudaGetLastError();
 }
 
-// Gathers every persistent field into key order: dst_f[k] = src_f[perm[k]].
+// Gathers every persistent field into key order, dst_f[k] = src_f[perm[k]], and
+// writes the two records the next phases gather from: the fp32 prefilter
+// position pos4 = (x, y, z) - box_min and rec_d = {x, y, z, m} (density).
+// HBM-bound: 11 x 8 B read (gather, near-identity permutation) + 11 x 8 B + 16 B
+// + 32 B written per particle.
 struct PermPtrs {
   const double* src[kNumStateF];
-  double* dst[kNumStateF];
 };
 
-__global__ void __launch_bounds__(256) permute_kernel(int64_t n, const uint32_t* __restrict__ perm,
-                                                      PermPtrs P, const int64_t* __restrict__ id_src,
-                                                      int64_t* __restrict__ id_dst) {
+__global__ void __launch_bounds__(256) permute_kernel(Fields F, const uint32_t* __restrict__ perm,
+                                                      PermPtrs P, const int64_t* __restrict__ id_src) {
   int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (i >= n) return;
+  if (i >= F.n) return;
   uint32_t p = perm[i];
+  double v[kNumStateF];
 #pragma unroll
-  for (int f = 0; f < kNumStateF; ++f) P.dst[f][i] = __ldg(P.src[f] + p);
-  id_dst[i] = __ldg(id_src + p);
+  for (int f = 0; f < kNumStateF; ++f) {
+    v[f] = __ldg(P.src[f] + p);
+    F.f[f][i] = v[f];
+  }
+  F.id[i] = __ldg(id_src + p);
+  const DevScalars* ds = F.ds;
+  F.pos4[i] = make_float4((float)(v[FX] - ds->box_min[0]), (float)(v[FY] - ds->box_min[1]),
+                          (float)(v[FZ] - ds->box_min[2]), 0.f);
+  st4(F.rec_d + i, v[FX], v[FY], v[FZ], v[FM]);
 }
 
-void launch_permute(int64_t n, const uint32_t* perm, double* const* src, double* const* dst,
-                    const int64_t* id_src, int64_t* id_dst, cudaStream_t st) {
-  if (n == 0) return;
+void launch_permute(const Fields& Fdst, const uint32_t* perm, double* const* src,
+                    const int64_t* id_src, cudaStream_t st) {
+  if (Fdst.n == 0) return;
   PermPtrs P;
-  for (int f = 0; f < kNumStateF; ++f) {
-    P.src[f] = src[f];
-    P.dst[f] = dst[f];
-  }
-  permute_kernel<<<(unsigned)div_up(n, 256), 256, 0, st>>>(n, perm, P, id_src, id_dst); note_launch();
+  for (int f = 0; f < kNumStateF; ++f) P.src[f] = src[f];
+  permute_kernel<<<(unsigned)div_up(Fdst.n, 256), 256, 0, st>>>(Fdst, perm, P, id_src);
+  note_launch();
 }
 
 }  // namespace sph

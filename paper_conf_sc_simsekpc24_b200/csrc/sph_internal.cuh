@@ -37,7 +37,7 @@ struct DevScalars {
   double box_min[3], box_max[3];      // the box used by this step
   unsigned long long hmax_ord;        // max h (cell level)
   unsigned long long minhc_ord;       // min h/c (time step)
-  int cell_level;
+  int cell_level;         // fine level of the cell table (= coarse + 1)
   int status;
   int max_nc, min_nc;
   unsigned long long total_nc;
@@ -45,6 +45,34 @@ struct DevScalars {
   int first;
   int pad;
 };
+
+// 32-byte record: one 256-bit load (LDG.E.256 on sm_100a).
+struct __align__(32) Rec4 {
+  double a, b, c, d;
+};
+__device__ __forceinline__ Rec4 ldg4(const Rec4* p) {
+  Rec4 r;
+  asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];"
+      : "=d"(r.a), "=d"(r.b), "=d"(r.c), "=d"(r.d)
+      : "l"(p));
+  return r;
+}
+__device__ __forceinline__ void st4(Rec4* p, double a, double b, double c, double d) {
+  asm volatile("st.global.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(p), "d"(a), "d"(b), "d"(c), "d"(d)
+               : "memory");
+}
+
+// Gather-friendly j-side records.  The neighbour sums
+// read, per pair, whole records instead of one 8-byte word from each of up to 19
+// separate arrays: 1 sector (density, IAD) or 4-5 sectors (momentum) per pair.
+//   rec_d[j]       = {x, y, z, m}                                (density)
+//   rec_i[j]       = {x, y, z, V = m/rho}                        (IAD)
+//   rec_m[5j + 0]  = {x, y, z, wq}      wq = (pi/2h)^2            (momentum)
+//   rec_m[5j + 1]  = {C11, C12, C13, wk}  wk = K/h^3
+//   rec_m[5j + 2]  = {C22, C23, C33, m}
+//   rec_m[5j + 3]  = {vx, vy, vz, p/rho^2}
+//   rec_m[5j + 4]  = {h, c, rho, 0}      (read only for approaching pairs)
+constexpr int kRecM = 5;
 
 // Everything the kernels need, passed by value.
 struct Fields {
@@ -59,7 +87,11 @@ struct Fields {
   int32_t* nc;
   int32_t* nbr;           // [ngmax][cap]
   int32_t ngmax;
-  uint32_t* cell_start;   // [8^L + 1]
+  uint32_t* cell_start;   // [8^L + 1], L = fine cell level
+  float4* pos4;           // fp32 (x, y, z) - box_min: neighbour-search prefilter
+  Rec4* rec_d;
+  Rec4* rec_i;
+  Rec4* rec_m;            // [kRecM * cap]
   DevScalars* ds;
 };
 
@@ -160,8 +192,8 @@ void sort_workspace(int64_t cap, size_t* hist_bytes, size_t* status_bytes);
 cudaError_t launch_sort(const Fields& F, uint64_t* key_in, uint64_t* key_tmp, uint32_t* val_a,
                         uint32_t* val_b, uint32_t* hist, uint32_t* status, size_t status_bytes,
                         uint32_t** perm_out, uint64_t** key_out, cudaStream_t st);
-void launch_permute(int64_t n, const uint32_t* perm, double* const* src, double* const* dst,
-                    const int64_t* id_src, int64_t* id_dst, cudaStream_t st);
+void launch_permute(const Fields& Fdst, const uint32_t* perm, double* const* src,
+                    const int64_t* id_src, cudaStream_t st);
 void launch_cells(const Fields& F, const Params& P, int level_cap, cudaStream_t st);
 void launch_neighbors(const Fields& F, const Params& P, cudaStream_t st);
 void launch_density(const Fields& F, const Params& P, cudaStream_t st);
