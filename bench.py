@@ -307,7 +307,10 @@ def main():
                            "parallelism": "single GPU" if world == 1 else
                            f"{world} independent replicas (SFC decomposition not yet built)",
                            "l2": "inputs (~1 GB state + ~3 GB lists) >> 126 MB L2; no flush",
-                           "mean_nc": mean_nc},
+                           "mean_nc": mean_nc,
+                           "cell_level": infos[-1]["cell_level"],
+                           "search_candidates_per_target": infos[-1]["search_candidates"] / n,
+                           "search_passes_per_warp": infos[-1]["search_passes"] / (n / 32)},
                 "phase_ms": phase_ms, "fp64_other": other, "roofline": roofline, "e2e": e2e,
                 "energy": energy, "cpu_baseline": cpu, "clocks": clk.summary(),
                 "gpu_launches": launches}

@@ -140,6 +140,8 @@ typedef struct sph_nbr_stats {
   int32_t min_nc, max_nc;   /* over all particles                                  */
   double mean_nc;
   int64_t total;            /* sum of nc                                           */
+  int64_t candidates;       /* diagnostic: candidate tests of the search (per lane) */
+  int64_t passes;           /* diagnostic: warp passes of the search               */
 } sph_nbr_stats;
 
 typedef struct sph_step_info {

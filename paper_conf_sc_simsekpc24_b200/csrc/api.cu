@@ -218,6 +218,8 @@ void fill_stats(sph_ctx* c, sph_nbr_stats* s) {
   s->max_nc = c->h_ds.max_nc;
   s->total = (int64_t)c->h_ds.total_nc;
   s->mean_nc = c->n ? (double)c->h_ds.total_nc / (double)c->n : 0.0;
+  s->candidates = (int64_t)c->h_ds.cand_total;
+  s->passes = (int64_t)c->h_ds.pass_total;
 }
 
 __global__ void set_time_kernel(DevScalars* ds, double t, double dt_prev, int first) {
@@ -236,6 +238,8 @@ __global__ void reset_nbr_stats_kernel(DevScalars* ds) {
   ds->max_nc = 0;
   ds->min_nc = 0x7fffffff;
   ds->total_nc = 0ull;
+  ds->cand_total = 0ull;
+  ds->pass_total = 0ull;
   ds->status &= ~ST_CAPACITY;
 }
 

@@ -188,6 +188,21 @@ __device__ __forceinline__ unsigned long long fma2(unsigned long long a, unsigne
 }
 
 
+// Position of the r-th (0-based) set bit of m (popc binary search).
+__device__ __forceinline__ int nth_set_bit(uint32_t m, int r) {
+  int pos = 0, c;
+  c = __popc(m & 0xffffu);
+  if (r >= c) { r -= c; m >>= 16; pos += 16; }
+  c = __popc(m & 0xffu);
+  if (r >= c) { r -= c; m >>= 8; pos += 8; }
+  c = __popc(m & 0xfu);
+  if (r >= c) { r -= c; m >>= 4; pos += 4; }
+  c = __popc(m & 0x3u);
+  if (r >= c) { r -= c; m >>= 2; pos += 2; }
+  if (r >= (int)(m & 1u)) pos += 1;
+  return pos;
+}
+
 constexpr int kMaxRuns = 4 * kMaxWarpCells;  // <= 4 runs of children per cell
 
 struct WarpSmem {
@@ -203,98 +218,124 @@ struct WarpSmem {
   alignas(16) float cy[32];
   alignas(16) float cz[32];
   uint32_t cj[32];
+  uint32_t selfm[32];             // per target: chunk slots holding the target itself
 };
 
-// Butterfly min/max within aligned groups of g lanes (g a power of two).
-__device__ __forceinline__ int group_min(int v, int g) {
-  for (int off = 1; off < g; off <<= 1) v = min(v, __shfl_xor_sync(0xffffffffu, v, off));
-  return v;
-}
-__device__ __forceinline__ int group_max(int v, int g) {
-  for (int off = 1; off < g; off <<= 1) v = max(v, __shfl_xor_sync(0xffffffffu, v, off));
-  return v;
-}
-
-// Coarse-cell box of a group of targets: [lo, lo + ext) per axis; "full" axes
-// cover the whole periodic axis (images then resolved per candidate).
+// The group's coarse cells: T distinct (wrapped key, unwrapped coordinates)
+// entries, sorted, in WarpSmem::cell / ::ucs.  "full" axes are periodic axes
+// with fewer than 3 coarse cells: there images are resolved per candidate
+// (minimum image in fp32) and every entry is its own wrapped cell.
 struct GroupBox {
-  int lo[3], ext[3];
   bool full[3];
   int T;
 };
 
-__device__ __forceinline__ GroupBox group_box(const Box& B, const Target& t, bool member, int g) {
+// Builds the sorted union of the 27-cell stencils of the group's distinct
+// coarse cells (at most kMaxGroupCells of them, leader lanes in `leaders`).
+// Entries for the same wrapped cell reached through different periodic images
+// are kept apart (each target uses exactly one image of any particle).
+constexpr int kMaxGroupCells = 4;  // 4 x 27 = 108 <= kMaxWarpCells stencil entries
+
+__device__ __forceinline__ GroupBox build_cells(const Box& B, const int (&cc)[3], uint32_t leaders,
+                                                int lane, WarpSmem& S) {
   GroupBox G;
-  G.T = 1;
+  const int n = B.nside, nm = n - 1;
 #pragma unroll
-  for (int a = 0; a < 3; ++a) {
-    int l = member ? (int)floorf((t.m[a] - t.rc) / B.side[a]) : 0x3fffffff;
-    int h = member ? (int)floorf((t.m[a] + t.rc) / B.side[a]) : -0x3fffffff;
-    l = group_min(l, g);
-    h = group_max(h, g);
-    G.full[a] = false;
-    if (B.per[a]) {
-      if (h - l + 1 >= B.nside) {
-        l = 0;
-        h = B.nside - 1;
-        G.full[a] = true;
-      }
-    } else {
-      l = max(l, 0);
-      h = min(h, B.nside - 1);
+  for (int a = 0; a < 3; ++a) G.full[a] = B.per[a] && n < 3;
+  const int D = __popc(leaders);
+  // the leaders' coarse coordinates, broadcast
+  int lc[kMaxGroupCells][3];
+  {
+    uint32_t l = leaders;
+#pragma unroll
+    for (int d = 0; d < kMaxGroupCells; ++d) {
+      const int src = l ? __ffs(l) - 1 : 0;
+      if (l) l &= l - 1;
+#pragma unroll
+      for (int a = 0; a < 3; ++a) lc[d][a] = __shfl_sync(0xffffffffu, cc[a], src);
     }
-    G.lo[a] = l;
-    G.ext[a] = max(h - l + 1, 0);
-    G.T *= G.ext[a];
   }
+  // stencil entries, 4 per lane: 64-bit sort key (wrapped key << 30 | packed unwrapped)
+  unsigned long long v[kMaxWarpCells / 32];
+#pragma unroll
+  for (int r = 0; r < kMaxWarpCells / 32; ++r) {
+    const int e = r * 32 + lane;
+    v[r] = ~0ull;
+    if (e < D * 27) {
+      int d = e / 27, s = e - d * 27;
+      int base[3] = {lc[0][0], lc[0][1], lc[0][2]};
+#pragma unroll
+      for (int q = 1; q < kMaxGroupCells; ++q)
+        if (d == q) {
+          base[0] = lc[q][0];
+          base[1] = lc[q][1];
+          base[2] = lc[q][2];
+        }
+      const int o[3] = {s / 9 - 1, (s / 3) % 3 - 1, s % 3 - 1};
+      int u[3];
+      bool ok = true;
+#pragma unroll
+      for (int a = 0; a < 3; ++a) {
+        u[a] = base[a] + o[a];
+        if (G.full[a]) u[a] &= nm;                         // one entry per wrapped cell
+        else if (!B.per[a] && (u[a] < 0 || u[a] >= n)) ok = false;  // open face
+      }
+      if (ok) {
+        const uint64_t key = morton3((uint32_t)(u[0] & nm), (uint32_t)(u[1] & nm), (uint32_t)(u[2] & nm));
+        const uint32_t pk = (uint32_t)(u[0] + 4) | ((uint32_t)(u[1] + 4) << 10) | ((uint32_t)(u[2] + 4) << 20);
+        v[r] = (key << 30) | pk;
+      }
+    }
+  }
+  // rank sort (ties -> lower slot first), then drop duplicates
+  unsigned long long* sk = reinterpret_cast<unsigned long long*>(S.run_start);  // scratch (>= 1 KB)
+#pragma unroll
+  for (int r = 0; r < kMaxWarpCells / 32; ++r) sk[r * 32 + lane] = v[r];
+  __syncwarp();
+  uint32_t rank[kMaxWarpCells / 32] = {0, 0, 0, 0};
+  const int E = D * 27;
+  for (int u = 0; u < E; ++u) {
+    const unsigned long long w = sk[u];
+#pragma unroll
+    for (int r = 0; r < kMaxWarpCells / 32; ++r)
+      rank[r] += (w < v[r] || (w == v[r] && u < r * 32 + lane)) ? 1u : 0u;
+  }
+  __syncwarp();
+#pragma unroll
+  for (int r = 0; r < kMaxWarpCells / 32; ++r)
+    if (r * 32 + lane < E) sk[rank[r]] = v[r];
+  __syncwarp();
+  int T = 0;
+#pragma unroll
+  for (int r = 0; r < (E + 31) / 32; ++r) {
+    const int p = r * 32 + lane;
+    const unsigned long long w = p < E ? sk[p] : ~0ull;
+    const bool keep = w != ~0ull && (p == 0 || sk[p - 1] != w);
+    const uint32_t b = __ballot_sync(0xffffffffu, keep);
+    const int pos = T + __popc(b & ((1u << lane) - 1u));
+    T += __popc(b);
+    __syncwarp();
+    if (keep) {
+      S.cell[pos] = (uint32_t)(w >> 30);
+      S.ucs[pos] = (uint32_t)(w & 0x3fffffffull);
+    }
+  }
+  __syncwarp();
+  G.T = T;
   return G;
 }
 
-// The group's candidate stream (see the file header, steps 1-4).  Lanes with
+// The group's candidate stream (see the file header, steps 2-4).  Lanes with
 // t.rc < 0 take part in the warp collectives but test nothing.
 template <bool kFull>
 __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const Target& t, int64_t i,
                                           const GroupBox& G, WarpSmem& S, int lane, int& cnt) {
-  const int n = B.nside, nm = n - 1;
+  const int n = B.nside;
   const int T = G.T;
   const int64_t cap = F.cap;
   const int ngmax = F.ngmax;
   const float rc2 = t.rc * t.rc;
   const bool live = t.rc >= 0.f;
-  // ---- 1. rank the T cells by Morton key (keys are distinct)
-  {
-    uint32_t mykey[kMaxWarpCells / 32], myuc[kMaxWarpCells / 32], rank[kMaxWarpCells / 32];
-#pragma unroll
-    for (int r = 0; r < kMaxWarpCells / 32; ++r) {
-      const int tt = r * 32 + lane;
-      mykey[r] = kNoCell;
-      myuc[r] = 0;
-      rank[r] = 0;
-      if (tt < T) {
-        const int q = tt / G.ext[2];
-        const int uc[3] = {G.lo[0] + q / G.ext[1], G.lo[1] + q % G.ext[1], G.lo[2] + tt - q * G.ext[2]};
-        // wrap (n is a power of two; open axes are clipped to [0, n) already)
-        mykey[r] = (uint32_t)morton3((uint32_t)(uc[0] & nm), (uint32_t)(uc[1] & nm), (uint32_t)(uc[2] & nm));
-        // unwrapped coordinates (>= -2), biased by +4, 10 bits each
-        myuc[r] = (uint32_t)(uc[0] + 4) | ((uint32_t)(uc[1] + 4) << 10) | ((uint32_t)(uc[2] + 4) << 20);
-      }
-      S.cell[tt] = mykey[r];
-    }
-    __syncwarp();
-    for (int u = 0; u < T; ++u) {
-      const uint32_t k = S.cell[u];
-#pragma unroll
-      for (int r = 0; r < kMaxWarpCells / 32; ++r) rank[r] += (k < mykey[r]) ? 1u : 0u;
-    }
-    __syncwarp();
-#pragma unroll
-    for (int r = 0; r < kMaxWarpCells / 32; ++r)
-      if (r * 32 + lane < T) {
-        S.cell[rank[r]] = mykey[r];
-        S.ucs[rank[r]] = myuc[r];
-      }
-    __syncwarp();
-  }
   // ---- 2a. needed children per cell (warp OR)
   for (int u = 0; u < T; ++u) {
     const uint32_t pk = S.ucs[u];
@@ -371,27 +412,12 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
     nruns += __shfl_sync(0xffffffffu, sr, 31);
     ncand += __shfl_sync(0xffffffffu, sc, 31);
   }
-  if (lane == 0) S.run_pos[nruns] = ncand;
-  __syncwarp();
-
-  // ---- where the target itself sits in the stream (always there: its own fine
-  // cell is at distance 0), so that it can be dropped from its hits
-  int c_self = -1, k_self = 0;
-  if (live && nruns > 0) {
-    int lo = 0, hi = (int)nruns - 1;
-    while (lo < hi) {
-      const int mid = (lo + hi + 1) >> 1;
-      if ((int64_t)S.run_start[mid] <= i) lo = mid;
-      else hi = mid - 1;
-    }
-    const int64_t s0 = S.run_start[lo];
-    const int64_t len = (int64_t)S.run_pos[lo + 1] - S.run_pos[lo];
-    if (s0 <= i && i < s0 + len) {
-      const int64_t g = S.run_pos[lo] + (i - s0);
-      c_self = (int)(g >> 5);
-      k_self = (int)(g & 31);
-    }
+  if (lane == 0) {
+    S.run_pos[nruns] = ncand;
+    atomicAdd(&F.ds->cand_total, (unsigned long long)ncand);  // diagnostics
+    atomicAdd(&F.ds->pass_total, 1ull);
   }
+  __syncwarp();
 
   // ---- 3./4. stream, test, append
   const uint32_t nchunks = (ncand + 31) / 32;
@@ -420,13 +446,16 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
   };
   const unsigned long long mx2 = pack2(t.m[0], t.m[0]), my2 = pack2(t.m[1], t.m[1]),
                            mz2 = pack2(t.m[2], t.m[2]);
-  int32_t* wp = F.nbr + (int64_t)cnt * cap + i;
+  const int64_t wbase = i - lane;  // the warp's first target
+  S.selfm[lane] = 0u;
   if (nchunks) load(0);
   for (uint32_t c = 0; c < nchunks; ++c) {
     S.cx[lane] = q.x + sx;
     S.cy[lane] = q.y + sy;
     S.cz[lane] = q.z + sz;
     S.cj[lane] = qj;
+    if (c * 32 + (uint32_t)lane < ncand && (uint64_t)((int64_t)qj - wbase) < 32u)
+      atomicOr(&S.selfm[(int64_t)qj - wbase], 1u << lane);  // candidate is a target of this warp
     __syncwarp();
     if (c + 1 < nchunks) load(c + 1);
     uint32_t hin = 0, hout = 0;
@@ -456,10 +485,6 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
       hout |= (e0 < t.r_out2 ? 1u : 0u) << k;
       hout |= (e1 < t.r_out2 ? 1u : 0u) << (k + 1);
     }
-    if (c == (uint32_t)c_self) {  // the target itself is not its own neighbour
-      hin &= ~(1u << k_self);
-      hout &= ~(1u << k_self);
-    }
     // thin shell: the exact fp64 predicate decides (rare)
     uint32_t shell = hout & ~hin;
     if (__any_sync(0xffffffffu, shell != 0)) {
@@ -469,22 +494,44 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
         if (exact_in(F, B, t, S.cj[k])) hin |= 1u << k;
       }
     }
-    // append in candidate order (predicated, no per-lane loop imbalance)
-    if (__any_sync(0xffffffffu, hin != 0)) {
+    // the target itself (d = 0) is not its own neighbour
+    hin &= ~S.selfm[lane];
+    // cooperative append: the chunk's hits of all lanes (~100) are written by the
+    // 32 lanes together -- owner lane by binary search over the prefix of hit
+    // counts, its r-th hit by a popc search -- each list staying in candidate
+    // (= ascending index) order.
+    const int pc = __popc(hin);
+    int incl = pc;
 #pragma unroll
-      for (int k = 0; k < 32; ++k) {
-        if (hin & (1u << k)) {
-          if (cnt < ngmax) *wp = (int32_t)S.cj[k];
-          wp += cap;
-          ++cnt;
-        }
+    for (int off = 1; off < 32; off <<= 1) {
+      const int v = __shfl_up_sync(0xffffffffu, incl, off);
+      if (lane >= off) incl += v;
+    }
+    const int tot = __shfl_sync(0xffffffffu, incl, 31);
+    for (int hb = 0; hb < tot; hb += 32) {
+      const int h = hb + lane;
+      int owner = 0;
+#pragma unroll
+      for (int step = 16; step > 0; step >>= 1) {
+        const int v = __shfl_sync(0xffffffffu, incl, owner + step - 1);
+        if (v <= h) owner += step;
+      }
+      const int o_excl = __shfl_sync(0xffffffffu, incl - pc, owner);
+      const uint32_t o_mask = __shfl_sync(0xffffffffu, hin, owner);
+      const int o_cnt = __shfl_sync(0xffffffffu, cnt, owner);
+      if (h < tot) {
+        const int r = h - o_excl;
+        const int slot = o_cnt + r;
+        if (slot < ngmax) F.nbr[(int64_t)slot * cap + wbase + owner] = (int32_t)S.cj[nth_set_bit(o_mask, r)];
       }
     }
+    cnt += pc;
+    S.selfm[lane] = 0u;
     __syncwarp();
   }
 }
 
-__global__ void __launch_bounds__(kNbrThreads) neighbors_kernel(Fields F, Params P) {
+__global__ void __launch_bounds__(kNbrThreads, 6) neighbors_kernel(Fields F, Params P) {
   __shared__ WarpSmem s_w[kNbrWarps];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
@@ -503,26 +550,38 @@ __global__ void __launch_bounds__(kNbrThreads) neighbors_kernel(Fields F, Params
     B.per[a] = P.periodic[a] != 0;
   }
   const Target t = make_target(F, B, i, active);
+  int cc[3] = {0, 0, 0};
+  uint32_t ckey = 0;
+  if (active) {
+    const uint64_t key = F.key[i];
+    const int sh = 21 - B.Lc;
+    cc[0] = (int)(compact3(key >> 2) >> sh);
+    cc[1] = (int)(compact3(key >> 1) >> sh);
+    cc[2] = (int)(compact3(key) >> sh);
+    ckey = (uint32_t)(key >> (3 * sh));
+  }
   int cnt = 0;
 
-  // group size: the whole warp unless its box exceeds kMaxWarpCells cells
+  // group size: the whole warp unless it spans more than kMaxGroupCells distinct
+  // coarse cells (Morton jumps); then halves, quarters, ...
   int g = 32;
-  GroupBox mine = group_box(B, t, active, g);
-  while (g > 1 && __reduce_max_sync(0xffffffffu, mine.T) > kMaxWarpCells) {
+  uint32_t leaders;
+  while (true) {
+    const unsigned long long tag =
+        active ? (((unsigned long long)(lane / g)) << 32) | ckey : (0xffffffff00000000ull | (unsigned)lane);
+    const uint32_t peers = __match_any_sync(0xffffffffu, tag);
+    const bool lead = active && (peers & ((1u << lane) - 1u)) == 0;
+    leaders = __ballot_sync(0xffffffffu, lead);
+    const uint32_t gm = (g == 32) ? 0xffffffffu : (((1u << g) - 1u) << ((lane / g) * g));
+    const int D = __popc(leaders & gm);
+    if (g == 1 || __reduce_max_sync(0xffffffffu, D) <= kMaxGroupCells) break;
     g >>= 1;
-    mine = group_box(B, t, active, g);
   }
   for (int gid = 0; gid < 32 / g; ++gid) {
-    const int src = gid * g;
-    GroupBox G;
-#pragma unroll
-    for (int a = 0; a < 3; ++a) {
-      G.lo[a] = __shfl_sync(0xffffffffu, mine.lo[a], src);
-      G.ext[a] = __shfl_sync(0xffffffffu, mine.ext[a], src);
-      G.full[a] = __shfl_sync(0xffffffffu, (int)mine.full[a], src) != 0;
-    }
-    G.T = __shfl_sync(0xffffffffu, mine.T, src);
-    if (G.T == 0) continue;
+    const uint32_t gm = (g == 32) ? 0xffffffffu : (((1u << g) - 1u) << (gid * g));
+    const uint32_t gl = leaders & gm;
+    if (!gl) continue;
+    const GroupBox G = build_cells(B, cc, gl, lane, s_w[warp]);
     Target tg = t;
     if (lane / g != gid) tg.r_out2 = tg.r_in2 = tg.rc = -1.f;  // not in this pass
     if (G.full[0] || G.full[1] || G.full[2])

@@ -41,6 +41,8 @@ struct DevScalars {
   int status;
   int max_nc, min_nc;
   unsigned long long total_nc;
+  unsigned long long cand_total;  // neighbour-search candidates streamed (diagnostic)
+  unsigned long long pass_total;  // warp passes of the neighbour search (diagnostic)
   double t, dt, dt_prev;
   int first;
   int pad;

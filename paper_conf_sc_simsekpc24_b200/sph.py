@@ -54,7 +54,7 @@ class Config(C.Structure):
 
 class NbrStats(C.Structure):
     _fields_ = [("min_nc", C.c_int32), ("max_nc", C.c_int32), ("mean_nc", C.c_double),
-                ("total", C.c_int64)]
+                ("total", C.c_int64), ("candidates", C.c_int64), ("passes", C.c_int64)]
 
 
 class StepInfo(C.Structure):
@@ -299,6 +299,7 @@ class Simulation:
         self._ok(self.L.sph_step(self.ctx, C.byref(info)))
         return {"t": info.t, "dt": info.dt, "min_nc": info.nbr.min_nc, "max_nc": info.nbr.max_nc,
                 "mean_nc": info.nbr.mean_nc, "cell_level": info.cell_level,
+                "search_candidates": info.nbr.candidates, "search_passes": info.nbr.passes,
                 "phase_ms": {PHASES[p]: info.phase_ms[p] for p in range(NPHASES)}}
 
     # ---------------------------------------------------------------- energy / clocks
