@@ -283,10 +283,14 @@ int sph_set_accounting(sph_ctx* ctx, int mode);
  * for the bench's launch count. */
 int sph_kernel_launches(int64_t* count);
 
-/* Re-runs one pure phase (NEIGHBORS, DENSITY, EOS, IAD, MOMENTUM_ENERGY) reps
- * times back to back on the same inputs -- the KernelTuner-style isolated
- * measurement of P:81-87 -- and returns its mean time and energy per call
- * (joules < 0 when NVML is unavailable).  Synchronises. */
+/* Re-runs one phase reps times back to back on the same inputs -- the
+ * KernelTuner-style isolated measurement of P:81-87 -- and returns its mean time
+ * and energy per call (joules < 0 when NVML is unavailable).  Repeatable phases
+ * leave the pipeline state unchanged: KEYS (into a spare key buffer), SORT
+ * (re-sorts the sorted keys, permutes into the spare state buffer), CELLS,
+ * NEIGHBORS, DENSITY, EOS, IAD, MOMENTUM_ENERGY, TIMESTEP; UPDATE is not
+ * (SPH_ERR_ARG).  The NVML energy counter of a B200 advances about every 100 ms,
+ * so reps should make the call last >= 1 s.  Synchronises. */
 int sph_repeat_phase(sph_ctx* ctx, int phase, int reps, double* ms_per_call,
                      double* joules_per_call);
 

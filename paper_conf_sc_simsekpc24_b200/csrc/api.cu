@@ -795,12 +795,16 @@ int sph_kernel_launches(int64_t* count) {
 int sph_repeat_phase(sph_ctx* c, int phase, int reps, double* ms_per_call, double* joules_per_call) {
   int need;
   switch (phase) {
+    case SPH_PHASE_KEYS: need = S_TREE; break;
+    case SPH_PHASE_SORT: need = S_TREE; break;
+    case SPH_PHASE_CELLS: need = S_TREE; break;
     case SPH_PHASE_NEIGHBORS: need = S_TREE; break;
     case SPH_PHASE_DENSITY: need = S_NBR; break;
     case SPH_PHASE_EOS: need = S_DENS; break;
     case SPH_PHASE_IAD: need = S_EOS; break;
     case SPH_PHASE_MOMENTUM_ENERGY: need = S_IAD; break;
-    default: return fail(c, SPH_ERR_ARG, "phase %d is not a pure phase", phase);
+    case SPH_PHASE_TIMESTEP: need = S_DT; break;
+    default: return fail(c, SPH_ERR_ARG, "phase %d is not repeatable (it changes the state)", phase);
   }
   int rc = check_ready(c, need, "sph_repeat_phase");
   if (rc) return rc;
@@ -815,8 +819,29 @@ int sph_repeat_phase(sph_ctx* c, int phase, int reps, double* ms_per_call, doubl
   bool eok = c->nvml.energy_mj(&e0);
   cudaEventRecord(a, c->st);
   Fields F = fields(c);
+  // KEYS writes into the key buffer not holding the sorted keys; SORT re-sorts
+  // the (already sorted) keys in place and permutes into the spare state buffer
+  // without switching to it: both leave the pipeline state unchanged.
+  uint64_t* spare_keys = c->key_sorted == c->keyA ? c->keyB : c->keyA;
+  Fields Fk = F;
+  Fk.key = spare_keys;
+  const int prv = c->cur;
   for (int r = 0; r < reps; ++r) {
     switch (phase) {
+      case SPH_PHASE_KEYS: launch_box_keys(Fk, c->P, c->st); break;
+      case SPH_PHASE_SORT: {
+        uint32_t* perm = nullptr;
+        uint64_t* ks = nullptr;
+        launch_sort(F, c->key_sorted, spare_keys, c->valA, c->valB, c->sort_hist, c->sort_status,
+                    c->status_bytes, &perm, &ks, c->st);
+        c->cur = prv ^ 1;
+        Fields Fd = fields(c);
+        c->cur = prv;
+        launch_permute(Fd, perm, c->state[prv], c->ids[prv], c->st);
+        break;
+      }
+      case SPH_PHASE_CELLS: launch_cells(F, c->P, c->level_cap, c->st); break;
+      case SPH_PHASE_TIMESTEP: launch_timestep(F, c->P, c->st); break;
       case SPH_PHASE_NEIGHBORS: launch_neighbors(F, c->P, c->st); break;
       case SPH_PHASE_DENSITY: launch_density(F, c->P, c->st); break;
       case SPH_PHASE_EOS: launch_eos(F, c->P, c->st); break;
