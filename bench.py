@@ -288,8 +288,17 @@ def main():
     pairs = mean_nc * n
     mom_s = statistics.mean(mom_ms) * 1e-3
     achieved = FLOPS_PER_PAIR["momentum_energy"] * pairs / mom_s / 1e12
+    traffic = None
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            traffic = json.load(f)["momentum_energy_kernel"]["dram_bytes_per_launch"]
+    except (OSError, KeyError, ValueError):
+        pass
     roofline = {"bound": "alu", "achieved": achieved, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
-                "frac": achieved / FP64_PEAK_TFLOPS, "traffic": None, "kernel": "momentum_energy_kernel",
+                "frac": achieved / FP64_PEAK_TFLOPS, "traffic": traffic,
+                "traffic_unit": "DRAM bytes per launch (ncu --set full, profiles/ncu_traffic.json)",
+                "algorithmic_bytes_per_launch": (MOM_BYTES_PER_PARTICLE + 4 * mean_nc) * n,
+                "kernel": "momentum_energy_kernel",
                 "peak_source": "148 SM x 64 DFMA/clk x 2 x 1.965 GHz (FP64 pipe; DESIGN.md 6)",
                 "hbm_GBps_algorithmic": (MOM_BYTES_PER_PARTICLE + 4 * mean_nc) * n / mom_s / 1e9,
                 "share_of_step": statistics.mean(mom_ms) / (ms_max / args.steps)}

@@ -7,7 +7,7 @@
 //      histograms (warp-aggregated shared atomics, then global atomics);
 //   2. per pass, one kernel: each CTA takes the next tile id from a global
 //      counter (so every tile it may wait on is already running: forward
-//      progress without co-residency assumptions), ranks its 4096 keys stably
+//      progress without co-residency assumptions), ranks its 2048 keys stably
 //      with warp match/ballot (per-warp digit counters in shared memory),
 //      publishes its digit counts, resolves its global digit offsets by
 //      decoupled look-back over the preceding tiles' published words

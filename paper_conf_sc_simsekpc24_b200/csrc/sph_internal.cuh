@@ -21,8 +21,8 @@ enum StateField { FX = 0, FY, FZ, FVX, FVY, FVZ, FH, FM, FU, FDUM1 };
 
 // Onesweep radix sort geometry (k_sort.cu).
 constexpr int kSortThreads = 256;
-constexpr int kSortKPT = 16;
-constexpr int kSortTile = kSortThreads * kSortKPT;  // 4096 keys per tile
+constexpr int kSortKPT = 8;
+constexpr int kSortTile = kSortThreads * kSortKPT;  // 2048 keys per tile (3 CTAs/SM)
 constexpr int kRadixBits = 8;
 constexpr int kRadix = 256;
 constexpr int kSortPasses = 8;  // 8 x 8 bits >= 63-bit keys
@@ -74,6 +74,7 @@ __device__ __forceinline__ void st4(Rec4* p, double a, double b, double c, doubl
 //   rec_m[5j + 2]  = {C22, C23, C33, m}
 //   rec_m[5j + 3]  = {vx, vy, vz, p/rho^2}
 //   rec_m[5j + 4]  = {h, c, rho, 0}      (read only for approaching pairs)
+// (A chunk-major layout rec_m[k cap + j] was measured: no gain, +14 registers.)
 constexpr int kRecM = 5;
 
 // Everything the kernels need, passed by value.
