@@ -36,9 +36,9 @@ METRIC = "particle-updates/s per SPH step"
 UNIT = "particle-updates/s"
 
 # Algorithmic FP64 flops per neighbour pair, counting
-# add/sub/mul as 1 and fma as 2, sinc as its 13-FMA polynomial; the artificial
-# viscosity's 17 flops (approaching pairs only) are NOT counted (lower bound).
-FLOPS_PER_PAIR = {"density": 40, "iad": 55, "momentum_energy": 157}
+# add/sub/mul as 1 and fma as 2, sinc as its 10-FMA polynomial; the artificial
+# viscosity's flops (approaching pairs only) are NOT counted (lower bound).
+FLOPS_PER_PAIR = {"density": 34, "iad": 49, "momentum_energy": 145}
 # FP64 peak: 148 SMs x 64 FP64 FMA/clk x 2 flop x 1.965 GHz (guide's SM count and
 # max SM clock; DFMA microbenchmark measured 34.1 TF, tools/probe_fp64.cu).
 FP64_PEAK_TFLOPS = 148 * 64 * 2 * 1.965e9 / 1e12

@@ -185,21 +185,25 @@ __global__ void __launch_bounds__(128) momentum_energy_kernel(Fields F, Params P
     const int nci = min(F.nc[i], F.ngmax);
     double ax = 0, ay = 0, az = 0, de = 0;
     const int32_t* __restrict__ nb = F.nbr + i;
-    // software pipeline: neighbour index two ahead, its 4 record chunks one ahead
-    int jn = nci > 1 ? __ldg(nb + F.cap) : 0;
-    const Rec4* rj = rec + (int64_t)kRecM * (nci > 0 ? __ldg(nb) : 0);
-    Rec4 n0 = ldg4(rj), n1 = ldg4(rj + 1), n2 = ldg4(rj + 2), n3 = ldg4(rj + 3);
+    // software pipeline: neighbour index three ahead, the position chunk (needed
+    // first) two ahead; the other chunks are loaded at the top of the iteration
+    // and arrive while the two sinc polynomials run.
+    const int64_t cap = F.cap;
+    const Rec4* r0 = rec + (int64_t)kRecM * (nci > 0 ? __ldg(nb) : 0);
+    const Rec4* r1 = rec + (int64_t)kRecM * (nci > 1 ? __ldg(nb + cap) : 0);
+    int jn = nci > 2 ? __ldg(nb + 2 * cap) : 0;
+    Rec4 p0 = ldg4(r0), p1 = ldg4(r1);
     for (int k = 0; k < nci; ++k) {
-      const Rec4 j0 = n0, j1 = n1, j2 = n2, j3 = n3;
-      const Rec4* rcur = rj;
-      if (k + 1 < nci) {
-        rj = rec + (int64_t)kRecM * jn;
-        n0 = ldg4(rj);
-        n1 = ldg4(rj + 1);
-        n2 = ldg4(rj + 2);
-        n3 = ldg4(rj + 3);
+      const Rec4* rcur = r0;
+      const Rec4 j1 = ldg4(rcur + 1), j2 = ldg4(rcur + 2), j3 = ldg4(rcur + 3);
+      const Rec4 j0 = p0;
+      p0 = p1;
+      r0 = r1;
+      if (k + 2 < nci) {
+        r1 = rec + (int64_t)kRecM * jn;
+        p1 = ldg4(r1);
       }
-      if (k + 2 < nci) jn = __ldg(nb + (int64_t)(k + 2) * F.cap);
+      if (k + 3 < nci) jn = __ldg(nb + (int64_t)(k + 3) * cap);
       double dx, dy, dz;
       pair_d(g, xi, yi, zi, j0.a, j0.b, j0.c, dx, dy, dz);
       const double r2 = dx * dx + dy * dy + dz * dz;
@@ -223,8 +227,12 @@ __global__ void __launch_bounds__(128) momentum_energy_kernel(Fields F, Params P
         const double hbar = 0.5 * (hi + j4.a);
         const double cbar = 0.5 * (ci + j4.b);
         const double rhobar = 0.5 * (rhoi + j4.c);
-        const double mu = hbar * rv / (r2 + eps * hbar * hbar);
-        Pi = (-alpha * cbar * mu + beta * mu * mu) / rhobar;
+        // mu = hbar rv / D, Pi = (-alpha cbar mu + beta mu^2) / rhobar with one
+        // division: q = 1 / (D rhobar), 1/D = rhobar q, 1/rhobar = D q
+        const double D = fma(eps * hbar, hbar, r2);
+        const double q = 1.0 / (D * rhobar);
+        const double mu = hbar * rv * (rhobar * q);
+        Pi = (fma(beta, mu, -alpha * cbar) * mu) * (D * q);
       }
       const double mj = j2.d, prj = j3.d;
       ax -= mj * (pri * Ax + prj * Bx + Pi * Gx);
