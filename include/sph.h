@@ -211,6 +211,24 @@ int sph_get_n(const sph_ctx* ctx, int64_t* n);
  * SPH_F_NC, double otherwise) to dst (host or device).  Synchronises. */
 int sph_get_field(sph_ctx* ctx, int field, void* dst, int mem);
 
+/* Multi-GPU halo support (SFC domain decomposition).  A particle
+ * whose id has bit SPH_GHOST_BIT set is a ghost: a copy of a particle owned by
+ * another rank, present only as a neighbour j.  Its own sums use an incomplete
+ * neighbourhood and are meaningless (the IAD singularity check ignores ghosts);
+ * the owners' values are written over it with sph_set_field:
+ *   after sph_density:  SPH_F_RHO           (then sph_eos derives p, c, V);
+ *   after sph_iad:      SPH_F_C11..SPH_F_C33 (the momentum records are rebuilt).
+ * sph_set_field copies n values (current order) from src; only SPH_F_RHO and
+ * SPH_F_C11..SPH_F_C33 are settable (SPH_ERR_ARG otherwise). */
+#define SPH_GHOST_BIT (1ll << 62)
+int sph_set_field(sph_ctx* ctx, int field, const void* src, int mem);
+
+/* The local min_i h_i/c_i of the last sph_momentum_energy (synchronises), and
+ * the global one (the minimum over ranks, the P:220 collective) to be used by
+ * the next sph_timestep instead. */
+int sph_get_local_min_hc(sph_ctx* ctx, double* min_hc);
+int sph_set_global_min_hc(sph_ctx* ctx, double min_hc);
+
 /* --- the hot path (each call = one accounted phase group) ------------------- */
 
 /* Items 1-3: box (open axes: exact min/max), 63-bit Morton keys, stable LSD

@@ -84,6 +84,7 @@ struct sph_ctx {
   unsigned clock_mhz[SPH_NPHASES];
   unsigned current_lock = 0;
   bool locked_any = false;
+  bool rec_m_dirty = false;
 };
 
 namespace {
@@ -292,6 +293,10 @@ int body_simple(sph_ctx* c, int phase, int next_stage) {
     case SPH_PHASE_EOS: launch_eos(F, c->P, c->st); break;
     case SPH_PHASE_IAD: launch_iad(F, c->P, c->st); break;
     case SPH_PHASE_MOMENTUM_ENERGY:
+      if (c->rec_m_dirty) {  // ghosts' C were overwritten (sph_set_field)
+        launch_refresh_rec_m(F, c->st);
+        c->rec_m_dirty = false;
+      }
       cudaMemsetAsync(&c->ds->minhc_ord, 0xff, sizeof(unsigned long long), c->st);
       launch_momentum_energy(F, c->P, c->st);
       break;
@@ -587,6 +592,58 @@ int sph_get_field(sph_ctx* c, int field, void* dst, int mem) {
   rc = cuda_check(c, cudaStreamSynchronize(c->st), "sync");
   if (!rc) collect_all(c);
   return rc;
+}
+
+int sph_set_field(sph_ctx* c, int field, const void* src, int mem) {
+  int rc = check_ready(c, S_INIT, "sph_set_field");
+  if (rc) return rc;
+  if (!src && c->n > 0) return fail(c, SPH_ERR_ARG, "null src");
+  if (mem != SPH_MEM_HOST && mem != SPH_MEM_DEVICE) return fail(c, SPH_ERR_ARG, "mem must be HOST or DEVICE");
+  double* dst = nullptr;
+  if (field == SPH_F_RHO) {
+    if (c->stage < S_DENS) return fail(c, SPH_ERR_STATE, "sph_set_field(RHO) before sph_density");
+    dst = c->rho;
+  } else if (field >= SPH_F_C11 && field <= SPH_F_C33) {
+    if (c->stage < S_IAD) return fail(c, SPH_ERR_STATE, "sph_set_field(C) before sph_iad");
+    dst = c->C[field - SPH_F_C11];
+    c->rec_m_dirty = true;
+  } else {
+    return fail(c, SPH_ERR_ARG, "field %d is not settable", field);
+  }
+  if (c->n == 0) return SPH_OK;
+  const cudaMemcpyKind kind = mem == SPH_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
+  return cuda_check(c, cudaMemcpyAsync(dst, src, sizeof(double) * c->n, kind, c->st), "set field");
+}
+
+int sph_get_local_min_hc(sph_ctx* c, double* min_hc) {
+  int rc = check_ready(c, S_MOM, "sph_get_local_min_hc");
+  if (rc) return rc;
+  if (!min_hc) return fail(c, SPH_ERR_ARG, "null min_hc");
+  rc = cuda_check(c, cudaMemcpyAsync(&c->h_ds, c->ds, sizeof(DevScalars), cudaMemcpyDeviceToHost, c->st), "copy");
+  if (!rc) rc = cuda_check(c, cudaStreamSynchronize(c->st), "sync");
+  if (rc) return rc;
+  const unsigned long long o = c->h_ds.minhc_ord;
+  if (o == ~0ull) {
+    *min_hc = INFINITY;
+  } else {
+    const unsigned long long b = (o >> 63) ? (o & 0x7fffffffffffffffull) : ~o;
+    memcpy(min_hc, &b, sizeof(double));
+  }
+  return SPH_OK;
+}
+
+__global__ void set_minhc_kernel(DevScalars* ds, unsigned long long o) { ds->minhc_ord = o; }
+
+int sph_set_global_min_hc(sph_ctx* c, double min_hc) {
+  int rc = check_ready(c, S_MOM, "sph_set_global_min_hc");
+  if (rc) return rc;
+  if (!(min_hc > 0)) return fail(c, SPH_ERR_ARG, "min_hc must be > 0");
+  unsigned long long b;
+  memcpy(&b, &min_hc, sizeof(double));
+  const unsigned long long o = b | 0x8000000000000000ull;  // order-preserving code of a positive double
+  set_minhc_kernel<<<1, 1, 0, c->st>>>(c->ds, o);
+  note_launch();
+  return cuda_check(c, cudaSuccess, "set_minhc");
 }
 
 int sph_build_tree(sph_ctx* c) {

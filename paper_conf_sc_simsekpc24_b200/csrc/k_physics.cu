@@ -150,7 +150,10 @@ __global__ void __launch_bounds__(256) iad_kernel(Fields F, Params P) {
   F.C[3][i] = c22;
   F.C[4][i] = c23;
   F.C[5][i] = c33;
-  if (!(det > 0.0) || !isfinite(det)) atomicOr(&F.ds->status, (int)ST_SINGULAR);
+  // ghosts (another rank's particles, SPH_GHOST_BIT in the id) have truncated
+  // neighbourhoods; their C is overwritten by the owner's
+  if ((!(det > 0.0) || !isfinite(det)) && !(F.id[i] & SPH_GHOST_BIT))
+    atomicOr(&F.ds->status, (int)ST_SINGULAR);
   Rec4* rm = F.rec_m + (int64_t)kRecM * i;
   st4(rm + 0, me.a, me.b, me.c, q);
   st4(rm + 1, c11, c12, c13, kh3);
@@ -299,6 +302,22 @@ __global__ void advance_time_kernel(DevScalars* ds) {
   ds->t += ds->dt;
   ds->dt_prev = ds->dt;
   ds->first = 0;
+}
+
+// Rebuilds the C chunks of the momentum records after sph_set_field wrote the
+// owners' C over the ghosts (multi-GPU halo, item 8(e)).
+__global__ void __launch_bounds__(256) refresh_rec_m_kernel(Fields F) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= F.n) return;
+  Rec4* rm = F.rec_m + (int64_t)kRecM * i;
+  st4(rm + 1, F.C[0][i], F.C[1][i], F.C[2][i], F.wk[i]);
+  st4(rm + 2, F.C[3][i], F.C[4][i], F.C[5][i], F.f[FM][i]);
+}
+
+void launch_refresh_rec_m(const Fields& F, cudaStream_t st) {
+  if (F.n == 0) return;
+  refresh_rec_m_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F);
+  note_launch();
 }
 
 // ------------------------------------------------------------------ launchers

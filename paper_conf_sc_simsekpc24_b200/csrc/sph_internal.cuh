@@ -205,4 +205,5 @@ void launch_momentum_energy(const Fields& F, const Params& P, cudaStream_t st);
 void launch_timestep(const Fields& F, const Params& P, cudaStream_t st);
 void launch_update(const Fields& F, const Params& P, cudaStream_t st);
 void launch_advance_time(const Fields& F, cudaStream_t st);
+void launch_refresh_rec_m(const Fields& F, cudaStream_t st);
 }  // namespace sph

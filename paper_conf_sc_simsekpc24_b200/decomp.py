@@ -1,0 +1,278 @@
+"""Multi-GPU SPH step: space-filling-curve domain decomposition with halo
+exchange ("domain decomposition, halo exchanges",
+P:216 DomainDecompAndSync, P:220 the end-of-step collective for dt).
+
+One process per GPU.  Every rank owns a contiguous range of the 63-bit Morton
+curve; the split points come from a global histogram of the top key bits
+(all-reduce).  Each step:
+
+  1. keys of the local particles (libsph sph_build_tree), migration of the
+     particles whose key left the rank's range (all-to-all);
+  2. ghosts: every local particle within 2 h_max (minimum image) of another
+     rank's domain box is sent to it (all-to-all) with SPH_GHOST_BIT in its id;
+  3. the full hot path in libsph on locals + ghosts, with two halo refreshes of
+     the owners' values over the ghosts: rho after DENSITY (then EOS derives
+     p, c, V) and C after IAD (H2, H3 of SURVEY 8(e));
+  4. dt = global min over ranks (all-reduce), update, ghosts dropped.
+
+The held set is sorted in the global Morton order and every target's
+neighbours are the same particles as in a single-GPU run, so for a periodic box
+the result is bit-identical to the one-GPU step (tests/test_gpu_decomp.py).
+
+The data-path collectives are torch.distributed calls on device tensors (NCCL
+over NVLink on GPUs; gloo on host tensors in the CPU tests).  All arithmetic of
+the method stays in libsph; this module moves particles and values between
+ranks and selects which to move (plumbing).
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+GHOST_BIT = 1 << 62
+STATE = ("x", "y", "z", "vx", "vy", "vz", "h", "m", "u", "du_m1")
+HIST_BITS = 15  # SFC partition granularity: 2^15 bins of the top key bits
+
+
+# ----------------------------------------------------------------------------- comm
+class Comm:
+    """Collectives over the default process group; host tensors for gloo."""
+
+    def __init__(self):
+        self.rank = dist.get_rank() if dist.is_initialized() else 0
+        self.world = dist.get_world_size() if dist.is_initialized() else 1
+        self.host = (dist.get_backend() == "gloo") if dist.is_initialized() else True
+
+    def _to(self, t):
+        return t.cpu() if self.host else t
+
+    def all_reduce(self, t, op):
+        if self.world == 1:
+            return t
+        x = self._to(t.clone())
+        dist.all_reduce(x, op=op)
+        return x.to(t.device)
+
+    def all_gather(self, t):
+        if self.world == 1:
+            return [t]
+        x = self._to(t.contiguous())
+        out = [torch.empty_like(x) for _ in range(self.world)]
+        dist.all_gather(out, x)
+        return [o.to(t.device) for o in out]
+
+    def alltoallv(self, parts):
+        """parts[r]: tensor [n_r, ...] for rank r -> list of received [m_s, ...]."""
+        if self.world == 1:
+            return [parts[0]]
+        dev = parts[0].device
+        tail = tuple(parts[0].shape[1:])
+        width = int(np.prod(tail)) if tail else 1
+        cdev = torch.device("cpu") if self.host else dev
+        counts = torch.tensor([p.shape[0] for p in parts], dtype=torch.int64, device=cdev)
+        rc = torch.empty_like(counts)
+        dist.all_to_all_single(rc, counts)
+        counts, rc = counts.cpu(), rc.cpu()
+        send = self._to(torch.cat([p.reshape(-1, width) for p in parts], 0).reshape(-1))
+        recv = torch.empty(int(rc.sum()) * width, dtype=send.dtype, device=send.device)
+        dist.all_to_all_single(recv, send, [int(c) * width for c in rc],
+                               [int(c) * width for c in counts])
+        recv = recv.to(dev).reshape((-1,) + tail)
+        return list(torch.split(recv, [int(c) for c in rc], 0))
+
+
+# ----------------------------------------------------------------------------- partition
+def sfc_splits(keys, comm: Comm, bits: int = HIST_BITS):
+    """Split bins of the global key histogram: rank r owns bins [s[r], s[r+1])."""
+    nb = 1 << bits
+    b = (keys >> (63 - bits)).to(torch.int64)
+    hist = torch.bincount(b, minlength=nb).to(torch.int64)
+    hist = comm.all_reduce(hist, dist.ReduceOp.SUM if comm.world > 1 else None)
+    cum = torch.cumsum(hist, 0)
+    total = int(cum[-1])
+    targets = torch.tensor([total * r // comm.world for r in range(1, comm.world)], dtype=torch.int64,
+                           device=cum.device)
+    inner = torch.searchsorted(cum, targets, right=True)  # first bin past each quota
+    s = torch.cat([torch.zeros(1, dtype=torch.int64, device=cum.device), inner,
+                   torch.full((1,), nb, dtype=torch.int64, device=cum.device)])
+    return s
+
+
+def owners(keys, splits, bits: int = HIST_BITS):
+    b = (keys >> (63 - bits)).to(torch.int64)
+    return torch.searchsorted(splits, b, right=True) - 1
+
+
+def domain_boxes(x, comm: Comm):
+    """[world, 2, 3] bounding boxes (min, max) of every rank's particles."""
+    if x.shape[0]:
+        lo, hi = x.min(0).values, x.max(0).values
+    else:
+        lo = torch.full((3,), float("inf"), dtype=x.dtype, device=x.device)
+        hi = torch.full((3,), -float("inf"), dtype=x.dtype, device=x.device)
+    return torch.stack(comm.all_gather(torch.stack([lo, hi])))
+
+
+def box_distance(x, lo, hi, box_len, periodic):
+    """Minimum-image distance of points x [n,3] to the axis-aligned box [lo, hi]."""
+    d2 = torch.zeros(x.shape[0], dtype=x.dtype, device=x.device)
+    for a in range(3):
+        if periodic[a]:
+            best = None
+            for k in (-1.0, 0.0, 1.0):
+                xa = x[:, a] + k * box_len[a]
+                da = torch.clamp(torch.maximum(lo[a] - xa, xa - hi[a]), min=0.0)
+                best = da if best is None else torch.minimum(best, da)
+        else:
+            best = torch.clamp(torch.maximum(lo[a] - x[:, a], x[:, a] - hi[a]), min=0.0)
+        d2 = d2 + best * best
+    return torch.sqrt(d2)
+
+
+def ghost_masks(x, boxes, rank, radius, box_len, periodic):
+    """masks[r]: local particles within `radius` of rank r's domain box (r != rank)."""
+    out = []
+    for r in range(boxes.shape[0]):
+        if r == rank or not torch.isfinite(boxes[r]).all():
+            out.append(torch.zeros(x.shape[0], dtype=torch.bool, device=x.device))
+            continue
+        out.append(box_distance(x, boxes[r, 0], boxes[r, 1], box_len, periodic) < radius)
+    return out
+
+
+# ----------------------------------------------------------------------------- rows
+def pack(state, idx=None):
+    """Particles as rows [n, 11] of float64 (id bit-cast into the last column)."""
+    cols = [state[k] if idx is None else state[k][idx] for k in STATE]
+    ids = state["id"] if idx is None else state["id"][idx]
+    return torch.cat([torch.stack(cols, 1), ids.view(torch.float64).unsqueeze(1)], 1)
+
+
+def unpack(rows):
+    st = {k: rows[:, c].contiguous() for c, k in enumerate(STATE)}
+    st["id"] = rows[:, len(STATE)].contiguous().view(torch.int64)
+    return st
+
+
+def positions_of(ids_current, query):
+    """Positions in the current order of the particles with ids `query`."""
+    order = torch.argsort(ids_current)
+    srt = ids_current[order]
+    p = torch.searchsorted(srt, query)
+    assert bool((srt[p.clamp(max=srt.numel() - 1)] == query).all()), "halo id not found"
+    return order[p]
+
+
+# ----------------------------------------------------------------------------- stepping
+class DistributedSim:
+    """One rank of the decomposed simulation.  `state` holds this rank's share of
+    the particles (torch tensors on its GPU)."""
+
+    def __init__(self, params, state, n_capacity: int, device: int = 0, **kw):
+        from . import sph
+        self.sph = sph
+        self.params = params
+        self.comm = Comm()
+        self.dev = torch.device("cuda", device)
+        self.sim = sph.Simulation(params, n_capacity=n_capacity, device=device, **kw)
+        self.local = {k: torch.as_tensor(np.ascontiguousarray(v)).to(self.dev) for k, v in state.items()}
+        self.box_len = [float(b - a) for a, b in zip(params.box_min, params.box_max)]
+        self.t, self.dt_prev, self.first = 0.0, float(params.dt_first), True
+        self.stats = {}
+
+    def _field(self, name, dtype=torch.float64):
+        out = torch.empty(self.sim.n, dtype=dtype, device=self.dev)
+        self.sim.get_field(name, out=out)
+        return out
+
+    def _held_state(self):
+        st = {k: self._field(k) for k in STATE}
+        st["id"] = self._field("id", torch.int64)
+        return st
+
+    def _load(self, st):
+        self.sim.set_particles({k: st[k].contiguous() for k in STATE + ("id",)})
+        self.sim.set_time(self.t, self.dt_prev, self.first)
+
+    def step(self):
+        comm, sim = self.comm, self.sim
+        # 1. keys of the locals, SFC partition, migration
+        self._load(self.local)
+        sim.build_tree()
+        st = self._held_state()
+        keys = self._field("key", torch.int64)
+        splits = sfc_splits(keys, comm)
+        own = owners(keys, splits)
+        rows = pack(st)
+        parts = [rows[own == r] for r in range(comm.world)]
+        local = unpack(torch.cat(comm.alltoallv(parts), 0))
+        # 2. ghosts within 2 h_max of every other rank's domain box
+        x = torch.stack([local["x"], local["y"], local["z"]], 1)
+        hmax = comm.all_reduce(local["h"].max().reshape(1) if local["h"].numel() else
+                               torch.zeros(1, dtype=torch.float64, device=self.dev),
+                               dist.ReduceOp.MAX if comm.world > 1 else None)
+        boxes = domain_boxes(x, comm)
+        radius = float(2.0 * hmax.item()) * (1.0 + 1e-9)
+        masks = ghost_masks(x, boxes, comm.rank, radius, self.box_len, self.params.periodic)
+        lrows = pack(local)
+        sent_ids = [local["id"][m] for m in masks]
+        gparts = []
+        for m in masks:
+            g = lrows[m].clone()
+            g[:, len(STATE)] = (local["id"][m] | GHOST_BIT).view(torch.float64)
+            gparts.append(g)
+        recv = comm.alltoallv(gparts)
+        ghost_ids = [unpack(r)["id"] for r in recv]
+        held = unpack(torch.cat([lrows] + list(recv), 0))
+        self.stats = {"n_local": int(local["x"].numel()),
+                      "n_ghost": int(sum(r.shape[0] for r in recv))}
+        # 3. the hot path with two halo refreshes
+        self._load(held)
+        sim.build_tree()
+        sim.find_neighbors(stats=False)
+        sim.density()
+        ids_now = self._field("id", torch.int64)
+        src_pos = [positions_of(ids_now, s) for s in sent_ids]        # my particles others hold
+        dst_pos = [positions_of(ids_now, g) for g in ghost_ids]       # their particles I hold
+        self._halo(["rho"], src_pos, dst_pos)
+        sim.eos()
+        sim.iad()
+        self._halo(["c11", "c12", "c13", "c22", "c23", "c33"], src_pos, dst_pos)
+        sim.momentum_energy()
+        # 4. global dt, update, drop ghosts
+        mhc = torch.tensor([sim.get_local_min_hc()], dtype=torch.float64, device=self.dev)
+        mhc = comm.all_reduce(mhc, dist.ReduceOp.MIN if comm.world > 1 else None)
+        sim.set_global_min_hc(float(mhc.item()))
+        dt = sim.timestep()
+        sim.update()
+        self.t, self.dt_prev, self.first = self.t + dt, dt, False
+        st = self._held_state()
+        keep = (st["id"] & GHOST_BIT) == 0
+        self.local = {k: v[keep].contiguous() for k, v in st.items()}
+        return dt
+
+    def _halo(self, names, src_pos, dst_pos):
+        if self.comm.world == 1:
+            return
+        vals = {k: self._field(k) for k in names}
+        parts = [torch.stack([vals[k][p] for k in names], 1) for p in src_pos]
+        recv = self.comm.alltoallv(parts)
+        for r, (rv, p) in enumerate(zip(recv, dst_pos)):
+            for c, k in enumerate(names):
+                vals[k][p] = rv[:, c]
+        for k in names:
+            self.sim.set_field(k, vals[k])
+
+    def gather_state(self):
+        """All particles on every rank, sorted by id (host numpy) -- for tests."""
+        rows = pack(self.local)
+        n = torch.tensor([rows.shape[0]], dtype=torch.int64, device=self.dev)
+        ns = [int(v.item()) for v in self.comm.all_gather(n)]
+        m = max(ns)
+        pad = torch.zeros((m, rows.shape[1]), dtype=rows.dtype, device=self.dev)
+        pad[:rows.shape[0]] = rows
+        allr = torch.cat([a[:k] for a, k in zip(self.comm.all_gather(pad), ns)], 0)
+        st = unpack(allr)
+        order = torch.argsort(st["id"])
+        return {k: v[order].cpu().numpy() for k, v in st.items()}

@@ -76,7 +76,9 @@ EXPORTS = ("sph_config_default", "sph_workspace_size", "sph_init", "sph_finalize
            "sph_get_neighbors", "sph_density", "sph_eos", "sph_iad", "sph_momentum_energy",
            "sph_timestep", "sph_update", "sph_step", "sph_set_clock_policy",
            "sph_energy_report", "sph_energy_reset", "sph_energy_counter_mj", "sph_repeat_phase",
-           "sph_set_accounting", "sph_kernel_launches")
+           "sph_set_accounting", "sph_kernel_launches", "sph_set_field",
+           "sph_get_local_min_hc", "sph_set_global_min_hc")
+GHOST_BIT = 1 << 62
 
 _lib = None
 
@@ -120,6 +122,9 @@ def load(build_if_missing: bool = True):
     L.sph_energy_counter_mj.argtypes = [P, C.POINTER(C.c_uint64)]
     L.sph_repeat_phase.argtypes = [P, I, I, C.POINTER(D), C.POINTER(D)]
     L.sph_set_accounting.argtypes = [P, I]
+    L.sph_set_field.argtypes = [P, I, V, I]
+    L.sph_get_local_min_hc.argtypes = [P, C.POINTER(D)]
+    L.sph_set_global_min_hc.argtypes = [P, D]
     L.sph_kernel_launches.argtypes = [C.POINTER(I64)]
     _lib = L
     return L
@@ -233,6 +238,8 @@ class Simulation:
                     raise ValueError("all arrays must live in the same memory kind")
             ptrs.append(C.c_void_p(p) if p is not None else None)
         self._keep = state  # host buffers must outlive the async copies
+        if mem == MEM_DEVICE:  # inputs produced on torch's stream: order libsph's copy after them
+            self.stream.wait_stream(self.torch.cuda.current_stream(self.device))
         self._ok(self.L.sph_set_particles(self.ctx, n, *ptrs, mem if mem is not None else MEM_HOST))
         self.n = n
 
@@ -249,8 +256,26 @@ class Simulation:
         if out is None:
             out = np.empty(self.n, dtype=dt)
         p, mem = _ptr(out)
+        if mem == MEM_DEVICE:  # the destination may be memory torch's stream still uses
+            self.stream.wait_stream(self.torch.cuda.current_stream(self.device))
         self._ok(self.L.sph_get_field(self.ctx, FIELD_ID[name], C.c_void_p(p), mem))
         return out
+
+    def set_field(self, name: str, src):
+        """Overwrite RHO or C11..C33 (n values, current order) -- multi-GPU halo."""
+        p, mem = _ptr(src)
+        if mem == MEM_DEVICE:
+            self.stream.wait_stream(self.torch.cuda.current_stream(self.device))
+        self._keep_field = src
+        self._ok(self.L.sph_set_field(self.ctx, FIELD_ID[name], C.c_void_p(p), mem))
+
+    def get_local_min_hc(self) -> float:
+        v = C.c_double()
+        self._ok(self.L.sph_get_local_min_hc(self.ctx, C.byref(v)))
+        return v.value
+
+    def set_global_min_hc(self, v: float):
+        self._ok(self.L.sph_set_global_min_hc(self.ctx, float(v)))
 
     def get_state(self):
         return {k: self.get_field(k) for k in ("x", "y", "z", "vx", "vy", "vz", "h", "m", "u",
