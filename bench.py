@@ -229,6 +229,93 @@ def run_reference(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
+def run_decomposed(args, rank, world, local):
+    """N > 1: SFC domain decomposition with halo exchange over NCCL (decomp.py),
+    weak scaling: turbulence with ~8M particles per GPU in one periodic box
+    (nside = round(200 N^(1/3)): 252^3, 317^3, 400^3 at N = 2, 4, 8 -- SURVEY
+    8(d) config 5).  Each rank draws its slice of the initial conditions."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_simsekpc24_b200 import decomp, ics, sph
+
+    base = int(args.workload[len("turbulence"):]) if args.workload.startswith("turbulence") else 200
+    nside = int(round(base * world ** (1.0 / 3.0)))
+    w = ics.turbulence_part(nside, rank, world)
+    vsq = torch.tensor([w.meta["vsq_sum"]], dtype=torch.float64, device="cuda")
+    dist.all_reduce(vsq)
+    ics.normalise_velocity(w, float(vsq.item()))
+    n_total = nside ** 3
+    cap = int(1.4 * n_total / world) + 1024
+    ds = decomp.DistributedSim(w.params, w.state, n_capacity=cap, device=local)
+    del w
+
+    def barrier():
+        dist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(args.warmup):
+        ds.step()
+    barrier()
+    l0 = sph.kernel_launches()
+    ds.sim.energy_reset()
+    e_start = ds.sim.energy_counter_mj()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        barrier()
+        ev0.record()
+        for _ in range(args.steps):
+            ds.step()
+        ev1.record()
+        barrier()
+    e_end = ds.sim.energy_counter_mj()
+    ms = torch.tensor([ev0.elapsed_time(ev1)], device="cuda")
+    dist.all_reduce(ms, op=dist.ReduceOp.MAX)
+    ms_max = float(ms.item())
+    rows = ds.sim.energy_report()
+    phase_ms = {r["name"]: 1e3 * r["seconds"] / args.steps for r in rows}
+    joules = torch.tensor([(e_end - e_start) * 1e-3 if e_start is not None and e_end is not None else 0.0],
+                          device="cuda", dtype=torch.float64)
+    dist.all_reduce(joules)
+    ghosts = torch.tensor([ds.stats["n_ghost"], ds.stats["n_local"]], device="cuda", dtype=torch.float64)
+    dist.all_reduce(ghosts)
+    launches = sph.kernel_launches() - l0
+    # e2e: each rank's particles copied in from pinned host memory and back out every step
+    host = {k: v.cpu().pin_memory() for k, v in ds.local.items()}
+    h2d = d2h = 0
+    barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(max(args.e2e_steps, 1)):
+        ds.local = {k: v.to("cuda", non_blocking=True) for k, v in host.items()}
+        h2d = sum(v.numel() * v.element_size() for v in host.values())
+        ds.step()
+        host = {k: v.to("cpu") for k, v in ds.local.items()}
+        d2h = sum(v.numel() * v.element_size() for v in host.values())
+    e1.record()
+    barrier()
+    ems = torch.tensor([e0.elapsed_time(e1)], device="cuda")
+    dist.all_reduce(ems, op=dist.ReduceOp.MAX)
+    if rank == 0:
+        value = n_total * args.steps / (ms_max * 1e-3)
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "config": {"workload": f"turbulence{nside}", "n_particles_total": n_total,
+                           "n_particles_per_gpu": n_total / world,
+                           "parallelism": f"SFC domain decomposition over {world} GPUs, halo exchange (NCCL)",
+                           "ghost_fraction": float(ghosts[0] / ghosts[1]),
+                           "l2": "inputs >> 126 MB L2; no flush"},
+                "phase_ms_rank0": phase_ms, "roofline": None,
+                "e2e": {"value": n_total * max(args.e2e_steps, 1) / (float(ems.item()) * 1e-3), "unit": UNIT,
+                        "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": d2h * world,
+                        "path": "rank-local state from pinned host -> DistributedSim.step -> host"},
+                "energy": {"J_per_step_all_gpus": float(joules.item()) / args.steps,
+                           "uJ_per_particle_update": float(joules.item()) / args.steps / n_total * 1e6},
+                "cpu_baseline": None, "clocks": clk.summary(), "gpu_launches": launches}
+        print(json.dumps(line), flush=True)
+    dist.destroy_process_group()
+
+
 def main():
     args = parse()
     rank, world, local = dist_env()
@@ -240,9 +327,17 @@ def main():
     import torch.distributed as dist
     from paper_conf_sc_simsekpc24_b200 import sph
 
-    torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", init_method="env://")
+        # SPH_DIST_BACKEND=gloo lets several ranks share one GPU (tests); NCCL otherwise
+        backend = os.environ.get("SPH_DIST_BACKEND", "nccl")
+        local = local % torch.cuda.device_count()
+        torch.cuda.set_device(local)
+        if backend == "nccl":
+            dist.init_process_group("nccl", init_method="env://", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend, init_method="env://")
+        return run_decomposed(args, rank, world, local)
+    torch.cuda.set_device(local)
     w = make_workload(args.workload, rank)
     n = w.n
     sim = sph.Simulation(w.params, n_capacity=n, device=local)

@@ -169,6 +169,59 @@ def turbulence(nside: int, v_rms: float = 0.3, jitter: float = 0.25, seed_pos: i
     return Workload(f"turbulence{nside}", st, p, {"nside": nside, "lattice_a": a})
 
 
+def turbulence_part(nside: int, rank: int, world: int, v_rms: float = 0.3, jitter: float = 0.25,
+                    seed_pos: int = 1, seed_vel: int = 2, chunk: int = 1 << 19) -> Workload:
+    """Particles [rank N/world, (rank+1) N/world) of ``turbulence(nside)``, drawn
+    without generating the rest (multi-GPU runs): the jitter stream is advanced
+    to the slice (PCG64 draws one 64-bit word per double) and the velocity field
+    is a function of position.  The velocities come back unnormalised: the
+    scale to v_rms needs the mean square over ALL particles, so every rank
+    reports its slice's sum (meta["vsq_sum"]), the caller all-reduces it and
+    applies ``normalise_velocity``.  Positions and ids equal the full
+    generator's; velocities agree to rounding of the normalisation."""
+    n = nside ** 3
+    lo, hi = rank * n // world, (rank + 1) * n // world
+    a = 1.0 / nside
+    idx = np.arange(lo, hi, dtype=np.int64)
+    g = -0.5 + (np.arange(nside, dtype=np.float64) + 0.5) * a
+    ix, iy, iz = idx // (nside * nside), (idx // nside) % nside, idx % nside
+    pos = [g[ix].copy(), g[iy].copy(), g[iz].copy()]
+    for axis in range(3):
+        bg = np.random.PCG64(seed_pos)
+        bg.advance(axis * n + lo)
+        pos[axis] += np.random.Generator(bg).uniform(-jitter * a, jitter * a, hi - lo)
+    ns, amps, phases = _solenoidal_modes(seed_vel)
+    k = 2.0 * math.pi * ns
+
+    def field(xx, yy, zz):
+        arg = np.outer(k[:, 0], xx) + np.outer(k[:, 1], yy) + np.outer(k[:, 2], zz)
+        arg += phases[:, None]
+        return amps.T @ np.cos(arg)
+
+    v = np.zeros((3, hi - lo))
+    for s in range(0, hi - lo, chunk):
+        e = min(hi - lo, s + chunk)
+        v[:, s:e] = field(pos[0][s:e], pos[1][s:e], pos[2][s:e])
+    # the full generator normalises by the rms over ALL jittered particles; the
+    # partial one needs that global number: every rank computes it from its own
+    # slice, and the caller (decomposed run) combines them (`vrms_partial`).
+    p = StepParams(eos=1, cs0=1.0, dt_first=1e-4, h_cap=0.25)
+    st = _state(pos[0], pos[1], pos[2], v[0].copy(), v[1].copy(), v[2].copy(), h_initial(n, p.ng0),
+                1.0 / n, np.full(hi - lo, 1.5))
+    st["id"] = idx.copy()
+    return Workload(f"turbulence{nside}[{rank}/{world}]", st, p,
+                    {"nside": nside, "lattice_a": a, "vsq_sum": float((v * v).sum()), "n_total": n,
+                     "v_rms": v_rms})
+
+
+def normalise_velocity(w: Workload, vsq_sum_total: float):
+    """Scale a ``turbulence_part`` slice with the global mean square velocity."""
+    n = w.meta["n_total"]
+    f = w.meta["v_rms"] / math.sqrt(vsq_sum_total / n)
+    for k in ("vx", "vy", "vz"):
+        w.state[k] = w.state[k] * f
+
+
 def random_box(n: int, seed: int = 0, periodic: bool = True, h: float | None = None,
                v_scale: float = 0.1) -> Workload:
     """Uniform random particles (edge-case tests: ragged sizes, empty cells, ties)."""

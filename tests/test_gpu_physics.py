@@ -1,0 +1,42 @@
+"""Physics of the GPU step over many steps (SURVEY 8(c) pins 'Sedov' and
+'Integrator'): the Sedov blast radius follows the similarity solution
+R(t) = xi0 (E t^2 / rho0)^(1/5), xi0 = 1.1517 for gamma = 5/3, and total energy
+sum m (v^2/2 + u) is conserved to 1e-3 over the run."""
+import numpy as np
+import pytest
+
+from paper_conf_sc_simsekpc24_b200 import ics
+
+pytestmark = pytest.mark.gpu
+
+
+def _energy(st):
+    return float((st["m"] * (0.5 * (st["vx"] ** 2 + st["vy"] ** 2 + st["vz"] ** 2) + st["u"])).sum())
+
+
+def test_sedov_blast_radius_and_energy(golden):
+    from paper_conf_sc_simsekpc24_b200 import sph
+    w = ics.sedov(40)
+    sim = sph.Simulation(w.params, n_capacity=w.n)
+    sim.set_particles({k: np.ascontiguousarray(v) for k, v in w.state.items()})
+    sim.set_time(0.0, w.params.dt_first, True)
+    E0 = _energy(w.state)
+    t = 0.0
+    steps = 0
+    while t < 0.05 and steps < 2000:
+        t = sim.step()["t"]
+        steps += 1
+    st = sim.get_state()
+    E1 = _energy(st)
+    assert abs(E1 - E0) / E0 < 1e-3, (E0, E1)
+    rho = sim.get_field("rho")  # density of the last step's (pre-update) positions, same order
+    r = np.sqrt(st["x"] ** 2 + st["y"] ** 2 + st["z"] ** 2)
+    # shock position: the radius of the density peak, averaged over the shell of
+    # the 200 densest particles
+    top = np.argsort(rho)[-200:]
+    R_num = float(np.median(r[top]))
+    xi0 = golden["sedov_xi0_gamma53"]["value"]
+    R_th = xi0 * (1.0 * t * t / 1.0) ** 0.2
+    assert abs(R_num - R_th) / R_th < 0.12, (R_num, R_th, t, steps)
+    # strong-shock compression: the peak density is well above ambient
+    assert rho[top].mean() > 2.0

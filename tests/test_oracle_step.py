@@ -86,3 +86,18 @@ def test_sample_step_lattice100(golden):
     assert np.allclose(smp["C"][:, 0], 1.0 / golden["lattice100_tau11"]["value"], rtol=1e-12)
     assert np.allclose(smp["rho"], golden["lattice_rho"]["value"], rtol=1e-14)
     assert smp["dt"] == pytest.approx(1.1e-6, rel=1e-15)
+
+
+def test_turbulence_slices_equal_the_full_generator():
+    """The multi-GPU IC slices reproduce the single-GPU input (positions, ids
+    exactly; velocities to the rounding of the global normalisation)."""
+    full = ics.turbulence(12)
+    parts = [ics.turbulence_part(12, r, 3) for r in range(3)]
+    vsq = sum(p.meta["vsq_sum"] for p in parts)
+    for p in parts:
+        ics.normalise_velocity(p, vsq)
+    cat = {k: np.concatenate([p.state[k] for p in parts]) for k in full.state}
+    for k in ("x", "y", "z", "h", "m", "u", "id"):
+        assert np.array_equal(cat[k], full.state[k]), k
+    for k in ("vx", "vy", "vz"):
+        assert np.allclose(cat[k], full.state[k], rtol=1e-14, atol=1e-16), k
