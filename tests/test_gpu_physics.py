@@ -28,7 +28,11 @@ def test_sedov_blast_radius_and_energy(golden):
         steps += 1
     st = sim.get_state()
     E1 = _energy(st)
-    assert abs(E1 - E0) / E0 < 1e-3, (E0, E1)
+    # The scheme of the readings (no grad-h terms with variable h, a sound-speed
+    # Courant condition) does not conserve energy through a strong shock: the
+    # ORACLE drifts +5.4% on Sedov 16^3 by t = 0.05 (reading 16), so the
+    # SURVEY's heuristic 1e-3 gate is replaced by 10%.
+    assert abs(E1 - E0) / E0 < 0.10, (E0, E1)
     rho = sim.get_field("rho")  # density of the last step's (pre-update) positions, same order
     r = np.sqrt(st["x"] ** 2 + st["y"] ** 2 + st["z"] ** 2)
     # shock position: the radius of the density peak, averaged over the shell of
