@@ -211,7 +211,7 @@ struct WarpSmem {
   uint32_t mask[kMaxWarpCells];   // children any lane needs
   uint32_t run_start[kMaxRuns];   // first particle of each run
   uint32_t run_pos[kMaxRuns + 1]; // stream position of each run (exclusive prefix)
-  uint32_t run_cell[kMaxRuns];    // index of the run's coarse cell
+  uint32_t run_cell[kMaxRuns];    // periodic image code of the run's cell (2 bits/axis)
   // staged chunk of 32 candidates (image-shifted fp32 position, SoA so that two
   // consecutive candidates are one 64-bit load for the packed f32x2 math)
   alignas(16) float cx[32];
@@ -400,12 +400,22 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
       }
     }
     uint32_t pr = nruns + sr - my_runs, pc = ncand + sc - my_cand;
+    // periodic image of this cell: per axis 0 (inside), 1 (u < 0: stored one box
+    // length above), 2 (u >= n: stored one box length below)
+    uint32_t code = 0;
+    if (my_runs) {
+      const uint32_t pk = S.ucs[u];
+      const int uc[3] = {(int)(pk & 1023u) - 4, (int)((pk >> 10) & 1023u) - 4, (int)(pk >> 20) - 4};
+#pragma unroll
+      for (int a = 0; a < 3; ++a)
+        if (!(kFull && G.full[a])) code |= (uint32_t)(uc[a] < 0 ? 1 : (uc[a] >= n ? 2 : 0)) << (2 * a);
+    }
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
       if (q < (int)my_runs) {
         S.run_start[pr + q] = rs[q];
         S.run_pos[pr + q] = pc;
-        S.run_cell[pr + q] = (uint32_t)u;
+        S.run_cell[pr + q] = code;
         pc += re[q] - rs[q];
       }
     }
@@ -438,11 +448,11 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
     q = F.pos4[qj];
     // unwrapped position of the candidate = stored + k L (k = -1, 0, 1); the
     // shift is applied when the chunk is staged (keeps the load latency hidden)
-    const uint32_t pk = S.ucs[S.run_cell[run]];
-    const int uc[3] = {(int)(pk & 1023u) - 4, (int)((pk >> 10) & 1023u) - 4, (int)(pk >> 20) - 4};
-    if (!(kFull && G.full[0])) sx = uc[0] < 0 ? -B.Lf[0] : (uc[0] >= n ? B.Lf[0] : 0.f);
-    if (!(kFull && G.full[1])) sy = uc[1] < 0 ? -B.Lf[1] : (uc[1] >= n ? B.Lf[1] : 0.f);
-    if (!(kFull && G.full[2])) sz = uc[2] < 0 ? -B.Lf[2] : (uc[2] >= n ? B.Lf[2] : 0.f);
+    const uint32_t code = S.run_cell[run];
+    const uint32_t c0 = code & 3u, c1 = (code >> 2) & 3u, c2 = (code >> 4) & 3u;
+    sx = c0 == 1u ? -B.Lf[0] : (c0 == 2u ? B.Lf[0] : 0.f);
+    sy = c1 == 1u ? -B.Lf[1] : (c1 == 2u ? B.Lf[1] : 0.f);
+    sz = c2 == 1u ? -B.Lf[2] : (c2 == 2u ? B.Lf[2] : 0.f);
   };
   const unsigned long long mx2 = pack2(t.m[0], t.m[0]), my2 = pack2(t.m[1], t.m[1]),
                            mz2 = pack2(t.m[2], t.m[2]);
@@ -499,7 +509,8 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
     // cooperative append: the chunk's hits of all lanes (~100) are written by the
     // 32 lanes together -- owner lane by binary search over the prefix of hit
     // counts, its r-th hit by a popc search -- each list staying in candidate
-    // (= ascending index) order.
+    // (= ascending index) order.  (A per-lane loop over the hit bits is slower:
+    // the warp runs the busiest lane's ~12 iterations per chunk.)
     const int pc = __popc(hin);
     int incl = pc;
 #pragma unroll
