@@ -63,17 +63,30 @@ __global__ void __launch_bounds__(256) density_kernel(Fields F, Params P) {
   double sum = me.d;
   const int32_t* __restrict__ nb = F.nbr + i;
   const Rec4* __restrict__ rec = F.rec_d;
-  // software pipeline: neighbour index two ahead, record one ahead
-  int j1 = nci > 1 ? __ldg(nb + F.cap) : 0;
-  Rec4 rn = nci > 0 ? ldg4(rec + __ldg(nb)) : Rec4{0, 0, 0, 0};
-  for (int k = 0; k < nci; ++k) {
-    const Rec4 rj = rn;
-    if (k + 1 < nci) rn = ldg4(rec + j1);
-    if (k + 2 < nci) j1 = __ldg(nb + (int64_t)(k + 2) * F.cap);
+  // two neighbours per iteration (two independent sinc chains in flight; the sum
+  // is still accumulated in list order), records one pair ahead, indices two
+  const int64_t cap = F.cap;
+  Rec4 ra = ldg4(rec + (nci > 0 ? __ldg(nb) : 0)), rb = ldg4(rec + (nci > 1 ? __ldg(nb + cap) : 0));
+  int jc = nci > 2 ? __ldg(nb + 2 * cap) : 0, jd = nci > 3 ? __ldg(nb + 3 * cap) : 0;
+  int k = 0;
+  for (; k + 1 < nci; k += 2) {
+    const Rec4 a = ra, b = rb;
+    if (k + 2 < nci) ra = ldg4(rec + jc);
+    if (k + 3 < nci) rb = ldg4(rec + jd);
+    if (k + 4 < nci) jc = __ldg(nb + (int64_t)(k + 4) * cap);
+    if (k + 5 < nci) jd = __ldg(nb + (int64_t)(k + 5) * cap);
+    double dxa, dya, dza, dxb, dyb, dzb;
+    pair_d(g, me.a, me.b, me.c, a.a, a.b, a.c, dxa, dya, dza);
+    pair_d(g, me.a, me.b, me.c, b.a, b.b, b.c, dxb, dyb, dzb);
+    const double sa = sinc6_t((dxa * dxa + dya * dya + dza * dza) * q);
+    const double sb = sinc6_t((dxb * dxb + dyb * dyb + dzb * dzb) * q);
+    sum = fma(a.d, sa, sum);
+    sum = fma(b.d, sb, sum);
+  }
+  if (k < nci) {
     double dx, dy, dz;
-    pair_d(g, me.a, me.b, me.c, rj.a, rj.b, rj.c, dx, dy, dz);
-    const double r2 = dx * dx + dy * dy + dz * dz;
-    sum = fma(rj.d, sinc6_t(r2 * q), sum);
+    pair_d(g, me.a, me.b, me.c, ra.a, ra.b, ra.c, dx, dy, dz);
+    sum = fma(ra.d, sinc6_t((dx * dx + dy * dy + dz * dz) * q), sum);
   }
   F.rho[i] = kh3 * sum;
   F.wq[i] = q;
@@ -118,13 +131,10 @@ __global__ void __launch_bounds__(256) iad_kernel(Fields F, Params P) {
   double t11 = 0, t12 = 0, t13 = 0, t22 = 0, t23 = 0, t33 = 0;
   const int32_t* __restrict__ nb = F.nbr + i;
   const Rec4* __restrict__ rec = F.rec_i;
-  // software pipeline: neighbour index two ahead, record one ahead
-  int j1 = nci > 1 ? __ldg(nb + F.cap) : 0;
-  Rec4 rn = nci > 0 ? ldg4(rec + __ldg(nb)) : Rec4{0, 0, 0, 0};
-  for (int k = 0; k < nci; ++k) {
-    const Rec4 rj = rn;
-    if (k + 1 < nci) rn = ldg4(rec + j1);
-    if (k + 2 < nci) j1 = __ldg(nb + (int64_t)(k + 2) * F.cap);
+  // two neighbours per iteration (independent sinc chains in flight; the sums
+  // are still accumulated in list order), records one pair ahead, indices two
+  const int64_t cap = F.cap;
+  auto add = [&](const Rec4& rj) {
     double dx, dy, dz;
     pair_d(g, me.a, me.b, me.c, rj.a, rj.b, rj.c, dx, dy, dz);
     const double r2 = dx * dx + dy * dy + dz * dz;
@@ -137,7 +147,20 @@ __global__ void __launch_bounds__(256) iad_kernel(Fields F, Params P) {
     t22 = fma(ay, dy, t22);
     t23 = fma(ay, dz, t23);
     t33 = fma(az, dz, t33);
+  };
+  Rec4 ra = ldg4(rec + (nci > 0 ? __ldg(nb) : 0)), rb = ldg4(rec + (nci > 1 ? __ldg(nb + cap) : 0));
+  int jc = nci > 2 ? __ldg(nb + 2 * cap) : 0, jd = nci > 3 ? __ldg(nb + 3 * cap) : 0;
+  int k = 0;
+  for (; k + 1 < nci; k += 2) {
+    const Rec4 a = ra, b = rb;
+    if (k + 2 < nci) ra = ldg4(rec + jc);
+    if (k + 3 < nci) rb = ldg4(rec + jd);
+    if (k + 4 < nci) jc = __ldg(nb + (int64_t)(k + 4) * cap);
+    if (k + 5 < nci) jd = __ldg(nb + (int64_t)(k + 5) * cap);
+    add(a);
+    add(b);
   }
+  if (k < nci) add(ra);
   const double det = t11 * (t22 * t33 - t23 * t23) - t12 * (t12 * t33 - t23 * t13) +
                      t13 * (t12 * t23 - t22 * t13);
   const double inv = 1.0 / det;
