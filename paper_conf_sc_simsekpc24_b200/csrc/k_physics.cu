@@ -121,7 +121,7 @@ __global__ void __launch_bounds__(256) eos_kernel(Fields F, Params P) {
 // tau_i = sum_j V_j W(r,h_i) Delta Delta^T, C_i = tau_i^{-1} (adjugate / det);
 // epilogue: the momentum record of particle i.  Per pair: one 32-B record
 // {x, y, z, V}, 55 DP flops.
-__global__ void __launch_bounds__(256) iad_kernel(Fields F, Params P) {
+__global__ void __launch_bounds__(256, 3) iad_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= F.n) return;
   const Geom g = load_geom(F.ds, P);
