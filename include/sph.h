@@ -248,6 +248,11 @@ int sph_find_neighbors(sph_ctx* ctx, sph_nbr_stats* stats);
  * SPH_ERR_CAPACITY with offsets still filled. */
 int sph_get_neighbors(sph_ctx* ctx, int64_t* offsets, int32_t* idx, int64_t idx_cap);
 
+/* The lists of nt chosen particles only (current-order indices `targets`):
+ * offsets[nt+1], idx as in sph_get_neighbors.  For sampled checks at full size. */
+int sph_get_neighbor_rows(sph_ctx* ctx, const int64_t* targets, int64_t nt, int64_t* offsets,
+                          int32_t* idx, int64_t idx_cap);
+
 /* Item 5 (XMass): rho_i = (K/h_i^3) [m_i + sum_j m_j S(pi r_ij/2h_i)^6].  DENSITY. */
 int sph_density(sph_ctx* ctx);
 

@@ -692,6 +692,32 @@ int sph_get_neighbors(sph_ctx* c, int64_t* offsets, int32_t* idx, int64_t idx_ca
   return SPH_OK;
 }
 
+int sph_get_neighbor_rows(sph_ctx* c, const int64_t* targets, int64_t nt, int64_t* offsets,
+                          int32_t* idx, int64_t idx_cap) {
+  int rc = check_ready(c, S_NBR, "sph_get_neighbor_rows");
+  if (rc) return rc;
+  if (nt < 0 || (nt > 0 && (!targets || !offsets))) return fail(c, SPH_ERR_ARG, "bad targets");
+  std::vector<int32_t> nc((size_t)nt);
+  for (int64_t q = 0; q < nt; ++q) {
+    if (targets[q] < 0 || targets[q] >= c->n) return fail(c, SPH_ERR_ARG, "target %lld out of range", (long long)targets[q]);
+    rc = cuda_check(c, cudaMemcpyAsync(&nc[q], c->nc + targets[q], 4, cudaMemcpyDeviceToHost, c->st), "nc copy");
+    if (rc) return rc;
+  }
+  if ((rc = cuda_check(c, cudaStreamSynchronize(c->st), "sync"))) return rc;
+  offsets[0] = 0;
+  for (int64_t q = 0; q < nt; ++q) offsets[q + 1] = offsets[q] + std::min(nc[q], c->cfg.ngmax);
+  if (offsets[nt] > idx_cap || (!idx && offsets[nt] > 0))
+    return fail(c, SPH_ERR_CAPACITY, "idx_cap %lld < %lld neighbours", (long long)idx_cap, (long long)offsets[nt]);
+  for (int64_t q = 0; q < nt; ++q) {
+    const int64_t k = offsets[q + 1] - offsets[q];
+    if (!k) continue;
+    rc = cuda_check(c, cudaMemcpy2DAsync(idx + offsets[q], 4, c->nbr + targets[q], 4 * c->cfg.n_capacity, 4, k,
+                                         cudaMemcpyDeviceToHost, c->st), "row copy");
+    if (rc) return rc;
+  }
+  return cuda_check(c, cudaStreamSynchronize(c->st), "sync");
+}
+
 int sph_density(sph_ctx* c) {
   int rc = check_ready(c, S_NBR, "sph_density");
   return rc ? rc : body_simple(c, SPH_PHASE_DENSITY, S_DENS);

@@ -77,7 +77,7 @@ EXPORTS = ("sph_config_default", "sph_workspace_size", "sph_init", "sph_finalize
            "sph_timestep", "sph_update", "sph_step", "sph_set_clock_policy",
            "sph_energy_report", "sph_energy_reset", "sph_energy_counter_mj", "sph_repeat_phase",
            "sph_set_accounting", "sph_kernel_launches", "sph_set_field",
-           "sph_get_local_min_hc", "sph_set_global_min_hc")
+           "sph_get_local_min_hc", "sph_set_global_min_hc", "sph_get_neighbor_rows")
 GHOST_BIT = 1 << 62
 
 _lib = None
@@ -123,6 +123,7 @@ def load(build_if_missing: bool = True):
     L.sph_repeat_phase.argtypes = [P, I, I, C.POINTER(D), C.POINTER(D)]
     L.sph_set_accounting.argtypes = [P, I]
     L.sph_set_field.argtypes = [P, I, V, I]
+    L.sph_get_neighbor_rows.argtypes = [P, V, I64, V, V, I64]
     L.sph_get_local_min_hc.argtypes = [P, C.POINTER(D)]
     L.sph_set_global_min_hc.argtypes = [P, D]
     L.sph_kernel_launches.argtypes = [C.POINTER(I64)]
@@ -298,6 +299,16 @@ class Simulation:
         self._ok(self.L.sph_get_neighbors(self.ctx, C.c_void_p(off.ctypes.data),
                                           C.c_void_p(idx.ctypes.data), total))
         return off, idx[:total]
+
+    def get_neighbor_rows(self, targets):
+        """Neighbour lists of the given current-order indices only."""
+        t = np.ascontiguousarray(targets, dtype=np.int64)
+        off = np.zeros(t.size + 1, dtype=np.int64)
+        cap = int(t.size * self.cfg.ngmax)
+        idx = np.zeros(max(cap, 1), dtype=np.int32)
+        self._ok(self.L.sph_get_neighbor_rows(self.ctx, C.c_void_p(t.ctypes.data), t.size,
+                                              C.c_void_p(off.ctypes.data), C.c_void_p(idx.ctypes.data), cap))
+        return off, idx[:off[-1]]
 
     def density(self):
         self._ok(self.L.sph_density(self.ctx))
