@@ -236,15 +236,20 @@ __global__ void __launch_bounds__(128) momentum_energy_kernel(Fields F, Params P
       const double wi = khi * sinc6_t(r2 * qi);
       const double tj = r2 * j0.d;
       const double wj = tj < kPi2 ? j1.d * sinc6_t(tj) : 0.0;
-      // Delta = -d
+      // Delta = -d.  With A = w_i C_i Delta, B = w_j C_j Delta, G = (A+B)/2 the
+      // pair terms regroup exactly (up to rounding) as
+      //   (p_i/rho_i^2) A + (p_j/rho_j^2) B + Pi G
+      //     = (p_i/rho_i^2 + Pi/2) w_i C_i Delta + (p_j/rho_j^2 + Pi/2) w_j C_j Delta,
+      //   (p_i/rho_i^2) v.A + Pi/2 v.G
+      //     = (p_i/rho_i^2 + Pi/4) w_i v.C_i Delta + (Pi/4) w_j v.C_j Delta,
+      // which saves the scaled vectors A, B, G (~9 DP instructions per pair).
       const double Dx = -dx, Dy = -dy, Dz = -dz;
-      const double Ax = (ci11 * Dx + ci12 * Dy + ci13 * Dz) * wi;
-      const double Ay = (ci12 * Dx + ci22 * Dy + ci23 * Dz) * wi;
-      const double Az = (ci13 * Dx + ci23 * Dy + ci33 * Dz) * wi;
-      const double Bx = (j1.a * Dx + j1.b * Dy + j1.c * Dz) * wj;
-      const double By = (j1.b * Dx + j2.a * Dy + j2.b * Dz) * wj;
-      const double Bz = (j1.c * Dx + j2.b * Dy + j2.c * Dz) * wj;
-      const double Gx = 0.5 * (Ax + Bx), Gy = 0.5 * (Ay + By), Gz = 0.5 * (Az + Bz);
+      const double CiDx = ci11 * Dx + ci12 * Dy + ci13 * Dz;
+      const double CiDy = ci12 * Dx + ci22 * Dy + ci23 * Dz;
+      const double CiDz = ci13 * Dx + ci23 * Dy + ci33 * Dz;
+      const double CjDx = j1.a * Dx + j1.b * Dy + j1.c * Dz;
+      const double CjDy = j1.b * Dx + j2.a * Dy + j2.b * Dz;
+      const double CjDz = j1.c * Dx + j2.b * Dy + j2.c * Dz;
       const double vx = vxi - j3.a, vy = vyi - j3.b, vz = vzi - j3.c;
       const double rv = dx * vx + dy * vy + dz * vz;
       double Pi = 0.0;
@@ -261,10 +266,13 @@ __global__ void __launch_bounds__(128) momentum_energy_kernel(Fields F, Params P
         Pi = (fma(beta, mu, -alpha * cbar) * mu) * (D * q);
       }
       const double mj = j2.d, prj = j3.d;
-      ax -= mj * (pri * Ax + prj * Bx + Pi * Gx);
-      ay -= mj * (pri * Ay + prj * By + Pi * Gy);
-      az -= mj * (pri * Az + prj * Bz + Pi * Gz);
-      de += mj * (pri * (vx * Ax + vy * Ay + vz * Az) + 0.5 * Pi * (vx * Gx + vy * Gy + vz * Gz));
+      const double ka = (pri + 0.5 * Pi) * wi, kb = (prj + 0.5 * Pi) * wj;
+      ax -= mj * fma(ka, CiDx, kb * CjDx);
+      ay -= mj * fma(ka, CiDy, kb * CjDy);
+      az -= mj * fma(ka, CiDz, kb * CjDz);
+      const double vCi = vx * CiDx + vy * CiDy + vz * CiDz;
+      const double vCj = vx * CjDx + vy * CjDy + vz * CjDz;
+      de += mj * fma((pri + 0.25 * Pi) * wi, vCi, 0.25 * Pi * wj * vCj);
     }
     F.ax[i] = ax;
     F.ay[i] = ay;
