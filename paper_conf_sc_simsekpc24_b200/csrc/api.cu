@@ -60,7 +60,7 @@ struct sph_ctx {
   uint64_t *keyA, *keyB, *key_sorted;
   uint32_t *valA, *valB;
   double *rho, *p, *c, *vol, *prho2, *wq, *wk, *C[6], *ax, *ay, *az, *du;
-  int32_t *nc, *nbr;
+  int32_t *nc, *nbr, *nrows;
   uint32_t* cell_start;
   float4* pos4;
   Rec4 *rec_d, *rec_i, *rec_m;
@@ -114,6 +114,9 @@ int check_ready(sph_ctx* c, int min_stage, const char* what) {
   return SPH_OK;
 }
 
+// Row stride of the neighbour-search scratch rows: ngmax rounded up to 8.
+int64_t nrows_ld(const sph_config* cfg) { return ((int64_t)cfg->ngmax + 7) / 8 * 8; }
+
 Fields fields(sph_ctx* c) {
   Fields F;
   F.n = c->n;
@@ -126,6 +129,7 @@ Fields fields(sph_ctx* c) {
   for (int e = 0; e < 6; ++e) F.C[e] = c->C[e];
   F.ax = c->ax; F.ay = c->ay; F.az = c->az; F.du = c->du;
   F.nc = c->nc; F.nbr = c->nbr; F.ngmax = c->cfg.ngmax;
+  F.nrows = c->nrows; F.nrows_ld = nrows_ld(&c->cfg);
   F.cell_start = c->cell_start;
   F.pos4 = c->pos4;
   F.rec_d = c->rec_d;
@@ -407,6 +411,7 @@ static size_t layout(const sph_config* cfg, char* base, sph_ctx* c) {
   }
   char* ncp = take(sizeof(int32_t) * cap);
   char* nbp = take(sizeof(int32_t) * cap * (size_t)cfg->ngmax);
+  char* nrp = take(sizeof(int32_t) * (size_t)kNbrSlots * kNbrSlotRows * (size_t)nrows_ld(cfg));
   const int Lc = level_cap_for(cfg);
   char* cs = take(sizeof(uint32_t) * ((size_t(1) << (3 * Lc)) + 1));
   size_t hb, sb;
@@ -417,7 +422,7 @@ static size_t layout(const sph_config* cfg, char* base, sph_ctx* c) {
   if (c) {
     c->keyA = (uint64_t*)kA; c->keyB = (uint64_t*)kB;
     c->valA = (uint32_t*)vA; c->valB = (uint32_t*)vB;
-    c->nc = (int32_t*)ncp; c->nbr = (int32_t*)nbp;
+    c->nc = (int32_t*)ncp; c->nbr = (int32_t*)nbp; c->nrows = (int32_t*)nrp;
     c->cell_start = (uint32_t*)cs;
     c->level_cap = Lc;
     c->sort_hist = (uint32_t*)hp; c->sort_status = (uint32_t*)sp; c->status_bytes = sb;

@@ -31,7 +31,13 @@
 //     operation, d2 < (2h_i)(2h_i)).  Every decision equals the exact predicate's:
 //     the neighbour sets are bit-identical to brute force;
 //  4. hits are appended with predicated stores in candidate order.
-// Lists are stored column-major nbr[k*cap + i].
+// Hits are appended to row-major scratch rows of the CTA slot (an owner's hits
+// of a chunk are consecutive words: a few lines per store instruction; the
+// scratch of the resident CTAs, ~70 MB, stays in L2); when a warp has finished
+// its targets, every lane copies its row to the column-major list nbr[k*cap + i]
+// (one 128-B line per store instruction) that the neighbour sums read.  The
+// kernel is persistent: a grid of (SMs x resident CTAs) CTAs strides over the
+// 128-target tiles, so the scratch is indexed by blockIdx.
 // Bound: issue (fp32 + integer work per candidate test, ~880 candidates per
 // warp of 32 targets at 100 neighbours).  Algorithmic bytes: pos4, x, y, z, h in
 // (48 B), nc out (4 B), the list out (4 B per neighbour).
@@ -84,7 +90,6 @@ void launch_cells(const Fields& F, const Params& P, int level_cap, cudaStream_t 
 constexpr int kNbrThreads = 128;
 constexpr int kNbrWarps = kNbrThreads / 32;
 constexpr int kMaxWarpCells = 128;
-constexpr uint32_t kNoCell = 0xffffffffu;
 
 // Per-target constants of the search.
 struct Target {
@@ -329,10 +334,10 @@ __device__ __forceinline__ GroupBox build_cells(const Box& B, const int (&cc)[3]
 // t.rc < 0 take part in the warp collectives but test nothing.
 template <bool kFull>
 __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const Target& t, int64_t i,
-                                          const GroupBox& G, WarpSmem& S, int lane, int& cnt) {
+                                          const GroupBox& G, WarpSmem& S, int lane, int& cnt,
+                                          int32_t* __restrict__ rows) {
   const int n = B.nside;
   const int T = G.T;
-  const int64_t cap = F.cap;
   const int ngmax = F.ngmax;
   const float rc2 = t.rc * t.rc;
   const bool live = t.rc >= 0.f;
@@ -533,7 +538,7 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
       if (h < tot) {
         const int r = h - o_excl;
         const int slot = o_cnt + r;
-        if (slot < ngmax) F.nbr[(int64_t)slot * cap + wbase + owner] = (int32_t)S.cj[nth_set_bit(o_mask, r)];
+        if (slot < ngmax) rows[owner * F.nrows_ld + slot] = (int32_t)S.cj[nth_set_bit(o_mask, r)];
       }
     }
     cnt += pc;
@@ -545,9 +550,6 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
 __global__ void __launch_bounds__(kNbrThreads, 6) neighbors_kernel(Fields F, Params P) {
   __shared__ WarpSmem s_w[kNbrWarps];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  const bool active = i < F.n;
-  if (!__any_sync(0xffffffffu, active)) return;  // whole warp past the end
   const DevScalars* ds = F.ds;
   Box B;
   B.Lc = ds->cell_level - 1;
@@ -560,69 +562,100 @@ __global__ void __launch_bounds__(kNbrThreads, 6) neighbors_kernel(Fields F, Par
     B.side[a] = (float)(B.L[a] / B.nside);
     B.per[a] = P.periodic[a] != 0;
   }
-  const Target t = make_target(F, B, i, active);
-  int cc[3] = {0, 0, 0};
-  uint32_t ckey = 0;
-  if (active) {
-    const uint64_t key = F.key[i];
-    const int sh = 21 - B.Lc;
-    cc[0] = (int)(compact3(key >> 2) >> sh);
-    cc[1] = (int)(compact3(key >> 1) >> sh);
-    cc[2] = (int)(compact3(key) >> sh);
-    ckey = (uint32_t)(key >> (3 * sh));
-  }
-  int cnt = 0;
+  // this warp's 32 scratch rows (row of lane l: rows + l * nrows_ld)
+  int32_t* const rows = F.nrows + ((int64_t)blockIdx.x * kNbrThreads + warp * 32) * F.nrows_ld;
+  const int64_t ntiles = div_up(F.n, kNbrThreads);
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t i = tile * kNbrThreads + threadIdx.x;
+    const bool active = i < F.n;
+    if (!__any_sync(0xffffffffu, active)) continue;  // whole warp past the end
+    const Target t = make_target(F, B, i, active);
+    int cc[3] = {0, 0, 0};
+    uint32_t ckey = 0;
+    if (active) {
+      const uint64_t key = F.key[i];
+      const int sh = 21 - B.Lc;
+      cc[0] = (int)(compact3(key >> 2) >> sh);
+      cc[1] = (int)(compact3(key >> 1) >> sh);
+      cc[2] = (int)(compact3(key) >> sh);
+      ckey = (uint32_t)(key >> (3 * sh));
+    }
+    int cnt = 0;
 
-  // group size: the whole warp unless it spans more than kMaxGroupCells distinct
-  // coarse cells (Morton jumps); then halves, quarters, ...
-  int g = 32;
-  uint32_t leaders;
-  while (true) {
-    const unsigned long long tag =
-        active ? (((unsigned long long)(lane / g)) << 32) | ckey : (0xffffffff00000000ull | (unsigned)lane);
-    const uint32_t peers = __match_any_sync(0xffffffffu, tag);
-    const bool lead = active && (peers & ((1u << lane) - 1u)) == 0;
-    leaders = __ballot_sync(0xffffffffu, lead);
-    const uint32_t gm = (g == 32) ? 0xffffffffu : (((1u << g) - 1u) << ((lane / g) * g));
-    const int D = __popc(leaders & gm);
-    if (g == 1 || __reduce_max_sync(0xffffffffu, D) <= kMaxGroupCells) break;
-    g >>= 1;
-  }
-  for (int gid = 0; gid < 32 / g; ++gid) {
-    const uint32_t gm = (g == 32) ? 0xffffffffu : (((1u << g) - 1u) << (gid * g));
-    const uint32_t gl = leaders & gm;
-    if (!gl) continue;
-    const GroupBox G = build_cells(B, cc, gl, lane, s_w[warp]);
-    Target tg = t;
-    if (lane / g != gid) tg.r_out2 = tg.r_in2 = tg.rc = -1.f;  // not in this pass
-    if (G.full[0] || G.full[1] || G.full[2])
-      warp_walk<true>(F, B, tg, i, G, s_w[warp], lane, cnt);
-    else
-      warp_walk<false>(F, B, tg, i, G, s_w[warp], lane, cnt);
-    __syncwarp();
-  }
-  if (active) F.nc[i] = cnt;
-
-  // nc statistics (min, max, total) and the capacity flag.
-  int mn = active ? cnt : 0x7fffffff, mx = active ? cnt : 0;
-  unsigned long long tot = active ? (unsigned long long)cnt : 0ull;
+    // group size: the whole warp unless it spans more than kMaxGroupCells distinct
+    // coarse cells (Morton jumps); then halves, quarters, ...
+    int g = 32;
+    uint32_t leaders;
+    while (true) {
+      const unsigned long long tag =
+          active ? (((unsigned long long)(lane / g)) << 32) | ckey : (0xffffffff00000000ull | (unsigned)lane);
+      const uint32_t peers = __match_any_sync(0xffffffffu, tag);
+      const bool lead = active && (peers & ((1u << lane) - 1u)) == 0;
+      leaders = __ballot_sync(0xffffffffu, lead);
+      const uint32_t gm = (g == 32) ? 0xffffffffu : (((1u << g) - 1u) << ((lane / g) * g));
+      const int D = __popc(leaders & gm);
+      if (g == 1 || __reduce_max_sync(0xffffffffu, D) <= kMaxGroupCells) break;
+      g >>= 1;
+    }
+    for (int gid = 0; gid < 32 / g; ++gid) {
+      const uint32_t gm = (g == 32) ? 0xffffffffu : (((1u << g) - 1u) << (gid * g));
+      const uint32_t gl = leaders & gm;
+      if (!gl) continue;
+      const GroupBox G = build_cells(B, cc, gl, lane, s_w[warp]);
+      Target tg = t;
+      if (lane / g != gid) tg.r_out2 = tg.r_in2 = tg.rc = -1.f;  // not in this pass
+      if (G.full[0] || G.full[1] || G.full[2])
+        warp_walk<true>(F, B, tg, i, G, s_w[warp], lane, cnt, rows);
+      else
+        warp_walk<false>(F, B, tg, i, G, s_w[warp], lane, cnt, rows);
+      __syncwarp();
+    }
+    if (active) F.nc[i] = cnt;
+    // copy the rows to the column-major list: lane l holds row l; the store of
+    // slot k by the 32 lanes is one 128-B line
+    const int len = active ? min(cnt, F.ngmax) : 0;
+    const int wlen = __reduce_max_sync(0xffffffffu, len);
+    const int32_t* myrow = rows + lane * F.nrows_ld;
+    int32_t* col = F.nbr + i;
+    for (int k0 = 0; k0 < wlen; k0 += 8) {
+      int v[8];
+      if (k0 < len) ld8i(myrow + k0, v);
 #pragma unroll
-  for (int off = 16; off > 0; off >>= 1) {
-    mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, off));
-    mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, off));
-    tot += __shfl_xor_sync(0xffffffffu, tot, off);
-  }
-  if (lane == 0) {
-    atomicMin(&F.ds->min_nc, mn);
-    atomicMax(&F.ds->max_nc, mx);
-    atomicAdd(&F.ds->total_nc, tot);
-    if (mx > F.ngmax) atomicOr(&F.ds->status, (int)ST_CAPACITY);
+      for (int u = 0; u < 8; ++u)
+        if (k0 + u < len) col[(int64_t)(k0 + u) * F.cap] = v[u];
+    }
+    __syncwarp();  // the rows are reused by the next tile
+
+    // nc statistics (min, max, total) and the capacity flag.
+    int mn = active ? cnt : 0x7fffffff, mx = active ? cnt : 0;
+    unsigned long long tot = active ? (unsigned long long)cnt : 0ull;
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) {
+      mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, off));
+      mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, off));
+      tot += __shfl_xor_sync(0xffffffffu, tot, off);
+    }
+    if (lane == 0) {
+      atomicMin(&F.ds->min_nc, mn);
+      atomicMax(&F.ds->max_nc, mx);
+      atomicAdd(&F.ds->total_nc, tot);
+      if (mx > F.ngmax) atomicOr(&F.ds->status, (int)ST_CAPACITY);
+    }
   }
 }
 
 void launch_neighbors(const Fields& F, const Params& P, cudaStream_t st) {
   if (F.n == 0) return;
-  neighbors_kernel<<<(unsigned)div_up(F.n, kNbrThreads), kNbrThreads, 0, st>>>(F, P);
+  static int resident = 0;  // SMs x resident CTAs of this kernel (<= kNbrSlots)
+  if (!resident) {
+    int dev = 0, sms = 0, per = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, neighbors_kernel, kNbrThreads, 0);
+    resident = std::max(1, std::min(kNbrSlots, sms * std::max(per, 1)));
+  }
+  const int64_t grid = std::min<int64_t>(div_up(F.n, kNbrThreads), resident);
+  neighbors_kernel<<<(unsigned)grid, kNbrThreads, 0, st>>>(F, P);
   note_launch();
 }
 

@@ -88,7 +88,9 @@ struct Fields {
   double* C[6];           // 11 12 13 22 23 33
   double *ax, *ay, *az, *du;
   int32_t* nc;
-  int32_t* nbr;           // [ngmax][cap]
+  int32_t* nbr;           // [ngmax][cap] column-major: neighbour k of target i at nbr[k * cap + i]
+  int32_t* nrows;         // neighbour-search scratch: row-major rows of the resident warps
+  int64_t nrows_ld;       // their row stride (ngmax rounded up to 8: 32-B aligned rows)
   int32_t ngmax;
   uint32_t* cell_start;   // [8^L + 1], L = fine cell level
   float4* pos4;           // fp32 (x, y, z) - box_min: neighbour-search prefilter
@@ -121,6 +123,15 @@ __device__ __forceinline__ unsigned long long ord_of(double v) {
 __device__ __forceinline__ double unord(unsigned long long o) {
   unsigned long long b = (o >> 63) ? (o & 0x7fffffffffffffffull) : ~o;
   return __longlong_as_double((long long)b);
+}
+
+// Eight consecutive 32-bit words in one 256-bit load (coherent: the data may
+// have been written earlier in the same kernel, ordered by __syncwarp).
+__device__ __forceinline__ void ld8i(const int32_t* p, int (&v)[8]) {
+  asm volatile("ld.global.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+               : "l"(p)
+               : "memory");
 }
 
 // 21-bit Morton spread / compact (x most significant in each triplet).
@@ -198,6 +209,8 @@ void launch_permute(const Fields& Fdst, const uint32_t* perm, double* const* src
                     const int64_t* id_src, cudaStream_t st);
 void launch_cells(const Fields& F, const Params& P, int level_cap, cudaStream_t st);
 void launch_neighbors(const Fields& F, const Params& P, cudaStream_t st);
+constexpr int kNbrSlots = 1024;    // neighbour-search CTAs in flight (>= SMs x resident CTAs)
+constexpr int kNbrSlotRows = 128;  // scratch rows per CTA (its threads)
 void launch_density(const Fields& F, const Params& P, cudaStream_t st);
 void launch_eos(const Fields& F, const Params& P, cudaStream_t st);
 void launch_iad(const Fields& F, const Params& P, cudaStream_t st);
