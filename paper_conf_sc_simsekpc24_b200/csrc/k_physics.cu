@@ -24,7 +24,7 @@ constexpr double kPi2Over4 = kPi * kPi / 4.0;
 constexpr double kPi2 = kPi * kPi;
 
 struct Geom {
-  double L[3], H[3];
+  double L[3], H[3], lo[3], hi[3];
   bool per[3];
 };
 
@@ -35,28 +35,50 @@ __device__ __forceinline__ Geom load_geom(const DevScalars* ds, const Params& P)
     g.L[a] = ds->box_max[a] - ds->box_min[a];
     g.H[a] = 0.5 * g.L[a];
     g.per[a] = P.periodic[a] != 0;
+    g.lo[a] = ds->box_min[a];
+    g.hi[a] = ds->box_max[a];
   }
   return g;
 }
 
-// d = x_i - x_j, minimum image (the oracle's order: raw difference, then +-L)
+// True unless every neighbour of a target at x with smoothing length h is
+// certainly reached without a periodic image: a neighbour needs the image only
+// if |x_i - x_j| > L - 2h_i, impossible when x_i is >= 2h_i from both faces
+// (2.5 h keeps a margin for rounding).  Then the oracle's conditional +-L never
+// fires and d = x_i - x_j is the same double.
+__device__ __forceinline__ bool needs_wrap(const Geom& g, double x, double y, double z, double h) {
+  const double m = 2.5 * h;
+  const double c[3] = {x, y, z};
+  bool w = false;
+#pragma unroll
+  for (int a = 0; a < 3; ++a)
+    if (g.per[a] && (c[a] - g.lo[a] < m || g.hi[a] - c[a] < m)) w = true;
+  return w;
+}
+
+// d = x_i - x_j, minimum image (the oracle's order: raw difference, then +-L);
+// kWrap = false for warps whose targets all pass needs_wrap() == false.
+template <bool kWrap>
 __device__ __forceinline__ void pair_d(const Geom& g, double xi, double yi, double zi, double xj,
                                        double yj, double zj, double& dx, double& dy, double& dz) {
-  dx = min_image(xi - xj, g.L[0], g.H[0], g.per[0]);
-  dy = min_image(yi - yj, g.L[1], g.H[1], g.per[1]);
-  dz = min_image(zi - zj, g.L[2], g.H[2], g.per[2]);
+  if (kWrap) {
+    dx = min_image(xi - xj, g.L[0], g.H[0], g.per[0]);
+    dy = min_image(yi - yj, g.L[1], g.H[1], g.per[1]);
+    dz = min_image(zi - zj, g.L[2], g.H[2], g.per[2]);
+  } else {
+    dx = xi - xj;
+    dy = yi - yj;
+    dz = zi - zj;
+  }
 }
 
 // ------------------------------------------------------------------ density
 // rho_i = (K/h_i^3) [m_i + sum_j m_j S(pi r_ij / 2h_i)^6]; also writes the
 // per-particle kernel factors wq = (pi/2h)^2 and wk = K/h^3 reused by IAD and
 // momentum-energy.  Per pair: one 32-B record {x, y, z, m}, 40 DP flops.
-__global__ void __launch_bounds__(256) density_kernel(Fields F, Params P) {
-  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (i >= F.n) return;
-  const Geom g = load_geom(F.ds, P);
-  const Rec4 me = F.rec_d[i];
-  const double hi = F.f[FH][i];
+template <bool kWrap>
+__device__ __forceinline__ void density_body(const Fields& F, const Params& P, const Geom& g, int64_t i,
+                                             const Rec4& me, double hi) {
   const double q = kPi2Over4 / (hi * hi);
   const double kh3 = P.K / (hi * hi * hi);
   const int nci = min(F.nc[i], F.ngmax);
@@ -76,8 +98,8 @@ __global__ void __launch_bounds__(256) density_kernel(Fields F, Params P) {
     if (k + 4 < nci) jc = __ldg(nb + (int64_t)(k + 4) * cap);
     if (k + 5 < nci) jd = __ldg(nb + (int64_t)(k + 5) * cap);
     double dxa, dya, dza, dxb, dyb, dzb;
-    pair_d(g, me.a, me.b, me.c, a.a, a.b, a.c, dxa, dya, dza);
-    pair_d(g, me.a, me.b, me.c, b.a, b.b, b.c, dxb, dyb, dzb);
+    pair_d<kWrap>(g, me.a, me.b, me.c, a.a, a.b, a.c, dxa, dya, dza);
+    pair_d<kWrap>(g, me.a, me.b, me.c, b.a, b.b, b.c, dxb, dyb, dzb);
     const double sa = sinc6_t((dxa * dxa + dya * dya + dza * dza) * q);
     const double sb = sinc6_t((dxb * dxb + dyb * dyb + dzb * dzb) * q);
     sum = fma(a.d, sa, sum);
@@ -85,12 +107,24 @@ __global__ void __launch_bounds__(256) density_kernel(Fields F, Params P) {
   }
   if (k < nci) {
     double dx, dy, dz;
-    pair_d(g, me.a, me.b, me.c, ra.a, ra.b, ra.c, dx, dy, dz);
+    pair_d<kWrap>(g, me.a, me.b, me.c, ra.a, ra.b, ra.c, dx, dy, dz);
     sum = fma(ra.d, sinc6_t((dx * dx + dy * dy + dz * dz) * q), sum);
   }
   F.rho[i] = kh3 * sum;
   F.wq[i] = q;
   F.wk[i] = kh3;
+}
+
+__global__ void __launch_bounds__(256, 4) density_kernel(Fields F, Params P) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= F.n) return;
+  const Geom g = load_geom(F.ds, P);
+  const Rec4 me = F.rec_d[i];
+  const double hi = F.f[FH][i];
+  if (__any_sync(__activemask(), needs_wrap(g, me.a, me.b, me.c, hi)))
+    density_body<true>(F, P, g, i, me, hi);
+  else
+    density_body<false>(F, P, g, i, me, hi);
 }
 
 // ------------------------------------------------------------------ EOS
@@ -121,11 +155,8 @@ __global__ void __launch_bounds__(256) eos_kernel(Fields F, Params P) {
 // tau_i = sum_j V_j W(r,h_i) Delta Delta^T, C_i = tau_i^{-1} (adjugate / det);
 // epilogue: the momentum record of particle i.  Per pair: one 32-B record
 // {x, y, z, V}, 55 DP flops.
-__global__ void __launch_bounds__(256, 3) iad_kernel(Fields F, Params P) {
-  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (i >= F.n) return;
-  const Geom g = load_geom(F.ds, P);
-  const Rec4 me = F.rec_i[i];
+template <bool kWrap>
+__device__ __forceinline__ void iad_body(const Fields& F, const Geom& g, int64_t i, const Rec4& me) {
   const double q = F.wq[i], kh3 = F.wk[i];
   const int nci = min(F.nc[i], F.ngmax);
   double t11 = 0, t12 = 0, t13 = 0, t22 = 0, t23 = 0, t33 = 0;
@@ -136,7 +167,7 @@ __global__ void __launch_bounds__(256, 3) iad_kernel(Fields F, Params P) {
   const int64_t cap = F.cap;
   auto add = [&](const Rec4& rj) {
     double dx, dy, dz;
-    pair_d(g, me.a, me.b, me.c, rj.a, rj.b, rj.c, dx, dy, dz);
+    pair_d<kWrap>(g, me.a, me.b, me.c, rj.a, rj.b, rj.c, dx, dy, dz);
     const double r2 = dx * dx + dy * dy + dz * dz;
     const double vw = rj.d * (kh3 * sinc6_t(r2 * q));
     // Delta = -d; the products Delta^a Delta^b equal d^a d^b.
@@ -185,6 +216,17 @@ __global__ void __launch_bounds__(256, 3) iad_kernel(Fields F, Params P) {
   st4(rm + 4, F.f[FH][i], F.c[i], F.rho[i], 0.0);
 }
 
+__global__ void __launch_bounds__(256, 3) iad_kernel(Fields F, Params P) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= F.n) return;
+  const Geom g = load_geom(F.ds, P);
+  const Rec4 me = F.rec_i[i];
+  if (__any_sync(__activemask(), needs_wrap(g, me.a, me.b, me.c, F.f[FH][i])))
+    iad_body<true>(F, g, i, me);
+  else
+    iad_body<false>(F, g, i, me);
+}
+
 // ------------------------------------------------------------------ momentum-energy
 // a_i = -sum_j m_j [(p_i/rho_i^2) A + (p_j/rho_j^2) B + Pi G],
 // du_i = sum_j m_j [(p_i/rho_i^2) v_ij.A + Pi/2 v_ij.G],
@@ -193,92 +235,102 @@ __global__ void __launch_bounds__(256, 3) iad_kernel(Fields F, Params P) {
 // order-preserving bit pattern of a positive double).
 // Per pair: 4 records (128 B) + 1 more (AV) for approaching pairs, 157 DP flops
 // (+ 17 and 2 divisions when approaching).
-__global__ void __launch_bounds__(128) momentum_energy_kernel(Fields F, Params P) {
+template <bool kWrap>
+__device__ __forceinline__ void momentum_body(const Fields& F, const Params& P, const Geom& g, int64_t i) {
+  const Rec4* __restrict__ rec = F.rec_m;
+  const Rec4* mi = rec + (int64_t)kRecM * i;
+  const Rec4 i0 = mi[0], i1 = mi[1], i2 = mi[2], i3 = mi[3], i4 = mi[4];
+  const double xi = i0.a, yi = i0.b, zi = i0.c, qi = i0.d;
+  const double ci11 = i1.a, ci12 = i1.b, ci13 = i1.c, khi = i1.d;
+  const double ci22 = i2.a, ci23 = i2.b, ci33 = i2.c;
+  const double vxi = i3.a, vyi = i3.b, vzi = i3.c, pri = i3.d;
+  const double hi = i4.a, ci = i4.b, rhoi = i4.c;
+  const double alpha = P.av_alpha, beta = P.av_beta, eps = P.av_eps;
+  const int nci = min(F.nc[i], F.ngmax);
+  double ax = 0, ay = 0, az = 0, de = 0;
+  const int32_t* __restrict__ nb = F.nbr + i;
+  // software pipeline: neighbour index three ahead, the position chunk (needed
+  // first) two ahead; the other chunks are loaded at the top of the iteration
+  // and arrive while the two sinc polynomials run.
+  const int64_t cap = F.cap;
+  const Rec4* r0 = rec + (int64_t)kRecM * (nci > 0 ? __ldg(nb) : 0);
+  const Rec4* r1 = rec + (int64_t)kRecM * (nci > 1 ? __ldg(nb + cap) : 0);
+  int jn = nci > 2 ? __ldg(nb + 2 * cap) : 0;
+  Rec4 p0 = ldg4(r0), p1 = ldg4(r1);
+  for (int k = 0; k < nci; ++k) {
+    const Rec4* rcur = r0;
+    const Rec4 j1 = ldg4(rcur + 1), j2 = ldg4(rcur + 2), j3 = ldg4(rcur + 3);
+    const Rec4 j0 = p0;
+    p0 = p1;
+    r0 = r1;
+    if (k + 2 < nci) {
+      r1 = rec + (int64_t)kRecM * jn;
+      p1 = ldg4(r1);
+    }
+    if (k + 3 < nci) jn = __ldg(nb + (int64_t)(k + 3) * cap);
+    double dx, dy, dz;
+    pair_d<kWrap>(g, xi, yi, zi, j0.a, j0.b, j0.c, dx, dy, dz);
+    const double r2 = dx * dx + dy * dy + dz * dz;
+    const double wi = khi * sinc6_t(r2 * qi);
+    const double tj = r2 * j0.d;
+    const double wj = tj < kPi2 ? j1.d * sinc6_t(tj) : 0.0;
+    // Delta = -d.  With A = w_i C_i Delta, B = w_j C_j Delta, G = (A+B)/2 the
+    // pair terms regroup exactly (up to rounding) as
+    //   (p_i/rho_i^2) A + (p_j/rho_j^2) B + Pi G
+    //     = (p_i/rho_i^2 + Pi/2) w_i C_i Delta + (p_j/rho_j^2 + Pi/2) w_j C_j Delta,
+    //   (p_i/rho_i^2) v.A + Pi/2 v.G
+    //     = (p_i/rho_i^2 + Pi/4) w_i v.C_i Delta + (Pi/4) w_j v.C_j Delta,
+    // which saves the scaled vectors A, B, G (~9 DP instructions per pair).
+    const double Dx = -dx, Dy = -dy, Dz = -dz;
+    const double CiDx = ci11 * Dx + ci12 * Dy + ci13 * Dz;
+    const double CiDy = ci12 * Dx + ci22 * Dy + ci23 * Dz;
+    const double CiDz = ci13 * Dx + ci23 * Dy + ci33 * Dz;
+    const double CjDx = j1.a * Dx + j1.b * Dy + j1.c * Dz;
+    const double CjDy = j1.b * Dx + j2.a * Dy + j2.b * Dz;
+    const double CjDz = j1.c * Dx + j2.b * Dy + j2.c * Dz;
+    const double vx = vxi - j3.a, vy = vyi - j3.b, vz = vzi - j3.c;
+    const double rv = dx * vx + dy * vy + dz * vz;
+    double Pi = 0.0;
+    if (rv < 0.0) {
+      const Rec4 j4 = ldg4(rcur + 4);
+      const double hbar = 0.5 * (hi + j4.a);
+      const double cbar = 0.5 * (ci + j4.b);
+      const double rhobar = 0.5 * (rhoi + j4.c);
+      // mu = hbar rv / D, Pi = (-alpha cbar mu + beta mu^2) / rhobar with one
+      // division: q = 1 / (D rhobar), 1/D = rhobar q, 1/rhobar = D q
+      const double D = fma(eps * hbar, hbar, r2);
+      const double q = 1.0 / (D * rhobar);
+      const double mu = hbar * rv * (rhobar * q);
+      Pi = (fma(beta, mu, -alpha * cbar) * mu) * (D * q);
+    }
+    const double mj = j2.d, prj = j3.d;
+    const double ka = (pri + 0.5 * Pi) * wi, kb = (prj + 0.5 * Pi) * wj;
+    ax -= mj * fma(ka, CiDx, kb * CjDx);
+    ay -= mj * fma(ka, CiDy, kb * CjDy);
+    az -= mj * fma(ka, CiDz, kb * CjDz);
+    const double vCi = vx * CiDx + vy * CiDy + vz * CiDz;
+    const double vCj = vx * CjDx + vy * CjDy + vz * CjDz;
+    de += mj * fma((pri + 0.25 * Pi) * wi, vCi, 0.25 * Pi * wj * vCj);
+  }
+  F.ax[i] = ax;
+  F.ay[i] = ay;
+  F.az[i] = az;
+  F.du[i] = de;
+}
+
+__global__ void __launch_bounds__(128, 4) momentum_energy_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   const bool active = i < F.n;
   unsigned long long hc = ~0ull;
   if (active) {
     const Geom g = load_geom(F.ds, P);
-    const Rec4* __restrict__ rec = F.rec_m;
-    const Rec4* mi = rec + (int64_t)kRecM * i;
-    const Rec4 i0 = mi[0], i1 = mi[1], i2 = mi[2], i3 = mi[3], i4 = mi[4];
-    const double xi = i0.a, yi = i0.b, zi = i0.c, qi = i0.d;
-    const double ci11 = i1.a, ci12 = i1.b, ci13 = i1.c, khi = i1.d;
-    const double ci22 = i2.a, ci23 = i2.b, ci33 = i2.c;
-    const double vxi = i3.a, vyi = i3.b, vzi = i3.c, pri = i3.d;
-    const double hi = i4.a, ci = i4.b, rhoi = i4.c;
-    const double alpha = P.av_alpha, beta = P.av_beta, eps = P.av_eps;
-    const int nci = min(F.nc[i], F.ngmax);
-    double ax = 0, ay = 0, az = 0, de = 0;
-    const int32_t* __restrict__ nb = F.nbr + i;
-    // software pipeline: neighbour index three ahead, the position chunk (needed
-    // first) two ahead; the other chunks are loaded at the top of the iteration
-    // and arrive while the two sinc polynomials run.
-    const int64_t cap = F.cap;
-    const Rec4* r0 = rec + (int64_t)kRecM * (nci > 0 ? __ldg(nb) : 0);
-    const Rec4* r1 = rec + (int64_t)kRecM * (nci > 1 ? __ldg(nb + cap) : 0);
-    int jn = nci > 2 ? __ldg(nb + 2 * cap) : 0;
-    Rec4 p0 = ldg4(r0), p1 = ldg4(r1);
-    for (int k = 0; k < nci; ++k) {
-      const Rec4* rcur = r0;
-      const Rec4 j1 = ldg4(rcur + 1), j2 = ldg4(rcur + 2), j3 = ldg4(rcur + 3);
-      const Rec4 j0 = p0;
-      p0 = p1;
-      r0 = r1;
-      if (k + 2 < nci) {
-        r1 = rec + (int64_t)kRecM * jn;
-        p1 = ldg4(r1);
-      }
-      if (k + 3 < nci) jn = __ldg(nb + (int64_t)(k + 3) * cap);
-      double dx, dy, dz;
-      pair_d(g, xi, yi, zi, j0.a, j0.b, j0.c, dx, dy, dz);
-      const double r2 = dx * dx + dy * dy + dz * dz;
-      const double wi = khi * sinc6_t(r2 * qi);
-      const double tj = r2 * j0.d;
-      const double wj = tj < kPi2 ? j1.d * sinc6_t(tj) : 0.0;
-      // Delta = -d.  With A = w_i C_i Delta, B = w_j C_j Delta, G = (A+B)/2 the
-      // pair terms regroup exactly (up to rounding) as
-      //   (p_i/rho_i^2) A + (p_j/rho_j^2) B + Pi G
-      //     = (p_i/rho_i^2 + Pi/2) w_i C_i Delta + (p_j/rho_j^2 + Pi/2) w_j C_j Delta,
-      //   (p_i/rho_i^2) v.A + Pi/2 v.G
-      //     = (p_i/rho_i^2 + Pi/4) w_i v.C_i Delta + (Pi/4) w_j v.C_j Delta,
-      // which saves the scaled vectors A, B, G (~9 DP instructions per pair).
-      const double Dx = -dx, Dy = -dy, Dz = -dz;
-      const double CiDx = ci11 * Dx + ci12 * Dy + ci13 * Dz;
-      const double CiDy = ci12 * Dx + ci22 * Dy + ci23 * Dz;
-      const double CiDz = ci13 * Dx + ci23 * Dy + ci33 * Dz;
-      const double CjDx = j1.a * Dx + j1.b * Dy + j1.c * Dz;
-      const double CjDy = j1.b * Dx + j2.a * Dy + j2.b * Dz;
-      const double CjDz = j1.c * Dx + j2.b * Dy + j2.c * Dz;
-      const double vx = vxi - j3.a, vy = vyi - j3.b, vz = vzi - j3.c;
-      const double rv = dx * vx + dy * vy + dz * vz;
-      double Pi = 0.0;
-      if (rv < 0.0) {
-        const Rec4 j4 = ldg4(rcur + 4);
-        const double hbar = 0.5 * (hi + j4.a);
-        const double cbar = 0.5 * (ci + j4.b);
-        const double rhobar = 0.5 * (rhoi + j4.c);
-        // mu = hbar rv / D, Pi = (-alpha cbar mu + beta mu^2) / rhobar with one
-        // division: q = 1 / (D rhobar), 1/D = rhobar q, 1/rhobar = D q
-        const double D = fma(eps * hbar, hbar, r2);
-        const double q = 1.0 / (D * rhobar);
-        const double mu = hbar * rv * (rhobar * q);
-        Pi = (fma(beta, mu, -alpha * cbar) * mu) * (D * q);
-      }
-      const double mj = j2.d, prj = j3.d;
-      const double ka = (pri + 0.5 * Pi) * wi, kb = (prj + 0.5 * Pi) * wj;
-      ax -= mj * fma(ka, CiDx, kb * CjDx);
-      ay -= mj * fma(ka, CiDy, kb * CjDy);
-      az -= mj * fma(ka, CiDz, kb * CjDz);
-      const double vCi = vx * CiDx + vy * CiDy + vz * CiDz;
-      const double vCj = vx * CjDx + vy * CjDy + vz * CjDz;
-      de += mj * fma((pri + 0.25 * Pi) * wi, vCi, 0.25 * Pi * wj * vCj);
-    }
-    F.ax[i] = ax;
-    F.ay[i] = ay;
-    F.az[i] = az;
-    F.du[i] = de;
-    hc = ord_of(__ddiv_rn(hi, ci));
+    const Rec4* mi = F.rec_m + (int64_t)kRecM * i;
+    const Rec4 i0 = mi[0], i4 = mi[4];
+    if (__any_sync(__activemask(), needs_wrap(g, i0.a, i0.b, i0.c, i4.a)))
+      momentum_body<true>(F, P, g, i);
+    else
+      momentum_body<false>(F, P, g, i);
+    hc = ord_of(__ddiv_rn(i4.a, i4.b));
   }
 #pragma unroll
   for (int off = 16; off > 0; off >>= 1) {
