@@ -23,6 +23,15 @@ constexpr double kPi = 3.14159265358979323846;
 constexpr double kPi2Over4 = kPi * kPi / 4.0;
 constexpr double kPi2 = kPi * kPi;
 
+// Block sizes of the neighbour sums: one large CTA per SM (the register file
+// allows 1024 x 64, 768 x 85, 512 x 128) keeps an SM on one run of consecutive
+// (Morton-adjacent) targets, so the gathered records of its warps overlap in L1
+// instead of coming from several distant regions (momentum 11.5 -> 11.0 ms; a
+// persistent contiguous-range grid was slower: spills and tail imbalance).
+constexpr int kDensThreads = 1024;
+constexpr int kIadThreads = 768;
+constexpr int kMomThreads = 512;
+
 struct Geom {
   double L[3], H[3], lo[3], hi[3];
   bool per[3];
@@ -115,7 +124,7 @@ __device__ __forceinline__ void density_body(const Fields& F, const Params& P, c
   F.wk[i] = kh3;
 }
 
-__global__ void __launch_bounds__(256, 4) density_kernel(Fields F, Params P) {
+__global__ void __launch_bounds__(kDensThreads, 1024 / kDensThreads) density_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= F.n) return;
   const Geom g = load_geom(F.ds, P);
@@ -216,7 +225,7 @@ __device__ __forceinline__ void iad_body(const Fields& F, const Geom& g, int64_t
   st4(rm + 4, F.f[FH][i], F.c[i], F.rho[i], 0.0);
 }
 
-__global__ void __launch_bounds__(256, 3) iad_kernel(Fields F, Params P) {
+__global__ void __launch_bounds__(kIadThreads, 768 / kIadThreads) iad_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= F.n) return;
   const Geom g = load_geom(F.ds, P);
@@ -318,7 +327,7 @@ __device__ __forceinline__ void momentum_body(const Fields& F, const Params& P, 
   F.du[i] = de;
 }
 
-__global__ void __launch_bounds__(128, 4) momentum_energy_kernel(Fields F, Params P) {
+__global__ void __launch_bounds__(kMomThreads, 512 / kMomThreads) momentum_energy_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   const bool active = i < F.n;
   unsigned long long hc = ~0ull;
@@ -406,7 +415,7 @@ void launch_refresh_rec_m(const Fields& F, cudaStream_t st) {
 // ------------------------------------------------------------------ launchers
 void launch_density(const Fields& F, const Params& P, cudaStream_t st) {
   if (F.n == 0) return;
-  density_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F, P);
+  density_kernel<<<(unsigned)div_up(F.n, kDensThreads), kDensThreads, 0, st>>>(F, P);
   note_launch();
 }
 void launch_eos(const Fields& F, const Params& P, cudaStream_t st) {
@@ -416,12 +425,12 @@ void launch_eos(const Fields& F, const Params& P, cudaStream_t st) {
 }
 void launch_iad(const Fields& F, const Params& P, cudaStream_t st) {
   if (F.n == 0) return;
-  iad_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F, P);
+  iad_kernel<<<(unsigned)div_up(F.n, kIadThreads), kIadThreads, 0, st>>>(F, P);
   note_launch();
 }
 void launch_momentum_energy(const Fields& F, const Params& P, cudaStream_t st) {
   if (F.n == 0) return;
-  momentum_energy_kernel<<<(unsigned)div_up(F.n, 128), 128, 0, st>>>(F, P);
+  momentum_energy_kernel<<<(unsigned)div_up(F.n, kMomThreads), kMomThreads, 0, st>>>(F, P);
   note_launch();
 }
 void launch_timestep(const Fields& F, const Params& P, cudaStream_t st) {
