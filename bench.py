@@ -57,6 +57,8 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--energy-steps", type=int, default=60,
                     help="steps for the whole-step energy (>= ~2 s: the counter ticks every ~100 ms)")
+    ap.add_argument("--trace-seconds", type=float, default=1.5,
+                    help="seconds of steps under the NVML DVFS trace (Fig. 9); 0 = off")
     ap.add_argument("--cpu-sample", type=int, default=0, help="oracle targets (0 = auto)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--out", default=None)
@@ -202,6 +204,38 @@ def measure_energy(sim, sph, n, args, gpu_index):
     out["phases"]["update"] = {"ms": ms_upd, "J": ms_upd * 1e-3 * out["step"]["W"], "W": out["step"]["W"],
                                "reps": 0, "note": "not repeatable; step-average power x time"}
     out["phase_J_sum_vs_step"] = (sum(p["J"] or 0.0 for p in out["phases"].values()) / step_J)
+    return out
+
+
+def dvfs_trace(sim, sph, seconds):
+    """Fig. 9 analog: SM clock and board power the driver picks while
+    each phase runs, from sph_trace_start's NVML sampling thread over ~`seconds`
+    of back-to-back steps at default (DVFS) clocks.  Samples are tagged with the
+    phase the device is executing (a device-written marker, not host timing)."""
+    import time
+    import numpy as np
+    try:
+        sim.trace_start(period_ms=1.0, capacity=1 << 18)
+    except sph.SphError as e:
+        return {"available": False, "why": str(e)}
+    t0 = time.perf_counter()
+    steps = 0
+    while time.perf_counter() - t0 < seconds:
+        sim.step()
+        steps += 1
+    tr = sim.trace_stop(capacity=1 << 18)
+    out = {"available": True, "steps": steps, "samples": int(tr.size),
+           "query_ms_median": float(np.median(tr["query_us"])) / 1e3 if tr.size else None,
+           "phases": {}}
+    for p, name in enumerate(sph.PHASES):
+        sel = tr[tr["phase"] == p]
+        if sel.size:
+            out["phases"][name] = {"samples": int(sel.size),
+                                   "sm_mhz_median": float(np.median(sel["sm_mhz"])),
+                                   "power_w_mean": float(sel["power_mw"].mean()) / 1e3}
+    gap = tr[tr["phase"] < 0]
+    if gap.size:
+        out["between_phases"] = {"samples": int(gap.size), "sm_mhz_median": float(np.median(gap["sm_mhz"]))}
     return out
 
 
@@ -430,6 +464,7 @@ def main():
                "path": "sph_set_particles(pinned host) + sph_step + sph_get_field x11 (host)"}
 
     energy = measure_energy(sim, sph, n, args, local) if args.energy_steps > 0 else None
+    trace = dvfs_trace(sim, sph, args.trace_seconds) if args.trace_seconds > 0 else None
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -452,7 +487,7 @@ def main():
                            "search_candidates_per_target": infos[-1]["search_candidates"] / n,
                            "search_passes_per_warp": infos[-1]["search_passes"] / (n / 32)},
                 "phase_ms": phase_ms, "fp64_other": other, "roofline": roofline, "e2e": e2e,
-                "energy": energy, "cpu_baseline": cpu, "clocks": clk.summary(),
+                "energy": energy, "dvfs_trace": trace, "cpu_baseline": cpu, "clocks": clk.summary(),
                 "gpu_launches": launches}
         s = json.dumps(line)
         print(s, flush=True)

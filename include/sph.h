@@ -164,6 +164,17 @@ typedef struct sph_energy_row {
   int32_t available;        /* 1 if joules are valid                               */
 } sph_energy_row;
 
+/* One sample of the DVFS trace (Fig. 9: the SM clock the driver
+ * picks while each function runs, over a few time steps). */
+typedef struct sph_trace_sample {
+  double t_ms;              /* host steady-clock time since sph_trace_start      */
+  int32_t phase;            /* sph_phase running on the device, -1 between phases */
+  uint32_t sm_mhz;          /* nvmlDeviceGetClockInfo(NVML_CLOCK_SM)              */
+  uint32_t power_mw;        /* nvmlDeviceGetPowerUsage                            */
+  uint32_t query_us;        /* time the three NVML queries of this sample took    */
+  uint64_t energy_mj;       /* nvmlDeviceGetTotalEnergyConsumption                */
+} sph_trace_sample;
+
 typedef struct sph_ctx sph_ctx;
 
 /* --- configuration and lifetime --------------------------------------------- */
@@ -316,6 +327,21 @@ int sph_kernel_launches(int64_t* count);
  * so reps should make the call last >= 1 s.  Synchronises. */
 int sph_repeat_phase(sph_ctx* ctx, int phase, int reps, double* ms_per_call,
                      double* joules_per_call);
+
+/* DVFS trace (Fig. 9).  sph_trace_start launches a host thread that
+ * samples NVML (SM clock, power, energy counter) every period_ms (>= 0.1; a
+ * sample is taken back to back when the NVML queries themselves take longer --
+ * several ms on a B200 host, see query_us) into a
+ * buffer of `capacity` samples, each tagged with the phase the device is running:
+ * while a trace is active, every phase writes its id (and -1 when it ends) into
+ * a pinned, device-mapped host word from the stream (one 1-thread kernel per
+ * edge, so the tag follows the device, not the asynchronous host).  The pinned
+ * word (4 bytes, cudaHostAlloc) is the only allocation the library makes.
+ * SPH_ERR_NVML when NVML is unavailable, SPH_ERR_STATE if a trace is running.
+ * sph_trace_stop joins the thread and copies min(cap, taken) samples in time
+ * order to `out` (may be NULL with cap = 0 to discard); *n = samples taken. */
+int sph_trace_start(sph_ctx* ctx, double period_ms, int64_t capacity);
+int sph_trace_stop(sph_ctx* ctx, sph_trace_sample* out, int64_t cap, int64_t* n);
 
 #ifdef __cplusplus
 }

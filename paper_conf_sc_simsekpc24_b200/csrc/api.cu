@@ -7,7 +7,9 @@
 #include <string.h>
 
 #include <algorithm>
+#include <atomic>
 #include <chrono>
+#include <thread>
 #include <vector>
 
 #include "nvml_dyn.h"
@@ -85,6 +87,16 @@ struct sph_ctx {
   unsigned current_lock = 0;
   bool locked_any = false;
   bool rec_m_dirty = false;
+  // DVFS trace (sph_trace_start / sph_trace_stop)
+  struct Trace {
+    std::thread th;
+    std::atomic<bool> run{false};
+    bool active = false;
+    volatile int* word = nullptr;  // pinned, device-mapped: the running phase
+    int* word_dev = nullptr;
+    std::vector<sph_trace_sample> buf;
+    int64_t taken = 0;
+  } trace;
 };
 
 namespace {
@@ -165,7 +177,20 @@ void apply_clock(sph_ctx* c, int p) {
   }
 }
 
+__global__ void trace_mark_kernel(int* word, int phase) {
+  *(volatile int*)word = phase;
+  __threadfence_system();
+}
+
+// Tags the DVFS trace with the phase the stream reaches next (trace active only).
+void trace_mark(sph_ctx* c, int phase) {
+  if (!c->trace.active) return;
+  trace_mark_kernel<<<1, 1, 0, c->st>>>(c->trace.word_dev, phase);
+  note_launch();
+}
+
 int phase_begin(sph_ctx* c, int p) {
+  trace_mark(c, p);
   if (c->pending[p]) {
     cudaEventSynchronize(c->ev[p][1]);
     collect_phase(c, p);
@@ -183,6 +208,7 @@ int phase_begin(sph_ctx* c, int p) {
 int phase_end(sph_ctx* c, int p) {
   int rc = cuda_check(c, cudaEventRecord(c->ev[p][1], c->st), "phase kernels");
   if (rc) return rc;
+  trace_mark(c, -1);
   c->pending[p] = true;
   c->rows[p].calls++;
   if (c->cfg.accounting == SPH_ACCOUNTING_PHASE) {
@@ -498,6 +524,8 @@ int sph_init(const sph_config* cfg, void* arena, size_t arena_bytes, void* strea
 
 void sph_finalize(sph_ctx* c) {
   if (!c) return;
+  if (c->trace.active) sph_trace_stop(c, nullptr, 0, nullptr);
+  if (c->trace.word) cudaFreeHost((void*)c->trace.word);
   if (c->locked_any) c->nvml.reset_sm_clock();
   c->nvml.shutdown();
   if (!c->poisoned) cudaStreamSynchronize(c->st);
@@ -952,3 +980,65 @@ int sph_repeat_phase(sph_ctx* c, int phase, int reps, double* ms_per_call, doubl
 }
 
 }  // extern "C"
+
+// ------------------------------------------------------------------ DVFS trace
+int sph_trace_start(sph_ctx* c, double period_ms, int64_t capacity) {
+  int rc = check_ready(c, S_INIT, "sph_trace_start");
+  if (rc) return rc;
+  if (!(period_ms >= 0.1) || capacity < 1) return fail(c, SPH_ERR_ARG, "period_ms >= 0.1 and capacity >= 1 required");
+  if (c->trace.active) return fail(c, SPH_ERR_STATE, "a trace is already running");
+  if (!c->nvml.ok) return fail(c, SPH_ERR_NVML, "NVML unavailable: %s", c->nvml.err);
+  if (!c->trace.word) {
+    void* h = nullptr;
+    if ((rc = cuda_check(c, cudaHostAlloc(&h, sizeof(int), cudaHostAllocMapped), "cudaHostAlloc"))) return rc;
+    void* d = nullptr;
+    if ((rc = cuda_check(c, cudaHostGetDevicePointer(&d, h, 0), "cudaHostGetDevicePointer"))) return rc;
+    c->trace.word = (volatile int*)h;
+    c->trace.word_dev = (int*)d;
+  }
+  *c->trace.word = -1;
+  c->trace.buf.assign((size_t)capacity, sph_trace_sample{});
+  c->trace.taken = 0;
+  c->trace.run.store(true);
+  c->trace.active = true;
+  sph_ctx::Trace* T = &c->trace;
+  Nvml* nv = &c->nvml;
+  c->trace.th = std::thread([T, nv, period_ms]() {
+    using clk = std::chrono::steady_clock;
+    const auto t0 = clk::now();
+    const auto dt = std::chrono::duration_cast<clk::duration>(std::chrono::duration<double, std::milli>(period_ms));
+    auto next = t0;
+    while (T->run.load(std::memory_order_relaxed)) {
+      sph_trace_sample s{};
+      const auto q0 = clk::now();
+      s.t_ms = std::chrono::duration<double, std::milli>(q0 - t0).count();
+      s.phase = *T->word;
+      unsigned v = 0;
+      if (nv->sm_clock_mhz(&v)) s.sm_mhz = v;
+      if (nv->power_mw(&v)) s.power_mw = v;
+      unsigned long long e = 0;
+      if (nv->energy_mj(&e)) s.energy_mj = e;
+      s.query_us = (uint32_t)std::chrono::duration<double, std::micro>(clk::now() - q0).count();
+      if (T->taken < (int64_t)T->buf.size()) T->buf[(size_t)T->taken] = s;
+      ++T->taken;
+      next += dt;
+      const auto now = clk::now();
+      if (next < now) next = now;
+      std::this_thread::sleep_until(next);
+    }
+  });
+  return SPH_OK;
+}
+
+int sph_trace_stop(sph_ctx* c, sph_trace_sample* out, int64_t cap, int64_t* n) {
+  if (!c) return fail(nullptr, SPH_ERR_ARG, "sph_trace_stop: null context");
+  if (!c->trace.active) return fail(c, SPH_ERR_STATE, "no trace running");
+  if (cap < 0 || (cap > 0 && !out)) return fail(c, SPH_ERR_ARG, "bad output buffer");
+  c->trace.run.store(false);
+  if (c->trace.th.joinable()) c->trace.th.join();
+  c->trace.active = false;
+  const int64_t m = std::min<int64_t>(std::min<int64_t>(c->trace.taken, (int64_t)c->trace.buf.size()), cap);
+  for (int64_t k = 0; k < m; ++k) out[k] = c->trace.buf[(size_t)k];
+  if (n) *n = c->trace.taken;
+  return SPH_OK;
+}

@@ -36,8 +36,9 @@
 // scratch of the resident CTAs, ~70 MB, stays in L2); when a warp has finished
 // its targets, every lane copies its row to the column-major list nbr[k*cap + i]
 // (one 128-B line per store instruction) that the neighbour sums read.  The
-// kernel is persistent: a grid of (SMs x resident CTAs) CTAs strides over the
-// 128-target tiles, so the scratch is indexed by blockIdx.
+// kernel is persistent (a grid of SMs x resident CTAs, so the scratch is indexed
+// by blockIdx and warp); each warp takes 32-target tiles from an atomic counter,
+// in order (dynamic schedule: no tail imbalance, adjacent tiles run together).
 // Bound: issue (fp32 + integer work per candidate test, ~880 candidates per
 // warp of 32 targets at 100 neighbours).  Algorithmic bytes: pos4, x, y, z, h in
 // (48 B), nc out (4 B), the list out (4 B per neighbour).
@@ -564,11 +565,15 @@ __global__ void __launch_bounds__(kNbrThreads, 6) neighbors_kernel(Fields F, Par
   }
   // this warp's 32 scratch rows (row of lane l: rows + l * nrows_ld)
   int32_t* const rows = F.nrows + ((int64_t)blockIdx.x * kNbrThreads + warp * 32) * F.nrows_ld;
-  const int64_t ntiles = div_up(F.n, kNbrThreads);
-  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-    const int64_t i = tile * kNbrThreads + threadIdx.x;
+  // warps take 32-target tiles dynamically, in order (Morton-adjacent tiles run
+  // at about the same time: L2 locality of the candidate data; no tail imbalance)
+  while (true) {
+    unsigned long long wt = 0;
+    if (lane == 0) wt = atomicAdd(&F.ds->nbr_next, 1ull);
+    wt = __shfl_sync(0xffffffffu, wt, 0);
+    const int64_t i = (int64_t)wt * 32 + lane;
+    if ((int64_t)wt * 32 >= F.n) break;
     const bool active = i < F.n;
-    if (!__any_sync(0xffffffffu, active)) continue;  // whole warp past the end
     const Target t = make_target(F, B, i, active);
     int cc[3] = {0, 0, 0};
     uint32_t ckey = 0;
@@ -655,6 +660,7 @@ void launch_neighbors(const Fields& F, const Params& P, cudaStream_t st) {
     resident = std::max(1, std::min(kNbrSlots, sms * std::max(per, 1)));
   }
   const int64_t grid = std::min<int64_t>(div_up(F.n, kNbrThreads), resident);
+  cudaMemsetAsync(&F.ds->nbr_next, 0, sizeof(unsigned long long), st);
   neighbors_kernel<<<(unsigned)grid, kNbrThreads, 0, st>>>(F, P);
   note_launch();
 }

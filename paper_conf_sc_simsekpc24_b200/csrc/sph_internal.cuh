@@ -46,6 +46,7 @@ struct DevScalars {
   double t, dt, dt_prev;
   int first;
   int pad;
+  unsigned long long nbr_next;    // neighbour search: next 32-target tile (dynamic schedule)
 };
 
 // 32-byte record: one 256-bit load (LDG.E.256 on sm_100a).

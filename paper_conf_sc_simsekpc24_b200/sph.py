@@ -69,6 +69,11 @@ class EnergyRow(C.Structure):
                 ("locked_mhz", C.c_uint32), ("available", C.c_int32)]
 
 
+class TraceSample(C.Structure):
+    _fields_ = [("t_ms", C.c_double), ("phase", C.c_int32), ("sm_mhz", C.c_uint32),
+                ("power_mw", C.c_uint32), ("query_us", C.c_uint32), ("energy_mj", C.c_uint64)]
+
+
 # Every symbol include/sph.h declares (checked by tests/test_abi.py).
 EXPORTS = ("sph_config_default", "sph_workspace_size", "sph_init", "sph_finalize",
            "sph_last_error", "sph_phase_name", "sph_set_particles", "sph_set_time",
@@ -77,7 +82,8 @@ EXPORTS = ("sph_config_default", "sph_workspace_size", "sph_init", "sph_finalize
            "sph_timestep", "sph_update", "sph_step", "sph_set_clock_policy",
            "sph_energy_report", "sph_energy_reset", "sph_energy_counter_mj", "sph_repeat_phase",
            "sph_set_accounting", "sph_kernel_launches", "sph_set_field",
-           "sph_get_local_min_hc", "sph_set_global_min_hc", "sph_get_neighbor_rows")
+           "sph_get_local_min_hc", "sph_set_global_min_hc", "sph_get_neighbor_rows",
+           "sph_trace_start", "sph_trace_stop")
 GHOST_BIT = 1 << 62
 
 _lib = None
@@ -127,6 +133,8 @@ def load(build_if_missing: bool = True):
     L.sph_get_local_min_hc.argtypes = [P, C.POINTER(D)]
     L.sph_set_global_min_hc.argtypes = [P, D]
     L.sph_kernel_launches.argtypes = [C.POINTER(I64)]
+    L.sph_trace_start.argtypes = [P, D, I64]
+    L.sph_trace_stop.argtypes = [P, V, I64, C.POINTER(I64)]
     _lib = L
     return L
 
@@ -366,3 +374,17 @@ class Simulation:
         ms, j = C.c_double(), C.c_double()
         self._ok(self.L.sph_repeat_phase(self.ctx, PHASES.index(phase), reps, C.byref(ms), C.byref(j)))
         return ms.value, (j.value if j.value >= 0 else None)
+
+    def trace_start(self, period_ms: float = 1.0, capacity: int = 1 << 20):
+        """sph_trace_start: NVML DVFS sampling thread (Fig. 9)."""
+        self._ok(self.L.sph_trace_start(self.ctx, float(period_ms), int(capacity)))
+
+    def trace_stop(self, capacity: int = 1 << 20):
+        """sph_trace_stop: the samples as a numpy structured array (t_ms, phase,
+        sm_mhz, power_mw, energy_mj)."""
+        buf = (TraceSample * capacity)()
+        n = C.c_int64()
+        self._ok(self.L.sph_trace_stop(self.ctx, C.cast(buf, C.c_void_p), capacity, C.byref(n)))
+        m = min(int(n.value), capacity)
+        a = np.ctypeslib.as_array(buf)[:m].copy()
+        return a

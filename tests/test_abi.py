@@ -65,3 +65,10 @@ def test_null_context_calls_fail_cleanly():
     assert L.sph_build_tree(None) == 1
     assert L.sph_step(None, None) == 1
     L.sph_finalize(None)
+
+
+def test_trace_entry_points_reject_null_context():
+    L = sph.load()
+    n = C.c_int64()
+    assert L.sph_trace_start(None, C.c_double(1.0), C.c_int64(10)) == 1  # SPH_ERR_ARG
+    assert L.sph_trace_stop(None, None, C.c_int64(0), C.byref(n)) == 1
