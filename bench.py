@@ -57,6 +57,8 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--energy-steps", type=int, default=60,
                     help="steps for the whole-step energy (>= ~2 s: the counter ticks every ~100 ms)")
+    ap.add_argument("--stir", action="store_true",
+                    help="turbulence driving (OU stirring, SURVEY 8(f)-3) inside every step")
     ap.add_argument("--trace-seconds", type=float, default=1.5,
                     help="seconds of steps under the NVML DVFS trace (Fig. 9); 0 = off")
     ap.add_argument("--cpu-sample", type=int, default=0, help="oracle targets (0 = auto)")
@@ -374,8 +376,13 @@ def main():
     torch.cuda.set_device(local)
     w = make_workload(args.workload, rank)
     n = w.n
-    sim = sph.Simulation(w.params, n_capacity=n, device=local)
+    stir_steps = 8192 if args.stir else 0
+    sim = sph.Simulation(w.params, n_capacity=n, device=local, stir_steps=stir_steps)
     stream = sim.stream
+    if args.stir:
+        from paper_conf_sc_simsekpc24_b200 import ics
+        si = ics.stir_inputs(sph.stir_modes(), stir_steps)
+        sim.stir_init(si.sigma, si.t_decay, si.zeta, si.w, si.noise)
 
     def barrier():
         if world > 1:
@@ -477,7 +484,8 @@ def main():
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-                "config": {"workload": args.workload, "n_particles_per_gpu": n,
+                "config": {"workload": args.workload + ("+stir" if args.stir else ""),
+                           "n_particles_per_gpu": n,
                            "n_particles_total": n * world,
                            "parallelism": "single GPU" if world == 1 else
                            f"{world} independent replicas (SFC decomposition not yet built)",

@@ -88,7 +88,9 @@ typedef enum sph_phase {
   SPH_PHASE_MOMENTUM_ENERGY = 7, /* momentum + energy + AV, local dt min (item 8) */
   SPH_PHASE_TIMESTEP = 8,        /* global dt (item 9; the P:220 collective)      */
   SPH_PHASE_UPDATE = 9,          /* positions, velocities, energy, h (item 10)    */
-  SPH_NPHASES = 10
+  SPH_PHASE_STIR = 10,           /* turbulence driving; runs after
+                                    MOMENTUM_ENERGY, before TIMESTEP, when enabled */
+  SPH_NPHASES = 11
 } sph_phase;
 
 typedef enum sph_clock_mode {
@@ -133,7 +135,9 @@ typedef struct sph_config {
   int32_t device;           /* CUDA device ordinal the arena lives on              */
   int32_t accounting;       /* sph_accounting_mode                                 */
   int32_t rank, nranks;     /* reserved for SFC domain decomposition (1 rank now)  */
-  int32_t reserved[16];
+  int32_t stir_steps;       /* capacity (steps) of the driving-noise table; 0 = no
+                               turbulence driving (sph_stir_init)                  */
+  int32_t reserved[15];
 } sph_config;
 
 typedef struct sph_nbr_stats {
@@ -174,6 +178,26 @@ typedef struct sph_trace_sample {
   uint32_t query_us;        /* time the three NVML queries of this sample took    */
   uint64_t energy_mj;       /* nvmlDeviceGetTotalEnergyConsumption                */
 } sph_trace_sample;
+
+/* Turbulence driving (Ornstein-Uhlenbeck stirring of the
+ * Subsonic Turbulence workload).  The mode set is fixed: the
+ * SPH_STIR_NMODES integer wave vectors n with 1 <= |n|^2 <= 9 in the half space
+ * (n_x > 0, or n_x = 0 and n_y > 0, or n_x = n_y = 0 and n_z > 0), in
+ * lexicographic order of (n_x, n_y, n_z) (sph_stir_modes), k_a = 2 pi n_a / L_a.
+ * Per mode the OU state holds a complex 3-vector A (6 doubles: Re x, Im x, Re y,
+ * Im y, Re z, Im z).  One STIR phase (step s = number of phases run so far):
+ *   A <- f A + sigma sqrt(1 - f^2) xi_s,  f = exp(-dt_prev / t_decay)
+ *   (xi_s = row s of the caller's Gaussian noise table: the random numbers are
+ *   inputs, so the oracle draws nothing);
+ *   A^ = zeta P_perp A + (1 - zeta) P_par A  (P_perp = I - k^k^T, P_par = k^k^T);
+ *   a_i += 2 sum_m w_m Re( A^_m exp(i k_m . (x_i - box_min)) ).
+ * Weights w_m, sigma, t_decay and zeta are conventions (parity unpinned). */
+#define SPH_STIR_NMODES 61
+typedef struct sph_stir_params {
+  double sigma;             /* stationary rms of each OU component                 */
+  double t_decay;           /* OU correlation time                                 */
+  double sol_weight;        /* zeta: 1 = solenoidal, 0 = compressive               */
+} sph_stir_params;
 
 typedef struct sph_ctx sph_ctx;
 
@@ -327,6 +351,31 @@ int sph_kernel_launches(int64_t* count);
  * so reps should make the call last >= 1 s.  Synchronises. */
 int sph_repeat_phase(sph_ctx* ctx, int phase, int reps, double* ms_per_call,
                      double* joules_per_call);
+
+/* --- turbulence driving ------------------------------------ */
+
+/* The fixed mode set: writes 3 * SPH_STIR_NMODES ints (n_x, n_y, n_z per mode)
+ * to n3 (cap >= SPH_STIR_NMODES modes) and returns the mode count.  Pure. */
+int sph_stir_modes(int32_t* n3, int cap);
+
+/* Enables driving: per-mode weights w[SPH_STIR_NMODES], the initial OU state
+ * A0[6 * SPH_STIR_NMODES] (NULL = zeros) and the noise table
+ * noise[nsteps][SPH_STIR_NMODES][6] (nsteps <= cfg.stir_steps; host or device
+ * pointers per mem).  Resets the step counter.  cfg.stir_steps == 0 ->
+ * SPH_ERR_NOT_SUPPORTED.  Once enabled, sph_step runs STIR after
+ * MOMENTUM_ENERGY; a step past the end of the noise table -> SPH_ERR_CAPACITY
+ * at the next synchronising call. */
+int sph_stir_init(sph_ctx* ctx, const sph_stir_params* prm, const double* w, const double* A0,
+                  const double* noise, int64_t nsteps, int mem);
+
+/* Phase STIR alone (after sph_momentum_energy, before sph_timestep): the OU
+ * update with the previous step's dt and the driving acceleration added to
+ * a_i.  SPH_ERR_STATE when driving is not enabled. */
+int sph_stir(sph_ctx* ctx);
+
+/* The OU state A (6 * SPH_STIR_NMODES doubles, host) and the number of STIR
+ * phases run since sph_stir_init.  Synchronises. */
+int sph_stir_get_state(sph_ctx* ctx, double* A, int64_t* steps);
 
 /* DVFS trace (Fig. 9).  sph_trace_start launches a host thread that
  * samples NVML (SM clock, power, energy counter) every period_ms (>= 0.1; a

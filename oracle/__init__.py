@@ -279,11 +279,74 @@ def update(state, acc, nc, dt, dt_m1, first_step, bmin, bmax, params):
 STATE_KEYS = ("x", "y", "z", "vx", "vy", "vz", "h", "m", "u", "du_m1", "id")
 
 
-def step(state: dict, params, dt_prev: float, first_step: bool, ngmax: int | None = None):
+# --------------------------------------------------------------------------
+# Turbulence driving (oracle.c "Turbulence driving")
+STIR_NMODES = 61
+
+
+def stir_modes() -> np.ndarray:
+    n3 = np.zeros((STIR_NMODES, 3), np.int32)
+    m = lib().oracle_stir_modes(_p(n3, _I32))
+    return n3[:m]
+
+
+def stir_ou(A, xi, dt: float, sigma: float, t_decay: float) -> np.ndarray:
+    """A <- f A + sigma sqrt(1-f^2) xi, f = exp(-dt/t_decay) (returns a new array)."""
+    A = np.array(A, dtype=np.float64, copy=True)
+    xi = _d(xi)
+    lib().oracle_stir_ou(C.c_int(A.shape[0]), _p(A, _D), _p(xi, _D), C.c_double(dt),
+                         C.c_double(sigma), C.c_double(t_decay))
+    return A
+
+
+def stir_project(A, w, zeta: float, L) -> np.ndarray:
+    """B = 2 w (zeta A_perp + (1-zeta) A_par), per mode and real/imaginary part."""
+    n3 = stir_modes()
+    A, w = _d(A), _d(w)
+    B = np.zeros_like(A)
+    Lv = _d(np.asarray(L, dtype=np.float64))
+    lib().oracle_stir_project(C.c_int(A.shape[0]), _p(n3, _I32), _p(Lv, _D), _p(A, _D), _p(w, _D),
+                              C.c_double(zeta), _p(B, _D))
+    return B
+
+
+def stir_accel(x, y, z, lo, L, B):
+    """sum_m Re(B_m exp(i k_m.(x - lo))) per particle -> (ax, ay, az)."""
+    n3 = stir_modes()
+    x, y, z, B = _d(x), _d(y), _d(z), _d(B)
+    lo, L = _d(np.asarray(lo, np.float64)), _d(np.asarray(L, np.float64))
+    ax, ay, az = (np.zeros(x.size) for _ in range(3))
+    lib().oracle_stir_accel(C.c_int64(x.size), _p(x, _D), _p(y, _D), _p(z, _D), _p(lo, _D), _p(L, _D),
+                            C.c_int(B.shape[0]), _p(n3, _I32), _p(B, _D), _p(ax, _D), _p(ay, _D),
+                            _p(az, _D))
+    return ax, ay, az
+
+
+def stir_apply(stir: dict, x, y, z, dt_prev: float, bmin, bmax, acc: dict):
+    """Phase STIR: advances stir["A"] with noise row stir["step"], adds the driving
+    acceleration to acc["ax"/"ay"/"az"] in place; returns B."""
+    xi = stir["noise"][stir["step"]]
+    stir["A"] = stir_ou(stir["A"], xi, dt_prev, stir["sigma"], stir["t_decay"])
+    L = [bmax[a] - bmin[a] for a in range(3)]
+    B = stir_project(stir["A"], stir["w"], stir["zeta"], L)
+    sx, sy, sz = stir_accel(x, y, z, bmin, L, B)
+    # tolerance scale of the driven sums: sum_m |Re B| + |Im B| per component
+    scale = np.abs(B).reshape(-1, 3, 2).sum(axis=(0, 2))
+    acc["a_abs"] = acc["a_abs"] + scale[None, :]
+    acc["ax"] = acc["ax"] + sx
+    acc["ay"] = acc["ay"] + sy
+    acc["az"] = acc["az"] + sz
+    stir["step"] += 1
+    return B
+
+
+def step(state: dict, params, dt_prev: float, first_step: bool, ngmax: int | None = None,
+         stir: dict | None = None):
     """One full oracle step.  Returns (new_state, out) where new_state is in this
     step's sorted (Morton) order after the update, and ``out`` holds every
     intermediate of the step in the same order (keys, perm, nb, rho, p, c, C,
-    accelerations, dt, box)."""
+    accelerations, dt, box).  ``stir`` (optional, updated in place): driving state
+    {A, w, noise, step, sigma, t_decay, zeta}; STIR runs after momentum-energy."""
     bmin, bmax = box(state["x"], state["y"], state["z"], params)
     k = keys(state["x"], state["y"], state["z"], bmin, bmax)
     perm = sort_order(k)
@@ -301,6 +364,8 @@ def step(state: dict, params, dt_prev: float, first_step: bool, ngmax: int | Non
         raise ArithmeticError("IAD matrix singular")
     acc = momentum_energy(st["x"], st["y"], st["z"], st["vx"], st["vy"], st["vz"], st["h"],
                           st["m"], rho, p, c, Cm, bmin, bmax, params.periodic, nb, params)
+    if stir is not None:
+        acc["stir_B"] = stir_apply(stir, st["x"], st["y"], st["z"], dt_prev, bmin, bmax, acc)
     dt = timestep(st["h"], c, dt_prev, params)
     out = {"bmin": bmin, "bmax": bmax, "keys": ks, "perm": perm, "nb": nb, "rho": rho, "p": p,
            "c": c, "C": Cm, "tau": tau, "tau_abs": tabs, "dt": dt,

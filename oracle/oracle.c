@@ -426,3 +426,85 @@ void oracle_update(int64_t n, double* x, double* y, double* z, double* vx, doubl
     h[i] = hn < P->h_cap ? hn : P->h_cap;
   }
 }
+
+/* ---------------------------------------------------------------------------
+ * Turbulence driving (Ornstein-Uhlenbeck stirring of the
+ * Subsonic Turbulence workload).  PAPER.md prints no driving
+ * formula; the definitions are the ones stated in include/sph.h and DESIGN.md
+ * (reading 17), restated here:
+ *   modes: integer n with 1 <= |n|^2 <= 9 in the half space (n_x > 0, or
+ *          n_x = 0 and n_y > 0, or n_x = n_y = 0 and n_z > 0), lexicographic
+ *          in (n_x, n_y, n_z); k_a = 2 pi n_a / L_a;
+ *   OU:    A <- f A + sigma sqrt(1 - f^2) xi,  f = exp(-dt / t_decay);
+ *   projection: A^ = zeta (A - k^(k^.A)) + (1 - zeta) k^(k^.A), applied to the
+ *          real and the imaginary 3-vector of each mode; B = 2 w A^;
+ *   acceleration: a_i += sum_m [ Re(B_m) cos(phi) - Im(B_m) sin(phi) ],
+ *          phi = k_m . (x_i - box_min).
+ * A mode's 6 numbers are (Re x, Im x, Re y, Im y, Re z, Im z).
+ * ------------------------------------------------------------------------- */
+int oracle_stir_modes(int32_t* n3) {
+  int m = 0;
+  for (int nx = 0; nx <= 3; ++nx)
+    for (int ny = -3; ny <= 3; ++ny)
+      for (int nz = -3; nz <= 3; ++nz) {
+        int q = nx * nx + ny * ny + nz * nz;
+        int half = nx > 0 || (nx == 0 && ny > 0) || (nx == 0 && ny == 0 && nz > 0);
+        if (half && q >= 1 && q <= 9) {
+          n3[3 * m + 0] = nx;
+          n3[3 * m + 1] = ny;
+          n3[3 * m + 2] = nz;
+          ++m;
+        }
+      }
+  return m;
+}
+
+void oracle_stir_ou(int nm, double* A, const double* xi, double dt, double sigma, double t_decay) {
+  double f = exp(-dt / t_decay);
+  double g = sigma * sqrt(1.0 - f * f);
+  for (int k = 0; k < 6 * nm; ++k) A[k] = f * A[k] + g * xi[k];
+}
+
+void oracle_stir_project(int nm, const int32_t* n3, const double L[3], const double* A,
+                         const double* w, double zeta, double* B) {
+  for (int m = 0; m < nm; ++m) {
+    double k[3], kn = 0.0;
+    for (int a = 0; a < 3; ++a) {
+      k[a] = 2.0 * M_PI * n3[3 * m + a] / L[a];
+      kn += k[a] * k[a];
+    }
+    kn = sqrt(kn);
+    for (int a = 0; a < 3; ++a) k[a] /= kn;
+    for (int part = 0; part < 2; ++part) {
+      double v[3], kv = 0.0;
+      for (int a = 0; a < 3; ++a) {
+        v[a] = A[6 * m + 2 * a + part];
+        kv += k[a] * v[a];
+      }
+      for (int a = 0; a < 3; ++a) {
+        double par = k[a] * kv;
+        double perp = v[a] - par;
+        B[6 * m + 2 * a + part] = 2.0 * w[m] * (zeta * perp + (1.0 - zeta) * par);
+      }
+    }
+  }
+}
+
+void oracle_stir_accel(int64_t n, const double* x, const double* y, const double* z,
+                       const double lo[3], const double L[3], int nm, const int32_t* n3,
+                       const double* B, double* ax, double* ay, double* az) {
+#pragma omp parallel for schedule(static)
+  for (int64_t i = 0; i < n; ++i) {
+    double s[3] = {0.0, 0.0, 0.0};
+    const double p[3] = {x[i] - lo[0], y[i] - lo[1], z[i] - lo[2]};
+    for (int m = 0; m < nm; ++m) {
+      double phi = 0.0;
+      for (int a = 0; a < 3; ++a) phi += 2.0 * M_PI * n3[3 * m + a] * p[a] / L[a];
+      double c = cos(phi), sn = sin(phi);
+      for (int a = 0; a < 3; ++a) s[a] += B[6 * m + 2 * a] * c - B[6 * m + 2 * a + 1] * sn;
+    }
+    ax[i] += s[0];
+    ay[i] += s[1];
+    az[i] += s[2];
+  }
+}

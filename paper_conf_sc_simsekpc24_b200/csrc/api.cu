@@ -25,7 +25,7 @@ enum Stage { S_INIT = 0, S_PART, S_TREE, S_NBR, S_DENS, S_EOS, S_IAD, S_MOM, S_D
 
 const char* kPhaseNames[SPH_NPHASES] = {"keys",    "sort",    "cells", "neighbors",
                                         "density", "eos",     "iad",   "momentum_energy",
-                                        "timestep", "update"};
+                                        "timestep", "update",  "stir"};
 
 thread_local char g_err[512] = "";
 
@@ -87,6 +87,8 @@ struct sph_ctx {
   unsigned current_lock = 0;
   bool locked_any = false;
   bool rec_m_dirty = false;
+  Stir stir{};          // turbulence driving (k_stir.cu)
+  bool stir_on = false;
   // DVFS trace (sph_trace_start / sph_trace_stop)
   struct Trace {
     std::thread th;
@@ -240,6 +242,7 @@ int sync_scalars(sph_ctx* c) {
   if (s & ST_CAPACITY)
     return fail(c, SPH_ERR_CAPACITY, "neighbour count %d exceeds ngmax %d", c->h_ds.max_nc, c->cfg.ngmax);
   if (s & ST_SINGULAR) return fail(c, SPH_ERR_SINGULAR, "singular IAD matrix (det <= 0 or non-finite)");
+  if (s & ST_STIR_NOISE) return fail(c, SPH_ERR_CAPACITY, "driving noise table exhausted (%lld steps)", (long long)c->stir.nsteps);
   return SPH_OK;
 }
 
@@ -335,6 +338,7 @@ int body_simple(sph_ctx* c, int phase, int next_stage) {
       launch_update(F, c->P, c->st);
       launch_advance_time(F, c->st);
       break;
+    case SPH_PHASE_STIR: launch_stir(F, c->P, c->stir, c->st); break;
   }
   if ((rc = phase_end(c, phase))) return rc;
   c->stage = next_stage;
@@ -388,6 +392,7 @@ static int validate(const sph_config* c) {
   if (c->eos != SPH_EOS_IDEAL && c->eos != SPH_EOS_ISOTHERMAL) return fail(nullptr, SPH_ERR_ARG, "unknown eos %d", c->eos);
   if (!(c->K > 0) || !(c->dt_first > 0) || !(c->h_cap > 0)) return fail(nullptr, SPH_ERR_ARG, "K, dt_first and h_cap must be > 0");
   if (c->nranks != 1) return fail(nullptr, SPH_ERR_NOT_SUPPORTED, "nranks > 1 is not built into this library version");
+  if (c->stir_steps < 0) return fail(nullptr, SPH_ERR_ARG, "stir_steps < 0");
   return SPH_OK;
 }
 
@@ -445,6 +450,17 @@ static size_t layout(const sph_config* cfg, char* base, sph_ctx* c) {
   char* hp = take(hb);
   char* sp = take(sb);
   char* dsp = take(sizeof(DevScalars));
+  const size_t sst = (size_t)cfg->stir_steps;
+  char* sA = sst ? take(sizeof(double) * kStirModes * 6) : nullptr;
+  char* sB = sst ? take(sizeof(double) * kStirModes * 6) : nullptr;
+  char* sw = sst ? take(sizeof(double) * kStirModes) : nullptr;
+  char* sn = sst ? take(sizeof(double) * kStirModes * 6 * sst) : nullptr;
+  if (c) {
+    c->stir.A = (double*)sA;
+    c->stir.B = (double*)sB;
+    c->stir.w = (double*)sw;
+    c->stir.noise = (double*)sn;
+  }
   if (c) {
     c->keyA = (uint64_t*)kA; c->keyB = (uint64_t*)kB;
     c->valA = (uint32_t*)vA; c->valB = (uint32_t*)vB;
@@ -794,6 +810,7 @@ int sph_step(sph_ctx* c, sph_step_info* info) {
   if ((rc = body_simple(c, SPH_PHASE_EOS, S_EOS))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_IAD, S_IAD))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_MOMENTUM_ENERGY, S_MOM))) return rc;
+  if (c->stir_on && (rc = body_simple(c, SPH_PHASE_STIR, S_MOM))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_TIMESTEP, S_DT))) return rc;
   // A data error (capacity, singular, box) makes the update meaningless: check
   // the device status after the update is enqueued (one sync per step).
@@ -1041,4 +1058,56 @@ int sph_trace_stop(sph_ctx* c, sph_trace_sample* out, int64_t cap, int64_t* n) {
   for (int64_t k = 0; k < m; ++k) out[k] = c->trace.buf[(size_t)k];
   if (n) *n = c->trace.taken;
   return SPH_OK;
+}
+
+// ------------------------------------------------------------------ driving
+int sph_stir_modes(int32_t* n3, int cap) {
+  if (!n3 || cap < kStirModes) return -SPH_ERR_ARG;
+  return stir_modes(n3);
+}
+
+int sph_stir_init(sph_ctx* c, const sph_stir_params* prm, const double* w, const double* A0,
+                  const double* noise, int64_t nsteps, int mem) {
+  int rc = check_ready(c, S_INIT, "sph_stir_init");
+  if (rc) return rc;
+  if (c->cfg.stir_steps == 0) return fail(c, SPH_ERR_NOT_SUPPORTED, "driving needs cfg.stir_steps > 0 (arena room for the noise table)");
+  if (!c->cfg.periodic[0] || !c->cfg.periodic[1] || !c->cfg.periodic[2])
+    return fail(c, SPH_ERR_NOT_SUPPORTED, "driving is defined on a fully periodic box");
+  if (!prm || !w || !noise) return fail(c, SPH_ERR_ARG, "null params, weights or noise");
+  if (nsteps < 1 || nsteps > c->cfg.stir_steps) return fail(c, SPH_ERR_ARG, "nsteps must be in [1, stir_steps = %d]", c->cfg.stir_steps);
+  if (!(prm->t_decay > 0) || !(prm->sigma >= 0) || !(prm->sol_weight >= 0 && prm->sol_weight <= 1))
+    return fail(c, SPH_ERR_ARG, "need t_decay > 0, sigma >= 0, 0 <= sol_weight <= 1");
+  if (mem != SPH_MEM_HOST && mem != SPH_MEM_DEVICE) return fail(c, SPH_ERR_ARG, "mem must be HOST or DEVICE");
+  const cudaMemcpyKind k = mem == SPH_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
+  const size_t M6 = sizeof(double) * kStirModes * 6;
+  rc = cuda_check(c, cudaMemcpyAsync(c->stir.w, w, sizeof(double) * kStirModes, k, c->st), "stir w");
+  if (!rc) rc = cuda_check(c, A0 ? cudaMemcpyAsync(c->stir.A, A0, M6, k, c->st) : cudaMemsetAsync(c->stir.A, 0, M6, c->st), "stir A0");
+  if (!rc) rc = cuda_check(c, cudaMemcpyAsync(c->stir.noise, noise, M6 * (size_t)nsteps, k, c->st), "stir noise");
+  if (!rc) rc = cuda_check(c, cudaMemsetAsync(&c->ds->stir_step, 0, sizeof(unsigned long long), c->st), "stir counter");
+  if (!rc) rc = cuda_check(c, cudaStreamSynchronize(c->st), "sync");
+  if (rc) return rc;
+  c->stir.nsteps = nsteps;
+  c->stir.sigma = prm->sigma;
+  c->stir.t_decay = prm->t_decay;
+  c->stir.zeta = prm->sol_weight;
+  c->stir_on = true;
+  return SPH_OK;
+}
+
+int sph_stir(sph_ctx* c) {
+  int rc = check_ready(c, S_MOM, "sph_stir");
+  if (rc) return rc;
+  if (!c->stir_on) return fail(c, SPH_ERR_STATE, "driving not enabled (sph_stir_init)");
+  return body_simple(c, SPH_PHASE_STIR, S_MOM);
+}
+
+int sph_stir_get_state(sph_ctx* c, double* A, int64_t* steps) {
+  int rc = check_ready(c, S_INIT, "sph_stir_get_state");
+  if (rc) return rc;
+  if (!c->stir_on) return fail(c, SPH_ERR_STATE, "driving not enabled (sph_stir_init)");
+  if (A) rc = cuda_check(c, cudaMemcpyAsync(A, c->stir.A, sizeof(double) * kStirModes * 6, cudaMemcpyDeviceToHost, c->st), "stir A");
+  if (rc) return rc;
+  rc = sync_scalars(c);
+  if (steps) *steps = (int64_t)c->h_ds.stir_step;
+  return rc;
 }

@@ -28,7 +28,7 @@ constexpr int kRadix = 256;
 constexpr int kSortPasses = 8;  // 8 x 8 bits >= 63-bit keys
 
 // Device status bits (reported at the next synchronising call).
-enum DevStatus : int { ST_BOX = 1, ST_CAPACITY = 2, ST_SINGULAR = 4 };
+enum DevStatus : int { ST_BOX = 1, ST_CAPACITY = 2, ST_SINGULAR = 4, ST_STIR_NOISE = 8 };
 
 // Small block of device scalars: reductions, the integrator clock and status.
 struct DevScalars {
@@ -47,6 +47,18 @@ struct DevScalars {
   int first;
   int pad;
   unsigned long long nbr_next;    // neighbour search: next 32-target tile (dynamic schedule)
+  unsigned long long stir_step;   // STIR phases run since sph_stir_init
+};
+
+// Turbulence driving (k_stir.cu): the OU state and its inputs, in the arena.
+constexpr int kStirModes = 61;
+struct Stir {
+  double* A;        // [61][6] OU state
+  double* B;        // [61][6] 2 w_m A^_m (projected, weighted) of the current step
+  double* w;        // [61] mode weights
+  double* noise;    // [nsteps][61][6] Gaussian draws (caller's)
+  int64_t nsteps;
+  double sigma, t_decay, zeta;
 };
 
 // 32-byte record: one 256-bit load (LDG.E.256 on sm_100a).
@@ -220,4 +232,6 @@ void launch_timestep(const Fields& F, const Params& P, cudaStream_t st);
 void launch_update(const Fields& F, const Params& P, cudaStream_t st);
 void launch_advance_time(const Fields& F, cudaStream_t st);
 void launch_refresh_rec_m(const Fields& F, cudaStream_t st);
+void launch_stir(const Fields& F, const Params& P, const Stir& S, cudaStream_t st);
+int stir_modes(int32_t* n3);  // host: the fixed mode set (returns kStirModes)
 }  // namespace sph

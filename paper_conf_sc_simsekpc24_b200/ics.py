@@ -246,3 +246,28 @@ PRESETS = {
     "turbulence200": lambda: turbulence(200),
     "noh300": lambda: noh(300),
 }
+
+
+# ---------------------------------------------------------------------------
+# Turbulence-driving inputs.  Conventions of the input, not the
+# method: a parabolic spectral shape over |n| peaking at |n| = 2 (zero at 1 and
+# 3, after Federrath et al.'s stirring), seeded Gaussian OU noise, and the OU
+# parameters of a Mach ~0.3 box (sigma, t_decay ~ a large-eddy turnover / 6).
+@dataclass
+class StirInputs:
+    sigma: float
+    t_decay: float
+    zeta: float
+    w: np.ndarray       # [61] per-mode weights
+    noise: np.ndarray   # [nsteps, 61, 6] standard normal draws
+
+
+def stir_inputs(n3, nsteps: int, seed: int = 4, sigma: float = 0.05, t_decay: float = 0.5,
+                zeta: float = 1.0) -> StirInputs:
+    """Driving inputs for the mode set n3 [61, 3] (from sph.stir_modes() or
+    oracle.stir_modes(): both enumerate the same fixed set)."""
+    kn = np.sqrt((np.asarray(n3, dtype=np.float64) ** 2).sum(axis=1))
+    w = np.maximum(0.0, 1.0 - (kn - 2.0) ** 2)
+    rng = np.random.default_rng(seed)
+    noise = rng.standard_normal((nsteps, len(kn), 6))
+    return StirInputs(sigma, t_decay, zeta, w, noise)

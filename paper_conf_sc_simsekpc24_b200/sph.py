@@ -21,7 +21,8 @@ STATUS = {0: "OK", 1: "ERR_ARG", 2: "ERR_STATE", 3: "ERR_CUDA", 4: "ERR_NCCL", 5
           6: "ERR_NO_PERMISSION", 7: "ERR_NOT_SUPPORTED", 8: "ERR_CAPACITY", 9: "ERR_HCAP",
           10: "ERR_SINGULAR", 11: "ERR_BOX"}
 PHASES = ("keys", "sort", "cells", "neighbors", "density", "eos", "iad", "momentum_energy",
-          "timestep", "update")
+          "timestep", "update", "stir")
+STIR_NMODES = 61
 NPHASES = len(PHASES)
 FIELDS = ("x", "y", "z", "vx", "vy", "vz", "h", "m", "u", "du_m1", "id", "key", "nc", "rho", "p",
           "c", "c11", "c12", "c13", "c22", "c23", "c33", "ax", "ay", "az", "du")
@@ -48,7 +49,7 @@ class Config(C.Structure):
         ("dt_max_growth", C.c_double), ("dt_first", C.c_double), ("av_alpha", C.c_double),
         ("av_beta", C.c_double), ("av_eps", C.c_double), ("device", C.c_int32),
         ("accounting", C.c_int32), ("rank", C.c_int32), ("nranks", C.c_int32),
-        ("reserved", C.c_int32 * 16),
+        ("stir_steps", C.c_int32), ("reserved", C.c_int32 * 15),
     ]
 
 
@@ -69,6 +70,10 @@ class EnergyRow(C.Structure):
                 ("locked_mhz", C.c_uint32), ("available", C.c_int32)]
 
 
+class StirParams(C.Structure):
+    _fields_ = [("sigma", C.c_double), ("t_decay", C.c_double), ("sol_weight", C.c_double)]
+
+
 class TraceSample(C.Structure):
     _fields_ = [("t_ms", C.c_double), ("phase", C.c_int32), ("sm_mhz", C.c_uint32),
                 ("power_mw", C.c_uint32), ("query_us", C.c_uint32), ("energy_mj", C.c_uint64)]
@@ -83,7 +88,8 @@ EXPORTS = ("sph_config_default", "sph_workspace_size", "sph_init", "sph_finalize
            "sph_energy_report", "sph_energy_reset", "sph_energy_counter_mj", "sph_repeat_phase",
            "sph_set_accounting", "sph_kernel_launches", "sph_set_field",
            "sph_get_local_min_hc", "sph_set_global_min_hc", "sph_get_neighbor_rows",
-           "sph_trace_start", "sph_trace_stop")
+           "sph_trace_start", "sph_trace_stop", "sph_stir_modes", "sph_stir_init", "sph_stir",
+           "sph_stir_get_state")
 GHOST_BIT = 1 << 62
 
 _lib = None
@@ -133,6 +139,10 @@ def load(build_if_missing: bool = True):
     L.sph_get_local_min_hc.argtypes = [P, C.POINTER(D)]
     L.sph_set_global_min_hc.argtypes = [P, D]
     L.sph_kernel_launches.argtypes = [C.POINTER(I64)]
+    L.sph_stir_modes.argtypes = [V, I]
+    L.sph_stir_init.argtypes = [P, C.POINTER(StirParams), V, V, V, I64, I]
+    L.sph_stir.argtypes = [P]
+    L.sph_stir_get_state.argtypes = [P, V, C.POINTER(I64)]
     L.sph_trace_start.argtypes = [P, D, I64]
     L.sph_trace_stop.argtypes = [P, V, I64, C.POINTER(I64)]
     _lib = L
@@ -147,7 +157,7 @@ def kernel_launches() -> int:
 
 
 def config_from_params(params, n_capacity: int, device: int = 0, accounting: int = 0,
-                       max_cell_level: int = 8) -> Config:
+                       max_cell_level: int = 8, stir_steps: int = 0) -> Config:
     """sph_config from the StepParams preset of paper_conf_sc_simsekpc24_b200.ics."""
     L = load()
     c = Config()
@@ -164,7 +174,17 @@ def config_from_params(params, n_capacity: int, device: int = 0, accounting: int
     c.max_cell_level = int(max_cell_level)
     c.device = int(device)
     c.accounting = int(accounting)
+    c.stir_steps = int(stir_steps)
     return c
+
+
+def stir_modes() -> np.ndarray:
+    """sph_stir_modes: the fixed driving mode set, int32 [61, 3] (host only)."""
+    n3 = np.zeros((STIR_NMODES, 3), np.int32)
+    m = load().sph_stir_modes(C.c_void_p(n3.ctypes.data), STIR_NMODES)
+    if m < 0:
+        raise SphError(-m, "sph_stir_modes")
+    return n3[:m]
 
 
 def _check(rc, ctx):
@@ -190,14 +210,14 @@ class Simulation:
     """One libsph context on one CUDA device (arena + stream owned by torch)."""
 
     def __init__(self, params, n_capacity: int, device: int = 0, accounting: int = ACCOUNTING_OFF,
-                 stream=None, max_cell_level: int = 8):
+                 stream=None, max_cell_level: int = 8, stir_steps: int = 0):
         import torch
         if not torch.cuda.is_available():
             raise RuntimeError("libsph needs a CUDA device (no CPU fallback)")
         self.L = load()
         self.torch = torch
         self.device = torch.device("cuda", device)
-        self.cfg = config_from_params(params, n_capacity, device, accounting, max_cell_level)
+        self.cfg = config_from_params(params, n_capacity, device, accounting, max_cell_level, stir_steps)
         nbytes = C.c_size_t(0)
         _check(self.L.sph_workspace_size(C.byref(self.cfg), C.byref(nbytes)), None)
         self.arena_bytes = int(nbytes.value)
@@ -388,3 +408,25 @@ class Simulation:
         m = min(int(n.value), capacity)
         a = np.ctypeslib.as_array(buf)[:m].copy()
         return a
+
+    # ---------------------------------------------------------------- driving
+    def stir_init(self, sigma: float, t_decay: float, sol_weight: float, w, noise, A0=None):
+        """sph_stir_init: weights w[61], noise[nsteps, 61, 6], optional A0[61, 6]."""
+        prm = StirParams(float(sigma), float(t_decay), float(sol_weight))
+        w = np.ascontiguousarray(w, np.float64)
+        noise = np.ascontiguousarray(noise, np.float64)
+        a0 = None if A0 is None else np.ascontiguousarray(A0, np.float64)
+        assert w.shape == (STIR_NMODES,) and noise.shape[1:] == (STIR_NMODES, 6)
+        self._ok(self.L.sph_stir_init(self.ctx, C.byref(prm), C.c_void_p(w.ctypes.data),
+                                      None if a0 is None else C.c_void_p(a0.ctypes.data),
+                                      C.c_void_p(noise.ctypes.data), noise.shape[0], MEM_HOST))
+
+    def stir(self):
+        self._ok(self.L.sph_stir(self.ctx))
+
+    def stir_state(self):
+        """(A[61, 6], number of STIR phases run)."""
+        A = np.zeros((STIR_NMODES, 6))
+        n = C.c_int64()
+        self._ok(self.L.sph_stir_get_state(self.ctx, C.c_void_p(A.ctypes.data), C.byref(n)))
+        return A, int(n.value)
