@@ -240,6 +240,8 @@ class DistributedSim:
         sim.iad()
         self._halo(["c11", "c12", "c13", "c22", "c23", "c33"], src_pos, dst_pos)
         sim.momentum_energy()
+        if sim.stir_enabled:  # driving: every rank holds the same OU state and noise
+            sim.stir()
         # 4. global dt, update, drop ghosts
         mhc = torch.tensor([sim.get_local_min_hc()], dtype=torch.float64, device=self.dev)
         mhc = comm.all_reduce(mhc, dist.ReduceOp.MIN if comm.world > 1 else None)

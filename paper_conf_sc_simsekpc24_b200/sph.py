@@ -229,6 +229,7 @@ class Simulation:
         _check(self.L.sph_init(C.byref(self.cfg), C.c_void_p(self._base), C.c_size_t(self.arena_bytes),
                                C.c_void_p(self.stream.cuda_stream), C.byref(self.ctx)), None)
         self.n = 0
+        self.stir_enabled = False
 
     # ---------------------------------------------------------------- lifetime
     def finalize(self):
@@ -420,6 +421,7 @@ class Simulation:
         self._ok(self.L.sph_stir_init(self.ctx, C.byref(prm), C.c_void_p(w.ctypes.data),
                                       None if a0 is None else C.c_void_p(a0.ctypes.data),
                                       C.c_void_p(noise.ctypes.data), noise.shape[0], MEM_HOST))
+        self.stir_enabled = True
 
     def stir(self):
         self._ok(self.L.sph_stir(self.ctx))
