@@ -42,25 +42,57 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
   return m;
 }
 
-// All 8 digit histograms in one read of the keys.
+// All 8 digit histograms in one read of the keys.  Each thread takes 8
+// consecutive keys.  The keys arrive nearly sorted (last step's order), so in
+// the high-digit passes a thread's 8 digits form one run and a warp's 256 keys
+// usually share the digit: runs are counted in registers and a warp whose
+// lanes all hold the same single-run digit adds once (warp reduction); the
+// low-digit passes (jitter bits, effectively random) add per run.
 __global__ void __launch_bounds__(kHistThreads) sort_hist_kernel(const uint64_t* __restrict__ keys,
                                                                  int64_t n, uint32_t* __restrict__ hist) {
   __shared__ uint32_t sh[kSortPasses][kRadix];
   for (int t = threadIdx.x; t < kSortPasses * kRadix; t += blockDim.x) (&sh[0][0])[t] = 0;
   __syncthreads();
-  const int lane = threadIdx.x & 31;
-  int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  // Whole warps iterate together so that match_any sees a full mask.
-  int64_t base = blockIdx.x * (int64_t)blockDim.x + (threadIdx.x & ~31);
-  for (; base < n; base += stride) {
-    int64_t i = base + lane;
-    bool valid = i < n;
-    uint64_t k = valid ? keys[i] : 0;
+  const int64_t nchunks = (n + 7) / 8;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  // whole warps iterate together (warp collectives below)
+  for (int64_t c0 = blockIdx.x * (int64_t)blockDim.x + (threadIdx.x & ~31); c0 < nchunks; c0 += stride) {
+    const int64_t c = c0 + (threadIdx.x & 31);
+    const int64_t i0 = c * 8;
+    const int cnt = c < nchunks ? (int)(n - i0 < 8 ? n - i0 : 8) : 0;
+    uint64_t k[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) k[j] = j < cnt ? keys[i0 + j] : 0ull;
 #pragma unroll
     for (int p = 0; p < kSortPasses; ++p) {
-      uint32_t d = valid ? (uint32_t)((k >> (p * kRadixBits)) & (kRadix - 1)) : 0x100u;
-      uint32_t peers = __match_any_sync(0xffffffffu, d);
-      if (valid && (peers & lanemask_lt()) == 0) atomicAdd(&sh[p][d], __popc(peers));
+      const int sh_bits = p * kRadixBits;
+      uint32_t prev = (uint32_t)((k[0] >> sh_bits) & (kRadix - 1));
+      bool single = true;
+#pragma unroll
+      for (int j = 1; j < 8; ++j)
+        if (j < cnt && (uint32_t)((k[j] >> sh_bits) & (kRadix - 1)) != prev) single = false;
+      const uint32_t d0 = __shfl_sync(0xffffffffu, prev, 0);
+      if (__all_sync(0xffffffffu, cnt == 0 || (single && prev == d0))) {
+        const uint32_t tot = __reduce_add_sync(0xffffffffu, (uint32_t)cnt);
+        if ((threadIdx.x & 31) == 0 && tot) atomicAdd(&sh[p][d0], tot);
+        continue;
+      }
+      if (cnt == 0) continue;
+      uint32_t run = 1;
+#pragma unroll
+      for (int j = 1; j < 8; ++j) {
+        if (j < cnt) {
+          const uint32_t d = (uint32_t)((k[j] >> sh_bits) & (kRadix - 1));
+          if (d == prev) {
+            ++run;
+          } else {
+            atomicAdd(&sh[p][prev], run);
+            prev = d;
+            run = 1;
+          }
+        }
+      }
+      atomicAdd(&sh[p][prev], run);
     }
   }
   __syncthreads();
@@ -217,7 +249,17 @@ cudaError_t launch_sort(const Fields& F, uint64_t* key_in, uint64_t* key_tmp, ui
   const int64_t tiles = div_up(n, kSortTile);
   cudaMemsetAsync(status, 0, sizeof(uint32_t) * (size_t)tiles * kRadix * kSortPasses, st);
   (void)status_bytes;
-  int hb = (int)std::min<int64_t>(div_up(n, kHistThreads), 148 * 8);
+  // Few CTAs: every CTA ends with one global atomic per nonzero bin (8 x 256),
+  // and with keys spread over the whole array every bin is nonzero, so the
+  // flush contends on 2048 L2 addresses: 2 CTAs per SM keep it ~0.6M atomics.
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    sms = std::max(sms, 1);
+  }
+  int hb = (int)std::min<int64_t>(div_up(div_up(n, 8), kHistThreads), 2 * sms);
   sort_hist_kernel<<<hb, kHistThreads, 0, st>>>(key_in, n, hist); note_launch();
   uint32_t* tile_ctr = hist + kSortPasses * kRadix;
   uint64_t* ks[2] = {key_in, key_tmp};
