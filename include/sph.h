@@ -326,6 +326,12 @@ int sph_step(sph_ctx* ctx, sph_step_info* info);
  * -> SPH_ERR_NO_PERMISSION / SPH_ERR_NOT_SUPPORTED leave the policy DEFAULT. */
 int sph_set_clock_policy(sph_ctx* ctx, int mode, const uint32_t mhz[SPH_NPHASES]);
 
+/* The SM (graphics) clocks the device supports at its highest memory clock,
+ * descending (NVML nvmlDeviceGetSupportedGraphicsClocks) -- the candidate set of
+ * the per-function frequency search (Fig. 2).  *n = count (<= cap).
+ * SPH_ERR_NVML when NVML is unavailable.  Does not change any clock. */
+int sph_supported_clocks(sph_ctx* ctx, uint32_t* mhz, int cap, int* n);
+
 /* One row per phase (cap >= SPH_NPHASES).  Time is always filled; joules only
  * with PHASE accounting and a working NVML energy counter. */
 int sph_energy_report(sph_ctx* ctx, sph_energy_row* rows, int cap, int* n_rows);

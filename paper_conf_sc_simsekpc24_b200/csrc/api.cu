@@ -1111,3 +1111,17 @@ int sph_stir_get_state(sph_ctx* c, double* A, int64_t* steps) {
   if (steps) *steps = (int64_t)c->h_ds.stir_step;
   return rc;
 }
+
+int sph_supported_clocks(sph_ctx* c, uint32_t* mhz, int cap, int* n) {
+  int rc = check_ready(c, S_INIT, "sph_supported_clocks");
+  if (rc) return rc;
+  if (!mhz || cap < 1 || !n) return fail(c, SPH_ERR_ARG, "bad output buffer");
+  if (!c->nvml.ok) return fail(c, SPH_ERR_NVML, "NVML unavailable: %s", c->nvml.err);
+  unsigned sup[512];
+  int ns = c->nvml.supported_sm_clocks(sup, 512);
+  if (ns <= 0) return fail(c, SPH_ERR_NVML, "no supported graphics clocks reported");
+  std::sort(sup, sup + ns, [](unsigned a, unsigned b) { return a > b; });
+  *n = std::min(ns, cap);
+  for (int k = 0; k < *n; ++k) mhz[k] = sup[k];
+  return SPH_OK;
+}

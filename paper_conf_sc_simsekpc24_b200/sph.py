@@ -89,7 +89,7 @@ EXPORTS = ("sph_config_default", "sph_workspace_size", "sph_init", "sph_finalize
            "sph_set_accounting", "sph_kernel_launches", "sph_set_field",
            "sph_get_local_min_hc", "sph_set_global_min_hc", "sph_get_neighbor_rows",
            "sph_trace_start", "sph_trace_stop", "sph_stir_modes", "sph_stir_init", "sph_stir",
-           "sph_stir_get_state")
+           "sph_stir_get_state", "sph_supported_clocks")
 GHOST_BIT = 1 << 62
 
 _lib = None
@@ -143,6 +143,7 @@ def load(build_if_missing: bool = True):
     L.sph_stir_init.argtypes = [P, C.POINTER(StirParams), V, V, V, I64, I]
     L.sph_stir.argtypes = [P]
     L.sph_stir_get_state.argtypes = [P, V, C.POINTER(I64)]
+    L.sph_supported_clocks.argtypes = [P, V, I, C.POINTER(I)]
     L.sph_trace_start.argtypes = [P, D, I64]
     L.sph_trace_stop.argtypes = [P, V, I64, C.POINTER(I64)]
     _lib = L
@@ -371,6 +372,13 @@ class Simulation:
     def set_clock_policy(self, mode: int, mhz=None):
         arr = (C.c_uint32 * NPHASES)(*([0] * NPHASES if mhz is None else [int(v) for v in mhz]))
         self._ok(self.L.sph_set_clock_policy(self.ctx, mode, arr))
+
+    def supported_clocks(self):
+        """sph_supported_clocks: SM clocks (MHz, descending) the device supports."""
+        buf = (C.c_uint32 * 512)()
+        n = C.c_int()
+        self._ok(self.L.sph_supported_clocks(self.ctx, C.cast(buf, C.c_void_p), 512, C.byref(n)))
+        return [int(buf[k]) for k in range(n.value)]
 
     def energy_report(self):
         rows = (EnergyRow * NPHASES)()
