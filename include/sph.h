@@ -109,6 +109,9 @@ typedef enum sph_field {
   SPH_F_RHO, SPH_F_P, SPH_F_C,
   SPH_F_C11, SPH_F_C12, SPH_F_C13, SPH_F_C22, SPH_F_C23, SPH_F_C33,
   SPH_F_AX, SPH_F_AY, SPH_F_AZ, SPH_F_DU,
+  SPH_F_DIVV,   /* velocity divergence (cfg.divcurl; valid after sph_iad)       */
+  SPH_F_CURLX, SPH_F_CURLY, SPH_F_CURLZ,  /* velocity curl (cfg.divcurl)        */
+  SPH_F_BAL,    /* Balsara switch factor (cfg.av_switch; valid after sph_iad)  */
   SPH_NFIELDS
 } sph_field;
 
@@ -137,7 +140,10 @@ typedef struct sph_config {
   int32_t rank, nranks;     /* reserved for SFC domain decomposition (1 rank now)  */
   int32_t stir_steps;       /* capacity (steps) of the driving-noise table; 0 = no
                                turbulence driving (sph_stir_init)                  */
-  int32_t reserved[15];
+  int32_t divcurl;          /* 1: IADVelocityDivCurl also computes div v, curl v
+                               (reading 19)                                        */
+  int32_t av_switch;        /* 1: Balsara switch on the AV (implies divcurl)       */
+  int32_t reserved[13];
 } sph_config;
 
 typedef struct sph_nbr_stats {
@@ -252,9 +258,10 @@ int sph_get_field(sph_ctx* ctx, int field, void* dst, int mem);
  * neighbourhood and are meaningless (the IAD singularity check ignores ghosts);
  * the owners' values are written over it with sph_set_field:
  *   after sph_density:  SPH_F_RHO           (then sph_eos derives p, c, V);
- *   after sph_iad:      SPH_F_C11..SPH_F_C33 (the momentum records are rebuilt).
- * sph_set_field copies n values (current order) from src; only SPH_F_RHO and
- * SPH_F_C11..SPH_F_C33 are settable (SPH_ERR_ARG otherwise). */
+ *   after sph_iad:      SPH_F_C11..SPH_F_C33 and, with cfg.av_switch, SPH_F_BAL
+ *                       (the momentum records are rebuilt).
+ * sph_set_field copies n values (current order) from src; only SPH_F_RHO,
+ * SPH_F_C11..SPH_F_C33 and SPH_F_BAL are settable (SPH_ERR_ARG otherwise). */
 #define SPH_GHOST_BIT (1ll << 62)
 int sph_set_field(sph_ctx* ctx, int field, const void* src, int mem);
 
@@ -295,9 +302,14 @@ int sph_density(sph_ctx* ctx);
  * p = c0^2 rho, c = c0.  EOS. */
 int sph_eos(sph_ctx* ctx);
 
-/* Item 7 (IADVelocityDivCurl, matrix part): tau_i = sum_j (m_j/rho_j) W(r,h_i)
- * Delta Delta^T, C_i = tau_i^{-1} (adjugate).  SPH_ERR_SINGULAR is reported at
- * the next synchronising call.  IAD. */
+/* Item 7 (IADVelocityDivCurl): tau_i = sum_j (m_j/rho_j) W(r,h_i)
+ * Delta Delta^T, C_i = tau_i^{-1} (adjugate).  With cfg.divcurl the same pass
+ * accumulates M_i = sum_j V_j W Delta (v_j - v_i)^T and forms the IAD velocity
+ * gradient T_i = C_i M_i (T_ab = dv_b/dx_a; exact for linear fields): div v =
+ * tr T, curl v = (T_yz - T_zy, T_zx - T_xz, T_xy - T_yx); with cfg.av_switch
+ * also the Balsara factor f_i = |div| / (|div| + |curl| + 1e-4 c_i/h_i) that
+ * scales the AV of a pair by (f_i + f_j)/2 in MOMENTUM_ENERGY (reading 19).
+ * SPH_ERR_SINGULAR is reported at the next synchronising call.  IAD. */
 int sph_iad(sph_ctx* ctx);
 
 /* Item 8 (MomentumEnergy): a_i, du_i with IAD gradients and Monaghan AV, plus

@@ -229,9 +229,38 @@ def iad(x, y, z, h, m, rho, bmin, bmax, periodic, nb: Neighbors, params):
     return Cm, tau, tabs, rc == 2
 
 
+def divcurl(x, y, z, vx, vy, vz, h, m, rho, Cm, bmin, bmax, periodic, nb: Neighbors, params):
+    """IAD velocity gradient T [n, 9] (T_ab = dv_b/dx_a), its scale T_abs, div v [n]
+    and curl v [n, 3] (oracle.c oracle_divcurl)."""
+    arrs = list(map(_d, (x, y, z, vx, vy, vz, h, m, rho)))
+    Cm = np.ascontiguousarray(Cm, dtype=np.float64)
+    per = np.ascontiguousarray(periodic, dtype=np.int32)
+    bmin, bmax = _d(bmin), _d(bmax)
+    n = arrs[0].size
+    T, Tabs, curl = np.zeros((n, 9)), np.zeros((n, 9)), np.zeros((n, 3))
+    dv = np.zeros(n)
+    ps = params_struct(params)
+    idx = nb.idx if nb.idx.size else np.zeros(1, dtype=np.int64)
+    lib().oracle_divcurl(C.c_int64(n), *[_p(a, _D) for a in arrs], _p(Cm, _D), _p(bmin, _D),
+                         _p(bmax, _D), _p(per, _I32), _p(nb.offsets, _I64), _p(idx, _I64),
+                         C.byref(ps), _p(T, _D), _p(Tabs, _D), _p(dv, _D), _p(curl, _D))
+    return T, Tabs, dv, curl
+
+
+def balsara(divv, curl, c, h):
+    """Balsara switch f = |div| / (|div| + |curl| + 1e-4 c/h)."""
+    divv, c, h = _d(divv), _d(c), _d(h)
+    curl = np.ascontiguousarray(curl, dtype=np.float64)
+    f = np.zeros(divv.size)
+    lib().oracle_balsara(C.c_int64(divv.size), _p(divv, _D), _p(curl, _D), _p(c, _D), _p(h, _D),
+                         _p(f, _D))
+    return f
+
+
 def momentum_energy(x, y, z, vx, vy, vz, h, m, rho, p, c, Cm, bmin, bmax, periodic,
-                    nb: Neighbors, params):
-    """Returns dict(ax, ay, az, du, a_abs [n,3], du_abs)."""
+                    nb: Neighbors, params, fav=None):
+    """Returns dict(ax, ay, az, du, a_abs [n,3], du_abs).  ``fav``: per-particle AV
+    switch factors (None = 1, the plain Monaghan viscosity)."""
     arrs = list(map(_d, (x, y, z, vx, vy, vz, h, m, rho, p, c)))
     Cm = np.ascontiguousarray(Cm, dtype=np.float64)
     per = np.ascontiguousarray(periodic, dtype=np.int32)
@@ -241,9 +270,11 @@ def momentum_energy(x, y, z, vx, vy, vz, h, m, rho, p, c, Cm, bmin, bmax, period
     aabs = np.zeros((n, 3))
     ps = params_struct(params)
     idx = nb.idx if nb.idx.size else np.zeros(1, dtype=np.int64)
+    fv = None if fav is None else _d(fav)
     lib().oracle_momentum_energy(C.c_int64(n), *[_p(a, _D) for a in arrs], _p(Cm, _D),
                                  _p(bmin, _D), _p(bmax, _D), _p(per, _I32), _p(nb.offsets, _I64),
-                                 _p(idx, _I64), C.byref(ps), _p(ax, _D), _p(ay, _D), _p(az, _D),
+                                 _p(idx, _I64), C.byref(ps), None if fv is None else _p(fv, _D),
+                                 _p(ax, _D), _p(ay, _D), _p(az, _D),
                                  _p(du, _D), _p(aabs, _D), _p(dabs, _D))
     return {"ax": ax, "ay": ay, "az": az, "du": du, "a_abs": aabs, "du_abs": dabs}
 
@@ -362,8 +393,19 @@ def step(state: dict, params, dt_prev: float, first_step: bool, ngmax: int | Non
                                   params.periodic, nb, params)
     if singular:
         raise ArithmeticError("IAD matrix singular")
+    dc = {}
+    fav = None
+    if getattr(params, "divcurl", 0) or getattr(params, "av_switch", 0):
+        T, Tabs, dvv, curl = divcurl(st["x"], st["y"], st["z"], st["vx"], st["vy"], st["vz"],
+                                     st["h"], st["m"], rho, Cm, bmin, bmax, params.periodic, nb,
+                                     params)
+        dc = {"T": T, "T_abs": Tabs, "divv": dvv, "curl": curl}
+        if getattr(params, "av_switch", 0):
+            fav = balsara(dvv, curl, c, st["h"])
+            dc["bal"] = fav
     acc = momentum_energy(st["x"], st["y"], st["z"], st["vx"], st["vy"], st["vz"], st["h"],
-                          st["m"], rho, p, c, Cm, bmin, bmax, params.periodic, nb, params)
+                          st["m"], rho, p, c, Cm, bmin, bmax, params.periodic, nb, params, fav)
+    acc.update(dc)
     if stir is not None:
         acc["stir_B"] = stir_apply(stir, st["x"], st["y"], st["z"], dt_prev, bmin, bmax, acc)
     dt = timestep(st["h"], c, dt_prev, params)

@@ -325,7 +325,8 @@ void oracle_momentum_energy(int64_t n, const double* x, const double* y, const d
                             const double* h, const double* m, const double* rho, const double* p,
                             const double* c, const double* C, const double bmin[3],
                             const double bmax[3], const int32_t per[3], const int64_t* off,
-                            const int64_t* idx, const oracle_params* P, double* ax, double* ay,
+                            const int64_t* idx, const oracle_params* P, const double* fav,
+                            double* ax, double* ay,
                             double* az, double* du, double* a_abs /* n x 3 */, double* du_abs) {
 #pragma omp parallel for schedule(dynamic, 64)
   for (int64_t i = 0; i < n; ++i) {
@@ -354,6 +355,7 @@ void oracle_momentum_energy(int64_t n, const double* x, const double* y, const d
       double cbar = (c[i] + c[j]) / 2.0;
       double rhobar = (rho[i] + rho[j]) / 2.0;
       double Pi = oracle_av_pi(rv, d2, hbar, cbar, rhobar, P);
+      if (fav) Pi = Pi * ((fav[i] + fav[j]) / 2.0);  /* AV switch (reading 19) */
       double prj = p[j] / (rho[j] * rho[j]);
       for (int a = 0; a < 3; ++a) {
         double t1 = pri * A[a], t2 = prj * B[a], t3 = Pi * G[a];
@@ -506,5 +508,62 @@ void oracle_stir_accel(int64_t n, const double* x, const double* y, const double
     ax[i] += s[0];
     ay[i] += s[1];
     az[i] += s[2];
+  }
+}
+
+/* ---------------------------------------------------------------------------
+ * Velocity divergence and curl of IADVelocityDivCurl (SURVEY 8(f)-1,
+ * DESIGN.md reading 19).  The IAD gradient of a field f at particle i is
+ *   (grad f)_i = sum_j V_j W(r_ij, h_i) (C_i Delta_ij) (f_j - f_i),
+ *   V_j = m_j / rho_j, Delta_ij = x_j - x_i (minimum image),
+ * exact for linear f (C_i = tau_i^-1).  Applied to the velocity it gives the
+ * tensor T_ab = d v_b / d x_a:
+ *   T_ab = sum_j V_j W(r_ij, h_i) (C_i Delta_ij)_a (v_j - v_i)_b,
+ *   div v = T_xx + T_yy + T_zz,
+ *   curl v = (T_yz - T_zy, T_zx - T_xz, T_xy - T_yx).
+ * T_abs holds sum_j |term_ab| (the tolerance scale).
+ * ------------------------------------------------------------------------- */
+void oracle_divcurl(int64_t n, const double* x, const double* y, const double* z,
+                    const double* vx, const double* vy, const double* vz, const double* h,
+                    const double* m, const double* rho, const double* C, const double bmin[3],
+                    const double bmax[3], const int32_t per[3], const int64_t* off,
+                    const int64_t* idx, const oracle_params* P, double* T /* n x 9 */,
+                    double* T_abs /* n x 9 */, double* divv, double* curl /* n x 3 */) {
+#pragma omp parallel for schedule(dynamic, 64)
+  for (int64_t i = 0; i < n; ++i) {
+    double t[9] = {0, 0, 0, 0, 0, 0, 0, 0, 0}, ta[9] = {0, 0, 0, 0, 0, 0, 0, 0, 0};
+    for (int64_t k = off[i]; k < off[i + 1]; ++k) {
+      int64_t j = idx[k];
+      double d[3];
+      double r = sqrt(pair_d(x, y, z, i, j, bmin, bmax, per, d));
+      double D[3] = {-d[0], -d[1], -d[2]};
+      double CD[3];
+      sym_mul(C + 6 * i, D, CD);
+      double vw = (m[j] / rho[j]) * oracle_W(r, h[i], P->K);
+      double dv[3] = {vx[j] - vx[i], vy[j] - vy[i], vz[j] - vz[i]};
+      for (int a = 0; a < 3; ++a)
+        for (int b = 0; b < 3; ++b) {
+          double term = vw * CD[a] * dv[b];
+          t[3 * a + b] += term;
+          ta[3 * a + b] += fabs(term);
+        }
+    }
+    for (int e = 0; e < 9; ++e) { T[9 * i + e] = t[e]; T_abs[9 * i + e] = ta[e]; }
+    divv[i] = t[0] + t[4] + t[8];
+    curl[3 * i + 0] = t[5] - t[7];  /* dv_z/dy - dv_y/dz */
+    curl[3 * i + 1] = t[6] - t[2];  /* dv_x/dz - dv_z/dx */
+    curl[3 * i + 2] = t[1] - t[3];  /* dv_y/dx - dv_x/dy */
+  }
+}
+
+/* Balsara (1995) switch: f_i = |div v| / (|div v| + |curl v| + 1e-4 c_i / h_i);
+ * the artificial viscosity of a pair is multiplied by (f_i + f_j) / 2. */
+void oracle_balsara(int64_t n, const double* divv, const double* curl, const double* c,
+                    const double* h, double* f) {
+  for (int64_t i = 0; i < n; ++i) {
+    double ad = fabs(divv[i]);
+    double ac = sqrt(curl[3 * i] * curl[3 * i] + curl[3 * i + 1] * curl[3 * i + 1] +
+                     curl[3 * i + 2] * curl[3 * i + 2]);
+    f[i] = ad / (ad + ac + 1e-4 * c[i] / h[i]);
   }
 }

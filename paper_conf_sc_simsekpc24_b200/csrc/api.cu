@@ -62,6 +62,8 @@ struct sph_ctx {
   uint64_t *keyA, *keyB, *key_sorted;
   uint32_t *valA, *valB;
   double *rho, *p, *c, *vol, *prho2, *wq, *wk, *C[6], *ax, *ay, *az, *du;
+  double *divv, *curl[3], *bal;
+  Rec4* rec_iv = nullptr;
   int32_t *nc, *nbr, *nrows;
   uint32_t* cell_start;
   float4* pos4;
@@ -142,6 +144,8 @@ Fields fields(sph_ctx* c) {
   F.wq = c->wq; F.wk = c->wk;
   for (int e = 0; e < 6; ++e) F.C[e] = c->C[e];
   F.ax = c->ax; F.ay = c->ay; F.az = c->az; F.du = c->du;
+  F.divv = c->divv; F.bal = c->P.av_switch ? c->bal : nullptr; F.rec_iv = c->rec_iv;
+  for (int a = 0; a < 3; ++a) F.curl[a] = c->curl[a];
   F.nc = c->nc; F.nbr = c->nbr; F.ngmax = c->cfg.ngmax;
   F.nrows = c->nrows; F.nrows_ld = nrows_ld(&c->cfg);
   F.cell_start = c->cell_start;
@@ -393,6 +397,8 @@ static int validate(const sph_config* c) {
   if (!(c->K > 0) || !(c->dt_first > 0) || !(c->h_cap > 0)) return fail(nullptr, SPH_ERR_ARG, "K, dt_first and h_cap must be > 0");
   if (c->nranks != 1) return fail(nullptr, SPH_ERR_NOT_SUPPORTED, "nranks > 1 is not built into this library version");
   if (c->stir_steps < 0) return fail(nullptr, SPH_ERR_ARG, "stir_steps < 0");
+  if (c->divcurl < 0 || c->divcurl > 1 || c->av_switch < 0 || c->av_switch > 1)
+    return fail(nullptr, SPH_ERR_ARG, "divcurl and av_switch must be 0 or 1");
   return SPH_OK;
 }
 
@@ -421,7 +427,9 @@ static size_t layout(const sph_config* cfg, char* base, sph_ctx* c) {
   double** dst[] = {c ? &c->rho : nullptr, c ? &c->p : nullptr, c ? &c->c : nullptr,
                     c ? &c->vol : nullptr, c ? &c->prho2 : nullptr, c ? &c->wq : nullptr,
                     c ? &c->wk : nullptr, c ? &c->ax : nullptr, c ? &c->ay : nullptr,
-                    c ? &c->az : nullptr, c ? &c->du : nullptr};
+                    c ? &c->az : nullptr, c ? &c->du : nullptr, c ? &c->divv : nullptr,
+                    c ? &c->curl[0] : nullptr, c ? &c->curl[1] : nullptr,
+                    c ? &c->curl[2] : nullptr, c ? &c->bal : nullptr};
   for (double** d : dst) {
     char* p = take(D);
     if (c) *d = (double*)p;
@@ -434,6 +442,8 @@ static size_t layout(const sph_config* cfg, char* base, sph_ctx* c) {
   char* rd = take(sizeof(Rec4) * cap);
   char* ri = take(sizeof(Rec4) * cap);
   char* rm = take(sizeof(Rec4) * kRecM * cap);
+  char* riv = (cfg->divcurl || cfg->av_switch) ? take(sizeof(Rec4) * cap) : nullptr;
+  if (c) c->rec_iv = (Rec4*)riv;
   if (c) {
     c->pos4 = (float4*)p4;
     c->rec_d = (Rec4*)rd;
@@ -509,6 +519,8 @@ int sph_init(const sph_config* cfg, void* arena, size_t arena_bytes, void* strea
   c->P.ng0 = cfg->ng0; c->P.h_cap = cfg->h_cap; c->P.k_cour = cfg->k_cour;
   c->P.dt_max_growth = cfg->dt_max_growth; c->P.av_alpha = cfg->av_alpha;
   c->P.av_beta = cfg->av_beta; c->P.av_eps = cfg->av_eps; c->P.max_cell_level = cfg->max_cell_level;
+  c->P.av_switch = cfg->av_switch ? 1 : 0;
+  c->P.divcurl = (cfg->divcurl || cfg->av_switch) ? 1 : 0;
   layout(cfg, (char*)arena, c);
   for (int p = 0; p < SPH_NPHASES; ++p) {
     c->pending[p] = false;
@@ -633,6 +645,9 @@ int sph_get_field(sph_ctx* c, int field, void* dst, int mem) {
   else if (field == SPH_F_AY) src = c->ay;
   else if (field == SPH_F_AZ) src = c->az;
   else if (field == SPH_F_DU) src = c->du;
+  else if (field == SPH_F_DIVV) src = c->divv;
+  else if (field >= SPH_F_CURLX && field <= SPH_F_CURLZ) src = c->curl[field - SPH_F_CURLX];
+  else if (field == SPH_F_BAL) src = c->bal;
   else return fail(c, SPH_ERR_ARG, "unknown field %d", field);
   if (c->n == 0) return SPH_OK;
   const cudaMemcpyKind kind = mem == SPH_MEM_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
@@ -655,6 +670,10 @@ int sph_set_field(sph_ctx* c, int field, const void* src, int mem) {
   } else if (field >= SPH_F_C11 && field <= SPH_F_C33) {
     if (c->stage < S_IAD) return fail(c, SPH_ERR_STATE, "sph_set_field(C) before sph_iad");
     dst = c->C[field - SPH_F_C11];
+    c->rec_m_dirty = true;
+  } else if (field == SPH_F_BAL && c->P.av_switch) {
+    if (c->stage < S_IAD) return fail(c, SPH_ERR_STATE, "sph_set_field(BAL) before sph_iad");
+    dst = c->bal;
     c->rec_m_dirty = true;
   } else {
     return fail(c, SPH_ERR_ARG, "field %d is not settable", field);

@@ -158,6 +158,7 @@ __global__ void __launch_bounds__(256) eos_kernel(Fields F, Params P) {
   F.vol[i] = V;
   F.prho2[i] = __ddiv_rn(p, __dmul_rn(rho, rho));
   st4(F.rec_i + i, rd.a, rd.b, rd.c, V);
+  if (P.divcurl) st4(F.rec_iv + i, F.f[FVX][i], F.f[FVY][i], F.f[FVZ][i], 0.0);
 }
 
 // ------------------------------------------------------------------ IAD
@@ -222,7 +223,103 @@ __device__ __forceinline__ void iad_body(const Fields& F, const Geom& g, int64_t
   st4(rm + 1, c11, c12, c13, kh3);
   st4(rm + 2, c22, c23, c33, F.f[FM][i]);
   st4(rm + 3, F.f[FVX][i], F.f[FVY][i], F.f[FVZ][i], F.prho2[i]);
-  st4(rm + 4, F.f[FH][i], F.c[i], F.rho[i], 0.0);
+  st4(rm + 4, F.f[FH][i], F.c[i], F.rho[i], 1.0);  // AV switch factor 1 (no switch)
+}
+
+// IADVelocityDivCurl with the velocity part (cfg.divcurl, reading 19): the same
+// list walk also accumulates M = sum_j V_j W Delta (v_j - v_i)^T (9 sums; one
+// more 32-B record {vx, vy, vz, 0} per pair), then T = C M (T_ab = dv_b/dx_a),
+// div v = tr T, curl v from the antisymmetric part, and the Balsara factor.
+template <bool kWrap>
+__device__ __forceinline__ void iad_dc_body(const Fields& F, const Params& P, const Geom& g, int64_t i,
+                                            const Rec4& me) {
+  const double q = F.wq[i], kh3 = F.wk[i];
+  const int nci = min(F.nc[i], F.ngmax);
+  const double vxi = F.f[FVX][i], vyi = F.f[FVY][i], vzi = F.f[FVZ][i];
+  double t11 = 0, t12 = 0, t13 = 0, t22 = 0, t23 = 0, t33 = 0;
+  double M[3][3] = {{0, 0, 0}, {0, 0, 0}, {0, 0, 0}};
+  const int32_t* __restrict__ nb = F.nbr + i;
+  const Rec4* __restrict__ rec = F.rec_i;
+  const Rec4* __restrict__ rv = F.rec_iv;
+  const int64_t cap = F.cap;
+  int jn = nci > 0 ? __ldg(nb) : 0;
+  Rec4 ra = ldg4(rec + jn), va = ldg4(rv + jn);
+  jn = nci > 1 ? __ldg(nb + cap) : 0;
+  for (int k = 0; k < nci; ++k) {
+    const Rec4 rj = ra, vj = va;
+    if (k + 1 < nci) {
+      ra = ldg4(rec + jn);
+      va = ldg4(rv + jn);
+    }
+    if (k + 2 < nci) jn = __ldg(nb + (int64_t)(k + 2) * cap);
+    double dx, dy, dz;
+    pair_d<kWrap>(g, me.a, me.b, me.c, rj.a, rj.b, rj.c, dx, dy, dz);
+    const double r2 = dx * dx + dy * dy + dz * dz;
+    const double vw = rj.d * (kh3 * sinc6_t(r2 * q));
+    const double ax = vw * dx, ay = vw * dy, az = vw * dz;
+    t11 = fma(ax, dx, t11);
+    t12 = fma(ax, dy, t12);
+    t13 = fma(ax, dz, t13);
+    t22 = fma(ay, dy, t22);
+    t23 = fma(ay, dz, t23);
+    t33 = fma(az, dz, t33);
+    // M_ab += V W Delta_a dv_b with Delta = -d
+    const double dv[3] = {vj.a - vxi, vj.b - vyi, vj.c - vzi};
+    const double aw[3] = {ax, ay, az};
+#pragma unroll
+    for (int a = 0; a < 3; ++a)
+#pragma unroll
+      for (int b = 0; b < 3; ++b) M[a][b] = fma(-aw[a], dv[b], M[a][b]);
+  }
+  const double det = t11 * (t22 * t33 - t23 * t23) - t12 * (t12 * t33 - t23 * t13) +
+                     t13 * (t12 * t23 - t22 * t13);
+  const double inv = 1.0 / det;
+  const double c11 = (t22 * t33 - t23 * t23) * inv, c12 = (t13 * t23 - t12 * t33) * inv;
+  const double c13 = (t12 * t23 - t13 * t22) * inv, c22 = (t11 * t33 - t13 * t13) * inv;
+  const double c23 = (t12 * t13 - t11 * t23) * inv, c33 = (t11 * t22 - t12 * t12) * inv;
+  F.C[0][i] = c11;
+  F.C[1][i] = c12;
+  F.C[2][i] = c13;
+  F.C[3][i] = c22;
+  F.C[4][i] = c23;
+  F.C[5][i] = c33;
+  if ((!(det > 0.0) || !isfinite(det)) && !(F.id[i] & SPH_GHOST_BIT))
+    atomicOr(&F.ds->status, (int)ST_SINGULAR);
+  const double Cm[3][3] = {{c11, c12, c13}, {c12, c22, c23}, {c13, c23, c33}};
+  double T[3][3];
+#pragma unroll
+  for (int a = 0; a < 3; ++a)
+#pragma unroll
+    for (int b = 0; b < 3; ++b) T[a][b] = Cm[a][0] * M[0][b] + Cm[a][1] * M[1][b] + Cm[a][2] * M[2][b];
+  const double div = T[0][0] + T[1][1] + T[2][2];
+  const double cx = T[1][2] - T[2][1], cy = T[2][0] - T[0][2], cz = T[0][1] - T[1][0];
+  F.divv[i] = div;
+  F.curl[0][i] = cx;
+  F.curl[1][i] = cy;
+  F.curl[2][i] = cz;
+  double f = 1.0;
+  if (P.av_switch) {
+    const double ad = fabs(div), ac = sqrt(cx * cx + cy * cy + cz * cz);
+    f = ad / (ad + ac + 1e-4 * F.c[i] / F.f[FH][i]);
+    F.bal[i] = f;
+  }
+  Rec4* rm = F.rec_m + (int64_t)kRecM * i;
+  st4(rm + 0, me.a, me.b, me.c, q);
+  st4(rm + 1, c11, c12, c13, kh3);
+  st4(rm + 2, c22, c23, c33, F.f[FM][i]);
+  st4(rm + 3, vxi, vyi, vzi, F.prho2[i]);
+  st4(rm + 4, F.f[FH][i], F.c[i], F.rho[i], f);
+}
+
+__global__ void __launch_bounds__(512, 1) iad_dc_kernel(Fields F, Params P) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= F.n) return;
+  const Geom g = load_geom(F.ds, P);
+  const Rec4 me = F.rec_i[i];
+  if (__any_sync(__activemask(), needs_wrap(g, me.a, me.b, me.c, F.f[FH][i])))
+    iad_dc_body<true>(F, P, g, i, me);
+  else
+    iad_dc_body<false>(F, P, g, i, me);
 }
 
 __global__ void __launch_bounds__(kIadThreads, 768 / kIadThreads) iad_kernel(Fields F, Params P) {
@@ -253,7 +350,7 @@ __device__ __forceinline__ void momentum_body(const Fields& F, const Params& P, 
   const double ci11 = i1.a, ci12 = i1.b, ci13 = i1.c, khi = i1.d;
   const double ci22 = i2.a, ci23 = i2.b, ci33 = i2.c;
   const double vxi = i3.a, vyi = i3.b, vzi = i3.c, pri = i3.d;
-  const double hi = i4.a, ci = i4.b, rhoi = i4.c;
+  const double hi = i4.a, ci = i4.b, rhoi = i4.c, fi = i4.d;
   const double alpha = P.av_alpha, beta = P.av_beta, eps = P.av_eps;
   const int nci = min(F.nc[i], F.ngmax);
   double ax = 0, ay = 0, az = 0, de = 0;
@@ -311,6 +408,7 @@ __device__ __forceinline__ void momentum_body(const Fields& F, const Params& P, 
       const double q = 1.0 / (D * rhobar);
       const double mu = hbar * rv * (rhobar * q);
       Pi = (fma(beta, mu, -alpha * cbar) * mu) * (D * q);
+      if (P.av_switch) Pi *= 0.5 * (fi + j4.d);  // Balsara switch (reading 19)
     }
     const double mj = j2.d, prj = j3.d;
     const double ka = (pri + 0.5 * Pi) * wi, kb = (prj + 0.5 * Pi) * wj;
@@ -404,6 +502,7 @@ __global__ void __launch_bounds__(256) refresh_rec_m_kernel(Fields F) {
   Rec4* rm = F.rec_m + (int64_t)kRecM * i;
   st4(rm + 1, F.C[0][i], F.C[1][i], F.C[2][i], F.wk[i]);
   st4(rm + 2, F.C[3][i], F.C[4][i], F.C[5][i], F.f[FM][i]);
+  if (F.bal) rm[4].d = F.bal[i];  // owners' Balsara factors over the ghosts (av_switch)
 }
 
 void launch_refresh_rec_m(const Fields& F, cudaStream_t st) {
@@ -425,7 +524,10 @@ void launch_eos(const Fields& F, const Params& P, cudaStream_t st) {
 }
 void launch_iad(const Fields& F, const Params& P, cudaStream_t st) {
   if (F.n == 0) return;
-  iad_kernel<<<(unsigned)div_up(F.n, kIadThreads), kIadThreads, 0, st>>>(F, P);
+  if (P.divcurl)
+    iad_dc_kernel<<<(unsigned)div_up(F.n, 512), 512, 0, st>>>(F, P);
+  else
+    iad_kernel<<<(unsigned)div_up(F.n, kIadThreads), kIadThreads, 0, st>>>(F, P);
   note_launch();
 }
 void launch_momentum_energy(const Fields& F, const Params& P, cudaStream_t st) {

@@ -100,6 +100,8 @@ struct Fields {
   double *wq, *wk;        // per-particle kernel factors (pi/2h)^2 and K/h^3
   double* C[6];           // 11 12 13 22 23 33
   double *ax, *ay, *az, *du;
+  double *divv, *curl[3], *bal;  // IADVelocityDivCurl extras (cfg.divcurl / av_switch)
+  Rec4* rec_iv;           // {vx, vy, vz, 0} gather record of the div/curl sums (EOS)
   int32_t* nc;
   int32_t* nbr;           // [ngmax][cap] column-major: neighbour k of target i at nbr[k * cap + i]
   int32_t* nrows;         // neighbour-search scratch: row-major rows of the resident warps
@@ -120,6 +122,7 @@ struct Params {
   double gamma, cs0, K, ng0, h_cap, k_cour, dt_max_growth;
   double av_alpha, av_beta, av_eps;
   int max_cell_level;
+  int divcurl, av_switch;
 };
 
 // Process-wide count of libsph kernel launches (sph_kernel_launches).

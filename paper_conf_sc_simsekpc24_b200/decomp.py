@@ -238,7 +238,11 @@ class DistributedSim:
         self._halo(["rho"], src_pos, dst_pos)
         sim.eos()
         sim.iad()
-        self._halo(["c11", "c12", "c13", "c22", "c23", "c33"], src_pos, dst_pos)
+        # H3: the owners' C (and Balsara factors when the AV switch is on)
+        h3 = ["c11", "c12", "c13", "c22", "c23", "c33"]
+        if getattr(self.params, "av_switch", 0):
+            h3.append("bal")
+        self._halo(h3, src_pos, dst_pos)
         sim.momentum_energy()
         if sim.stir_enabled:  # driving: every rank holds the same OU state and noise
             sim.stir()

@@ -53,6 +53,8 @@ class StepParams:
     av_beta: float = 2.0
     av_eps: float = 0.01
     h_cap: float = 0.25
+    divcurl: int = 0        # 1: IADVelocityDivCurl also computes div v, curl v
+    av_switch: int = 0      # 1: Balsara switch on the AV (implies divcurl)
 
     def as_dict(self):
         return asdict(self)

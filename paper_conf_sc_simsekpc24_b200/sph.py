@@ -25,7 +25,8 @@ PHASES = ("keys", "sort", "cells", "neighbors", "density", "eos", "iad", "moment
 STIR_NMODES = 61
 NPHASES = len(PHASES)
 FIELDS = ("x", "y", "z", "vx", "vy", "vz", "h", "m", "u", "du_m1", "id", "key", "nc", "rho", "p",
-          "c", "c11", "c12", "c13", "c22", "c23", "c33", "ax", "ay", "az", "du")
+          "c", "c11", "c12", "c13", "c22", "c23", "c33", "ax", "ay", "az", "du", "divv", "curlx",
+          "curly", "curlz", "bal")
 FIELD_ID = {name: k for k, name in enumerate(FIELDS)}
 FIELD_DTYPE = {"id": np.int64, "key": np.uint64, "nc": np.int32}
 MEM_HOST, MEM_DEVICE = 0, 1
@@ -49,7 +50,8 @@ class Config(C.Structure):
         ("dt_max_growth", C.c_double), ("dt_first", C.c_double), ("av_alpha", C.c_double),
         ("av_beta", C.c_double), ("av_eps", C.c_double), ("device", C.c_int32),
         ("accounting", C.c_int32), ("rank", C.c_int32), ("nranks", C.c_int32),
-        ("stir_steps", C.c_int32), ("reserved", C.c_int32 * 15),
+        ("stir_steps", C.c_int32), ("divcurl", C.c_int32), ("av_switch", C.c_int32),
+        ("reserved", C.c_int32 * 13),
     ]
 
 
@@ -176,6 +178,8 @@ def config_from_params(params, n_capacity: int, device: int = 0, accounting: int
     c.device = int(device)
     c.accounting = int(accounting)
     c.stir_steps = int(stir_steps)
+    c.divcurl = int(getattr(params, "divcurl", 0))
+    c.av_switch = int(getattr(params, "av_switch", 0))
     return c
 
 

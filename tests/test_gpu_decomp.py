@@ -26,9 +26,16 @@ def _free_port():
     return p
 
 
+def _sedov_balsara():
+    import dataclasses
+    w = ics.sedov(14)
+    w.params = dataclasses.replace(w.params, av_switch=1)  # halo of the Balsara factors too
+    return w
+
+
 def _make(name):
     return {"turbulence16": lambda: ics.turbulence(16), "random": lambda: ics.random_box(6000, seed=5),
-            "sedov14": lambda: ics.sedov(14)}[name]()
+            "sedov14": lambda: ics.sedov(14), "sedov14_balsara": _sedov_balsara}[name]()
 
 
 def _worker(rank, world, port, name, q):
@@ -62,7 +69,7 @@ def _single(name):
     return dts, {k: v[o] for k, v in st.items()}
 
 
-@pytest.mark.parametrize("name", ["turbulence16", "random", "sedov14"])
+@pytest.mark.parametrize("name", ["turbulence16", "random", "sedov14", "sedov14_balsara"])
 def test_two_ranks_bit_identical_to_one(name):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
