@@ -57,6 +57,8 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--energy-steps", type=int, default=60,
                     help="steps for the whole-step energy (>= ~2 s: the counter ticks every ~100 ms)")
+    ap.add_argument("--av-switch", action="store_true",
+                    help="IADVelocityDivCurl div/curl + Balsara AV switch (SURVEY 8(f)-1)")
     ap.add_argument("--stir", action="store_true",
                     help="turbulence driving (OU stirring, SURVEY 8(f)-3) inside every step")
     ap.add_argument("--trace-seconds", type=float, default=1.5,
@@ -376,6 +378,9 @@ def main():
     torch.cuda.set_device(local)
     w = make_workload(args.workload, rank)
     n = w.n
+    if args.av_switch:
+        import dataclasses
+        w.params = dataclasses.replace(w.params, av_switch=1)
     stir_steps = 8192 if args.stir else 0
     sim = sph.Simulation(w.params, n_capacity=n, device=local, stir_steps=stir_steps)
     stream = sim.stream
@@ -484,7 +489,8 @@ def main():
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-                "config": {"workload": args.workload + ("+stir" if args.stir else ""),
+                "config": {"workload": args.workload + ("+stir" if args.stir else "")
+                           + ("+balsara" if args.av_switch else ""),
                            "n_particles_per_gpu": n,
                            "n_particles_total": n * world,
                            "parallelism": "single GPU" if world == 1 else
