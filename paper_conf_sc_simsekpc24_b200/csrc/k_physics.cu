@@ -341,7 +341,7 @@ __global__ void __launch_bounds__(kIadThreads, 768 / kIadThreads) iad_kernel(Fie
 // order-preserving bit pattern of a positive double).
 // Per pair: 4 records (128 B) + 1 more (AV) for approaching pairs, 157 DP flops
 // (+ 17 and 2 divisions when approaching).
-template <bool kWrap>
+template <bool kWrap, bool kSwitch>
 __device__ __forceinline__ void momentum_body(const Fields& F, const Params& P, const Geom& g, int64_t i) {
   const Rec4* __restrict__ rec = F.rec_m;
   const Rec4* mi = rec + (int64_t)kRecM * i;
@@ -408,7 +408,7 @@ __device__ __forceinline__ void momentum_body(const Fields& F, const Params& P, 
       const double q = 1.0 / (D * rhobar);
       const double mu = hbar * rv * (rhobar * q);
       Pi = (fma(beta, mu, -alpha * cbar) * mu) * (D * q);
-      if (P.av_switch) Pi *= 0.5 * (fi + j4.d);  // Balsara switch (reading 19)
+      if (kSwitch) Pi *= 0.5 * (fi + j4.d);  // Balsara switch (reading 19)
     }
     const double mj = j2.d, prj = j3.d;
     const double ka = (pri + 0.5 * Pi) * wi, kb = (prj + 0.5 * Pi) * wj;
@@ -433,10 +433,14 @@ __global__ void __launch_bounds__(kMomThreads, 512 / kMomThreads) momentum_energ
     const Geom g = load_geom(F.ds, P);
     const Rec4* mi = F.rec_m + (int64_t)kRecM * i;
     const Rec4 i0 = mi[0], i4 = mi[4];
-    if (__any_sync(__activemask(), needs_wrap(g, i0.a, i0.b, i0.c, i4.a)))
-      momentum_body<true>(F, P, g, i);
-    else
-      momentum_body<false>(F, P, g, i);
+    const bool wrap = __any_sync(__activemask(), needs_wrap(g, i0.a, i0.b, i0.c, i4.a));
+    if (P.av_switch) {
+      if (wrap) momentum_body<true, true>(F, P, g, i);
+      else momentum_body<false, true>(F, P, g, i);
+    } else {
+      if (wrap) momentum_body<true, false>(F, P, g, i);
+      else momentum_body<false, false>(F, P, g, i);
+    }
     hc = ord_of(__ddiv_rn(i4.a, i4.b));
   }
 #pragma unroll
