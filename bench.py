@@ -84,6 +84,8 @@ def make_workload(name: str, rank: int):
         return ics.sedov(int(name[len("sedov"):]))
     if name.startswith("noh"):
         return ics.noh(int(name[len("noh"):]))
+    if name.startswith("evrard"):   # with self-gravity (Barnes-Hut, theta 0.5)
+        return ics.evrard(int(name[len("evrard"):]))
     raise SystemExit(f"unknown workload {name}")
 
 

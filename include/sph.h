@@ -90,7 +90,9 @@ typedef enum sph_phase {
   SPH_PHASE_UPDATE = 9,          /* positions, velocities, energy, h (item 10)    */
   SPH_PHASE_STIR = 10,           /* turbulence driving; runs after
                                     MOMENTUM_ENERGY, before TIMESTEP, when enabled */
-  SPH_NPHASES = 11
+  SPH_PHASE_GRAVITY = 11,        /* self-gravity; runs after
+                                    MOMENTUM_ENERGY when cfg.gravity              */
+  SPH_NPHASES = 12
 } sph_phase;
 
 typedef enum sph_clock_mode {
@@ -112,6 +114,7 @@ typedef enum sph_field {
   SPH_F_DIVV,   /* velocity divergence (cfg.divcurl; valid after sph_iad)       */
   SPH_F_CURLX, SPH_F_CURLY, SPH_F_CURLZ,  /* velocity curl (cfg.divcurl)        */
   SPH_F_BAL,    /* Balsara switch factor (cfg.av_switch; valid after sph_iad)  */
+  SPH_F_PHI,    /* gravitational potential (cfg.gravity; after sph_gravity)    */
   SPH_NFIELDS
 } sph_field;
 
@@ -143,7 +146,13 @@ typedef struct sph_config {
   int32_t divcurl;          /* 1: IADVelocityDivCurl also computes div v, curl v
                                (reading 19)                                        */
   int32_t av_switch;        /* 1: Balsara switch on the AV (implies divcurl)       */
-  int32_t reserved[13];
+  int32_t gravity;          /* 1: self-gravity phase (open boxes only)             */
+  int32_t grav_level;       /* leaf level Lt of the gravity octree, 1..8           */
+  double grav_G;            /* gravitational constant                              */
+  double grav_eps;          /* Plummer softening length                            */
+  double grav_theta;        /* opening angle: multipole when side < theta * dist;
+                               0 = direct summation                               */
+  int32_t reserved[8];
 } sph_config;
 
 typedef struct sph_nbr_stats {
@@ -161,6 +170,9 @@ typedef struct sph_step_info {
   int32_t cell_level;       /* cell-grid level used by the neighbour search        */
   int32_t reserved;
   double phase_ms[SPH_NPHASES]; /* CUDA-event time of each phase in this step      */
+  int64_t grav_multipoles;  /* diagnostic: multipoles evaluated per warp, summed    */
+  int64_t grav_pairs;       /* diagnostic: direct pairs per warp (32 targets), sum */
+  int64_t grav_pops;        /* diagnostic: tree nodes opened per warp, summed      */
 } sph_step_info;
 
 typedef struct sph_energy_row {
@@ -369,6 +381,19 @@ int sph_kernel_launches(int64_t* count);
  * so reps should make the call last >= 1 s.  Synchronises. */
 int sph_repeat_phase(sph_ctx* ctx, int phase, int reps, double* ms_per_call,
                      double* joules_per_call);
+
+/* --- self-gravity ------------------------------------------ */
+
+/* Phase GRAVITY (the Evrard collapse's extra function; reading
+ * 20): a_i += G sum_j m_j (x_j - x_i) / (|x_j - x_i|^2 + eps^2)^(3/2) and the
+ * potential phi_i, by a Barnes-Hut walk of the Morton octree (levels 0..Lt,
+ * monopole + traceless quadrupole per cell, a cell is used as a multipole when
+ * its side < theta * distance from the 32 targets' box to its centre of mass;
+ * leaves not accepted are summed directly).  theta = 0 is exact direct
+ * summation in ascending particle order.  Needs cfg.gravity (arena room for the
+ * octree) and a fully open box; after sph_momentum_energy.  Runs inside sph_step
+ * when enabled. */
+int sph_gravity(sph_ctx* ctx);
 
 /* --- turbulence driving ------------------------------------ */
 

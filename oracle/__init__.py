@@ -371,6 +371,18 @@ def stir_apply(stir: dict, x, y, z, dt_prev: float, bmin, bmax, acc: dict):
     return B
 
 
+def gravity(x, y, z, m, G: float, eps: float):
+    """Direct-sum softened gravity: dict(ax, ay, az, phi, a_abs [n, 3])."""
+    x, y, z, m = map(_d, (x, y, z, m))
+    n = x.size
+    ax, ay, az, phi = (np.zeros(n) for _ in range(4))
+    aabs = np.zeros((n, 3))
+    lib().oracle_gravity(C.c_int64(n), _p(x, _D), _p(y, _D), _p(z, _D), _p(m, _D), C.c_double(G),
+                         C.c_double(eps), _p(ax, _D), _p(ay, _D), _p(az, _D), _p(phi, _D),
+                         _p(aabs, _D))
+    return {"ax": ax, "ay": ay, "az": az, "phi": phi, "a_abs": aabs}
+
+
 def step(state: dict, params, dt_prev: float, first_step: bool, ngmax: int | None = None,
          stir: dict | None = None):
     """One full oracle step.  Returns (new_state, out) where new_state is in this
@@ -406,6 +418,12 @@ def step(state: dict, params, dt_prev: float, first_step: bool, ngmax: int | Non
     acc = momentum_energy(st["x"], st["y"], st["z"], st["vx"], st["vy"], st["vz"], st["h"],
                           st["m"], rho, p, c, Cm, bmin, bmax, params.periodic, nb, params, fav)
     acc.update(dc)
+    if getattr(params, "gravity", 0):
+        gr = gravity(st["x"], st["y"], st["z"], st["m"], params.grav_G, params.grav_eps)
+        for k in ("ax", "ay", "az"):
+            acc[k] = acc[k] + gr[k]
+        acc["a_abs"] = acc["a_abs"] + gr["a_abs"]
+        acc["phi"] = gr["phi"]
     if stir is not None:
         acc["stir_B"] = stir_apply(stir, st["x"], st["y"], st["z"], dt_prev, bmin, bmax, acc)
     dt = timestep(st["h"], c, dt_prev, params)

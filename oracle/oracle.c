@@ -567,3 +567,38 @@ void oracle_balsara(int64_t n, const double* divv, const double* curl, const dou
     f[i] = ad / (ad + ac + 1e-4 * c[i] / h[i]);
   }
 }
+
+/* ---------------------------------------------------------------------------
+ * Self-gravity (the Evrard collapse workload, P:108, P:135;
+ * DESIGN.md reading 20).  Newtonian attraction with Plummer softening eps,
+ * isolated (open) boundaries, by direct summation over j != i in ascending
+ * order -- the definition the GPU tree code approximates:
+ *   a_i   = G sum_j m_j (x_j - x_i) / (|x_j - x_i|^2 + eps^2)^(3/2),
+ *   phi_i = -G sum_j m_j / (|x_j - x_i|^2 + eps^2)^(1/2).
+ * a_abs[3i+a] = sum_j |term_a| (the tolerance scale).
+ * ------------------------------------------------------------------------- */
+void oracle_gravity(int64_t n, const double* x, const double* y, const double* z,
+                    const double* m, double G, double eps, double* ax, double* ay, double* az,
+                    double* phi, double* a_abs) {
+#pragma omp parallel for schedule(dynamic, 16)
+  for (int64_t i = 0; i < n; ++i) {
+    double a[3] = {0, 0, 0}, aa[3] = {0, 0, 0}, p = 0.0;
+    for (int64_t j = 0; j < n; ++j) {
+      if (j == i) continue;
+      double d[3] = {x[j] - x[i], y[j] - y[i], z[j] - z[i]};
+      double r2 = d[0] * d[0] + d[1] * d[1] + d[2] * d[2] + eps * eps;
+      double r = sqrt(r2);
+      double s = G * m[j] / (r2 * r);
+      for (int c = 0; c < 3; ++c) {
+        a[c] += s * d[c];
+        aa[c] += fabs(s * d[c]);
+      }
+      p -= G * m[j] / r;
+    }
+    ax[i] = a[0];
+    ay[i] = a[1];
+    az[i] = a[2];
+    phi[i] = p;
+    for (int c = 0; c < 3; ++c) a_abs[3 * i + c] = aa[c];
+  }
+}

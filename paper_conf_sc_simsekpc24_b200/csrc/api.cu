@@ -25,7 +25,7 @@ enum Stage { S_INIT = 0, S_PART, S_TREE, S_NBR, S_DENS, S_EOS, S_IAD, S_MOM, S_D
 
 const char* kPhaseNames[SPH_NPHASES] = {"keys",    "sort",    "cells", "neighbors",
                                         "density", "eos",     "iad",   "momentum_energy",
-                                        "timestep", "update",  "stir"};
+                                        "timestep", "update",  "stir", "gravity"};
 
 thread_local char g_err[512] = "";
 
@@ -64,6 +64,9 @@ struct sph_ctx {
   double *rho, *p, *c, *vol, *prho2, *wq, *wk, *C[6], *ax, *ay, *az, *du;
   double *divv, *curl[3], *bal;
   Rec4* rec_iv = nullptr;
+  double* phi = nullptr;
+  uint32_t* gcell_start = nullptr;
+  Rec4* gmom = nullptr;
   int32_t *nc, *nbr, *nrows;
   uint32_t* cell_start;
   float4* pos4;
@@ -145,6 +148,7 @@ Fields fields(sph_ctx* c) {
   for (int e = 0; e < 6; ++e) F.C[e] = c->C[e];
   F.ax = c->ax; F.ay = c->ay; F.az = c->az; F.du = c->du;
   F.divv = c->divv; F.bal = c->P.av_switch ? c->bal : nullptr; F.rec_iv = c->rec_iv;
+  F.phi = c->phi; F.gcell_start = c->gcell_start; F.gmom = c->gmom;
   for (int a = 0; a < 3; ++a) F.curl[a] = c->curl[a];
   F.nc = c->nc; F.nbr = c->nbr; F.ngmax = c->cfg.ngmax;
   F.nrows = c->nrows; F.nrows_ld = nrows_ld(&c->cfg);
@@ -343,6 +347,11 @@ int body_simple(sph_ctx* c, int phase, int next_stage) {
       launch_advance_time(F, c->st);
       break;
     case SPH_PHASE_STIR: launch_stir(F, c->P, c->stir, c->st); break;
+    case SPH_PHASE_GRAVITY: {
+      GravParams G{c->cfg.grav_G, c->cfg.grav_eps, c->cfg.grav_theta, c->cfg.grav_level};
+      launch_gravity(F, G, c->st);
+      break;
+    }
   }
   if ((rc = phase_end(c, phase))) return rc;
   c->stage = next_stage;
@@ -382,6 +391,10 @@ int sph_config_default(sph_config* cfg) {
   cfg->accounting = SPH_ACCOUNTING_OFF;
   cfg->rank = 0;
   cfg->nranks = 1;
+  cfg->grav_level = 6;
+  cfg->grav_G = 1.0;
+  cfg->grav_eps = 0.01;
+  cfg->grav_theta = 0.5;
   return SPH_OK;
 }
 
@@ -399,6 +412,13 @@ static int validate(const sph_config* c) {
   if (c->stir_steps < 0) return fail(nullptr, SPH_ERR_ARG, "stir_steps < 0");
   if (c->divcurl < 0 || c->divcurl > 1 || c->av_switch < 0 || c->av_switch > 1)
     return fail(nullptr, SPH_ERR_ARG, "divcurl and av_switch must be 0 or 1");
+  if (c->gravity) {
+    if (c->periodic[0] || c->periodic[1] || c->periodic[2])
+      return fail(nullptr, SPH_ERR_NOT_SUPPORTED, "gravity is for isolated (fully open) boxes");
+    if (c->grav_level < 1 || c->grav_level > 8) return fail(nullptr, SPH_ERR_ARG, "grav_level must be in [1, 8]");
+    if (!(c->grav_eps >= 0) || !(c->grav_theta >= 0) || !(c->grav_G >= 0))
+      return fail(nullptr, SPH_ERR_ARG, "grav_G, grav_eps, grav_theta must be >= 0");
+  }
   return SPH_OK;
 }
 
@@ -444,6 +464,18 @@ static size_t layout(const sph_config* cfg, char* base, sph_ctx* c) {
   char* rm = take(sizeof(Rec4) * kRecM * cap);
   char* riv = (cfg->divcurl || cfg->av_switch) ? take(sizeof(Rec4) * cap) : nullptr;
   if (c) c->rec_iv = (Rec4*)riv;
+  if (cfg->gravity) {
+    const int Lt = cfg->grav_level;
+    const size_t ncells = (size_t)((((int64_t)1 << (3 * (Lt + 1))) - 1) / 7);
+    char* ph = take(D);
+    char* gcs = take(sizeof(uint32_t) * (((size_t)1 << (3 * Lt)) + 1));
+    char* gm = take(sizeof(Rec4) * 3 * ncells);
+    if (c) {
+      c->phi = (double*)ph;
+      c->gcell_start = (uint32_t*)gcs;
+      c->gmom = (Rec4*)gm;
+    }
+  }
   if (c) {
     c->pos4 = (float4*)p4;
     c->rec_d = (Rec4*)rd;
@@ -648,6 +680,10 @@ int sph_get_field(sph_ctx* c, int field, void* dst, int mem) {
   else if (field == SPH_F_DIVV) src = c->divv;
   else if (field >= SPH_F_CURLX && field <= SPH_F_CURLZ) src = c->curl[field - SPH_F_CURLX];
   else if (field == SPH_F_BAL) src = c->bal;
+  else if (field == SPH_F_PHI) {
+    if (!c->phi) return fail(c, SPH_ERR_ARG, "SPH_F_PHI needs cfg.gravity");
+    src = c->phi;
+  }
   else return fail(c, SPH_ERR_ARG, "unknown field %d", field);
   if (c->n == 0) return SPH_OK;
   const cudaMemcpyKind kind = mem == SPH_MEM_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
@@ -829,6 +865,7 @@ int sph_step(sph_ctx* c, sph_step_info* info) {
   if ((rc = body_simple(c, SPH_PHASE_EOS, S_EOS))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_IAD, S_IAD))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_MOMENTUM_ENERGY, S_MOM))) return rc;
+  if (c->cfg.gravity && (rc = body_simple(c, SPH_PHASE_GRAVITY, S_MOM))) return rc;
   if (c->stir_on && (rc = body_simple(c, SPH_PHASE_STIR, S_MOM))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_TIMESTEP, S_DT))) return rc;
   // A data error (capacity, singular, box) makes the update meaningless: check
@@ -841,6 +878,9 @@ int sph_step(sph_ctx* c, sph_step_info* info) {
     fill_stats(c, &info->nbr);
     info->cell_level = c->h_ds.cell_level;
     for (int p = 0; p < SPH_NPHASES; ++p) info->phase_ms[p] = c->last_ms[p];
+    info->grav_multipoles = (int64_t)c->h_ds.grav_mp;
+    info->grav_pairs = (int64_t)c->h_ds.grav_pp;
+    info->grav_pops = (int64_t)c->h_ds.grav_pops;
   }
   return rc;
 }
@@ -1143,4 +1183,11 @@ int sph_supported_clocks(sph_ctx* c, uint32_t* mhz, int cap, int* n) {
   *n = std::min(ns, cap);
   for (int k = 0; k < *n; ++k) mhz[k] = sup[k];
   return SPH_OK;
+}
+
+int sph_gravity(sph_ctx* c) {
+  int rc = check_ready(c, S_MOM, "sph_gravity");
+  if (rc) return rc;
+  if (!c->cfg.gravity) return fail(c, SPH_ERR_STATE, "gravity not enabled (cfg.gravity = 0)");
+  return body_simple(c, SPH_PHASE_GRAVITY, S_MOM);
 }

@@ -1,0 +1,310 @@
+// k_gravity.cu -- phase GRAVITY: self-gravity by a Barnes-Hut octree with
+// quadrupole moments on the Morton cells (the Evrard collapse
+// workload of P:108; definitions in include/sph.h, reading 20).
+//
+// The tree is the Morton grid itself: the particles are already sorted by key,
+// so a cell at level l is the key prefix key >> 3(21-l) and its particles are a
+// contiguous range.  Dense levels 0..Lt (Lt = cfg.grav_level):
+//  1. grav_cells_kernel   leaf ranges at level Lt (like the neighbour grid);
+//  2. grav_leaf_kernel    per leaf: mass, centre of mass, traceless quadrupole
+//                         Q_ab = sum m (3 d_a d_b - d^2 delta_ab) about the COM;
+//  3. grav_up_kernel      per level, parents from their 8 children (parallel-axis
+//                         shift of each child's quadrupole to the parent's COM);
+//  4. grav_walk_kernel    one warp per 32 consecutive (Morton-adjacent) targets
+//                         walks the tree depth first with a shared-memory stack:
+//                         a cell is accepted as a multipole when side < theta *
+//                         distance(target box, COM) (one warp-uniform decision for
+//                         the 32 targets, no divergence), opened otherwise; leaves
+//                         that are not accepted are summed directly with the
+//                         Plummer-softened pair force.  Children are pushed in
+//                         reverse so leaves are visited in ascending particle
+//                         order: with theta = 0 the walk is the direct sum of the
+//                         oracle, in the oracle's order.
+// Bound: FP64 (direct pairs ~20 DP ops, multipoles ~45); the moments are
+// HBM-light (96 B per cell).
+#include <algorithm>
+
+#include "sph_internal.cuh"
+
+namespace sph {
+
+__host__ __device__ inline int64_t grav_level_off(int l) { return ((int64_t(1) << (3 * l)) - 1) / 7; }
+
+__global__ void __launch_bounds__(256) grav_cells_kernel(int64_t n, const uint64_t* __restrict__ key, int Lt,
+                                                         uint32_t* __restrict__ cs) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const int shift = 3 * (21 - Lt);
+  const int64_t ncell = int64_t(1) << (3 * Lt);
+  const int64_t ck = (int64_t)(key[i] >> shift);
+  const int64_t prev = i > 0 ? (int64_t)(key[i - 1] >> shift) : -1;
+  for (int64_t c = prev + 1; c <= ck; ++c) cs[c] = (uint32_t)i;
+  if (i == n - 1)
+    for (int64_t c = ck + 1; c <= ncell; ++c) cs[c] = (uint32_t)n;
+}
+
+__device__ __forceinline__ void store_mom(Rec4* g, int64_t cell, double m, const double c[3], const double q[6]) {
+  st4(g + 3 * cell + 0, m, c[0], c[1], c[2]);
+  st4(g + 3 * cell + 1, q[0], q[1], q[2], q[3]);
+  st4(g + 3 * cell + 2, q[4], q[5], 0.0, 0.0);
+}
+
+__global__ void __launch_bounds__(256) grav_leaf_kernel(Fields F, int Lt) {
+  const int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (c >= (int64_t(1) << (3 * Lt))) return;
+  const uint32_t s = F.gcell_start[c], e = F.gcell_start[c + 1];
+  double m = 0, com[3] = {0, 0, 0}, q[6] = {0, 0, 0, 0, 0, 0};
+  for (uint32_t j = s; j < e; ++j) {
+    const Rec4 r = ldg4(F.rec_d + j);
+    m += r.d;
+    com[0] = fma(r.d, r.a, com[0]);
+    com[1] = fma(r.d, r.b, com[1]);
+    com[2] = fma(r.d, r.c, com[2]);
+  }
+  if (m > 0) {
+    for (int a = 0; a < 3; ++a) com[a] /= m;
+    for (uint32_t j = s; j < e; ++j) {
+      const Rec4 r = ldg4(F.rec_d + j);
+      const double d[3] = {r.a - com[0], r.b - com[1], r.c - com[2]};
+      const double d2 = d[0] * d[0] + d[1] * d[1] + d[2] * d[2];
+      q[0] += r.d * (3 * d[0] * d[0] - d2);
+      q[1] += r.d * (3 * d[0] * d[1]);
+      q[2] += r.d * (3 * d[0] * d[2]);
+      q[3] += r.d * (3 * d[1] * d[1] - d2);
+      q[4] += r.d * (3 * d[1] * d[2]);
+      q[5] += r.d * (3 * d[2] * d[2] - d2);
+    }
+  }
+  store_mom(F.gmom, grav_level_off(Lt) + c, m, com, q);
+}
+
+__global__ void __launch_bounds__(256) grav_up_kernel(Fields F, int l) {
+  const int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (c >= (int64_t(1) << (3 * l))) return;
+  const int64_t ch0 = grav_level_off(l + 1) + 8 * c;
+  double m = 0, com[3] = {0, 0, 0}, q[6] = {0, 0, 0, 0, 0, 0};
+  Rec4 k0[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+    k0[k] = ldg4(F.gmom + 3 * (ch0 + k));
+    m += k0[k].a;
+    com[0] = fma(k0[k].a, k0[k].b, com[0]);
+    com[1] = fma(k0[k].a, k0[k].c, com[1]);
+    com[2] = fma(k0[k].a, k0[k].d, com[2]);
+  }
+  if (m > 0) {
+    for (int a = 0; a < 3; ++a) com[a] /= m;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      if (k0[k].a == 0.0) continue;
+      const Rec4 k1 = ldg4(F.gmom + 3 * (ch0 + k) + 1), k2 = ldg4(F.gmom + 3 * (ch0 + k) + 2);
+      const double d[3] = {k0[k].b - com[0], k0[k].c - com[1], k0[k].d - com[2]};
+      const double d2 = d[0] * d[0] + d[1] * d[1] + d[2] * d[2], mk = k0[k].a;
+      q[0] += k1.a + mk * (3 * d[0] * d[0] - d2);
+      q[1] += k1.b + mk * (3 * d[0] * d[1]);
+      q[2] += k1.c + mk * (3 * d[0] * d[2]);
+      q[3] += k1.d + mk * (3 * d[1] * d[1] - d2);
+      q[4] += k2.a + mk * (3 * d[1] * d[2]);
+      q[5] += k2.b + mk * (3 * d[2] * d[2] - d2);
+    }
+  }
+  store_mom(F.gmom, grav_level_off(l) + c, m, com, q);
+}
+
+constexpr int kGravThreads = 128;
+constexpr int kGravWarps = kGravThreads / 32;
+constexpr int kGravStack = 64;
+
+struct GravSmem {
+  uint32_t stack[kGravStack];   // parents whose 8 children are still to examine
+  double mom[8][10];            // the accepted children's moments (m, com, Q)
+  double px[32], py[32], pz[32], pm[32];  // a batch of leaf particles
+};
+
+// Multipole (monopole + traceless quadrupole, unsoftened) of cell moments q at
+// target offset r = x_i - com.
+__device__ __forceinline__ void add_multipole(const double* q, double xi, double yi, double zi, double Gc,
+                                              double& ax, double& ay, double& az, double& phi) {
+  const double rx = xi - q[1], ry = yi - q[2], rz = zi - q[3];
+  const double r2 = rx * rx + ry * ry + rz * rz;
+  const double ir = rsqrt(r2), ir2 = ir * ir, ir3 = ir * ir2, ir5 = ir3 * ir2;
+  const double Qx = q[4] * rx + q[5] * ry + q[6] * rz;
+  const double Qy = q[5] * rx + q[7] * ry + q[8] * rz;
+  const double Qz = q[6] * rx + q[8] * ry + q[9] * rz;
+  const double rQr = rx * Qx + ry * Qy + rz * Qz;
+  const double mono = -Gc * q[0] * ir3;
+  const double quad = -2.5 * Gc * rQr * ir5 * ir2;
+  ax += mono * rx + Gc * Qx * ir5 + quad * rx;
+  ay += mono * ry + Gc * Qy * ir5 + quad * ry;
+  az += mono * rz + Gc * Qz * ir5 + quad * rz;
+  phi += -Gc * q[0] * ir - 0.5 * Gc * rQr * ir5;
+}
+
+// One warp per 32 consecutive targets.  The stack holds parents; popping one
+// examines its 8 children together (lanes 0-7 load and classify one child each:
+// one memory round trip per 8 cells instead of 8 dependent ones): accepted
+// children are evaluated as multipoles from shared memory, leaf children are
+// summed directly in batches of 32 particles staged in shared memory (one load
+// per lane), the other children are pushed (in reverse: ascending pop order).
+// With theta = 0 every child of a level-(Lt-1) node is a leaf and no other node
+// has leaf children, so the direct sums run over ascending particle indices.
+__global__ void __launch_bounds__(kGravThreads) grav_walk_kernel(Fields F, GravParams G) {
+  __shared__ GravSmem s_w[kGravWarps];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  GravSmem& S = s_w[warp];
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  const bool active = i < F.n;
+  if (!__any_sync(0xffffffffu, active)) return;
+  const int64_t ii = active ? i : F.n - 1;
+  const double xi = F.f[FX][ii], yi = F.f[FY][ii], zi = F.f[FZ][ii];
+  double lo[3] = {xi, yi, zi}, hi[3] = {xi, yi, zi};
+#pragma unroll
+  for (int a = 0; a < 3; ++a)
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) {
+      lo[a] = fmin(lo[a], __shfl_xor_sync(0xffffffffu, lo[a], off));
+      hi[a] = fmax(hi[a], __shfl_xor_sync(0xffffffffu, hi[a], off));
+    }
+  const DevScalars* ds = F.ds;
+  const double Lmax = fmax(ds->box_max[0] - ds->box_min[0],
+                           fmax(ds->box_max[1] - ds->box_min[1], ds->box_max[2] - ds->box_min[2]));
+  const double th2 = G.theta * G.theta, eps2 = G.eps * G.eps, Gc = G.G;
+  const int Lt = G.level;
+  double ax = 0, ay = 0, az = 0, phi = 0;
+  unsigned long long n_mp = 0, n_pp = 0, n_pop = 0;  // diagnostics (warp-uniform)
+
+  // the root itself: accepted, a leaf (Lt = 0 is not allowed) or opened
+  int sp = 0;
+  {
+    const Rec4 m0 = ldg4(F.gmom);
+    if (m0.a == 0.0) goto done;
+    double dd2 = 0;
+    const double cc[3] = {m0.b, m0.c, m0.d};
+#pragma unroll
+    for (int a = 0; a < 3; ++a) {
+      const double t = fmax(fmax(lo[a] - cc[a], cc[a] - hi[a]), 0.0);
+      dd2 += t * t;
+    }
+    if (Lmax * Lmax < th2 * dd2) {
+      const Rec4 m1 = ldg4(F.gmom + 1), m2 = ldg4(F.gmom + 2);
+      const double q[10] = {m0.a, m0.b, m0.c, m0.d, m1.a, m1.b, m1.c, m1.d, m2.a, m2.b};
+      add_multipole(q, xi, yi, zi, Gc, ax, ay, az, phi);
+      goto done;
+    }
+    if (lane == 0) S.stack[0] = 0u;  // open the root
+    sp = 1;
+    __syncwarp();
+  }
+  while (sp > 0) {
+    const uint32_t e = S.stack[sp - 1];
+    __syncwarp();
+    --sp;
+    ++n_pop;
+    const int l = (int)(e >> 28) + 1;                 // the children's level
+    const int64_t c0 = 8 * (int64_t)(e & 0x0fffffffu);  // first child's index at level l
+    const int64_t g0 = grav_level_off(l) + c0;
+    // lanes 0-7: child k = lane
+    bool acc = false, open = false, leaf = false;
+    if (lane < 8) {
+      const Rec4 m0 = ldg4(F.gmom + 3 * (g0 + lane));
+      if (m0.a != 0.0) {
+        const double side = Lmax / (double)(1 << l);
+        double dd2 = 0;
+        const double cc[3] = {m0.b, m0.c, m0.d};
+#pragma unroll
+        for (int a = 0; a < 3; ++a) {
+          const double t = fmax(fmax(lo[a] - cc[a], cc[a] - hi[a]), 0.0);
+          dd2 += t * t;
+        }
+        if (side * side < th2 * dd2) {
+          acc = true;
+          const Rec4 m1 = ldg4(F.gmom + 3 * (g0 + lane) + 1), m2 = ldg4(F.gmom + 3 * (g0 + lane) + 2);
+          double* q = S.mom[lane];
+          q[0] = m0.a; q[1] = m0.b; q[2] = m0.c; q[3] = m0.d;
+          q[4] = m1.a; q[5] = m1.b; q[6] = m1.c; q[7] = m1.d; q[8] = m2.a; q[9] = m2.b;
+        } else if (l == Lt) {
+          leaf = true;
+        } else {
+          open = true;
+        }
+      }
+    }
+    const uint32_t am = __ballot_sync(0xffffffffu, acc);
+    const uint32_t lm = __ballot_sync(0xffffffffu, leaf);
+    const uint32_t om = __ballot_sync(0xffffffffu, open);
+    __syncwarp();
+    // multipoles
+    n_mp += __popc(am);
+    for (uint32_t m = am; m; m &= m - 1) {
+      const int k = __ffs(m) - 1;
+      add_multipole(S.mom[k], xi, yi, zi, Gc, ax, ay, az, phi);
+    }
+    // leaves, ascending: particles in batches of 32 through shared memory
+    for (uint32_t m = lm; m; m &= m - 1) {
+      const int k = __ffs(m) - 1;
+      const int64_t c = c0 + k;
+      const uint32_t s = F.gcell_start[c], en = F.gcell_start[c + 1];
+      for (uint32_t b = s; b < en; b += 32) {
+        const uint32_t nb = min(32u, en - b);
+        n_pp += nb;
+        __syncwarp();
+        if ((uint32_t)lane < nb) {
+          const Rec4 r = ldg4(F.rec_d + b + lane);
+          S.px[lane] = r.a;
+          S.py[lane] = r.b;
+          S.pz[lane] = r.c;
+          S.pm[lane] = r.d;
+        }
+        __syncwarp();
+        for (uint32_t t = 0; t < nb; ++t) {
+          if ((int64_t)(b + t) == ii) continue;
+          const double dx = S.px[t] - xi, dy = S.py[t] - yi, dz = S.pz[t] - zi;
+          const double r2 = dx * dx + dy * dy + dz * dz + eps2;
+          const double ir = rsqrt(r2);
+          const double s3 = Gc * S.pm[t] * ir * ir * ir;
+          ax = fma(s3, dx, ax);
+          ay = fma(s3, dy, ay);
+          az = fma(s3, dz, az);
+          phi -= Gc * S.pm[t] * ir;
+        }
+      }
+    }
+    // opened children: push in reverse so they pop in ascending order
+    const int no = __popc(om);
+    if (lane < 8 && open) {
+      const int rank_from_top = __popc(om & ((1u << lane) - 1u));  // 0 for the lowest child
+      S.stack[sp + no - 1 - rank_from_top] = ((uint32_t)l << 28) | (uint32_t)(c0 + lane);
+    }
+    sp += no;
+    __syncwarp();
+  }
+done:
+  if (lane == 0) {
+    atomicAdd(&F.ds->grav_mp, n_mp);
+    atomicAdd(&F.ds->grav_pp, n_pp);
+    atomicAdd(&F.ds->grav_pops, n_pop);
+  }
+  if (active) {
+    F.ax[i] += ax;
+    F.ay[i] += ay;
+    F.az[i] += az;
+    F.phi[i] = phi;
+  }
+}
+
+void launch_gravity(const Fields& F, const GravParams& G, cudaStream_t st) {
+  if (F.n == 0) return;
+  cudaMemsetAsync(&F.ds->grav_mp, 0, 3 * sizeof(unsigned long long), st);
+  const int Lt = G.level;
+  grav_cells_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F.n, F.key, Lt, F.gcell_start);
+  grav_leaf_kernel<<<(unsigned)div_up(int64_t(1) << (3 * Lt), 256), 256, 0, st>>>(F, Lt);
+  note_launch(2);
+  for (int l = Lt - 1; l >= 0; --l) {
+    grav_up_kernel<<<(unsigned)div_up(int64_t(1) << (3 * l), 256), 256, 0, st>>>(F, l);
+    note_launch();
+  }
+  grav_walk_kernel<<<(unsigned)div_up(F.n, kGravThreads), kGravThreads, 0, st>>>(F, G);
+  note_launch();
+}
+
+}  // namespace sph

@@ -48,6 +48,13 @@ struct DevScalars {
   int pad;
   unsigned long long nbr_next;    // neighbour search: next 32-target tile (dynamic schedule)
   unsigned long long stir_step;   // STIR phases run since sph_stir_init
+  unsigned long long grav_mp, grav_pp, grav_pops;  // gravity walk diagnostics (per warp sums)
+};
+
+// Self-gravity (k_gravity.cu).
+struct GravParams {
+  double G, eps, theta;
+  int level;
 };
 
 // Turbulence driving (k_stir.cu): the OU state and its inputs, in the arena.
@@ -102,6 +109,9 @@ struct Fields {
   double *ax, *ay, *az, *du;
   double *divv, *curl[3], *bal;  // IADVelocityDivCurl extras (cfg.divcurl / av_switch)
   Rec4* rec_iv;           // {vx, vy, vz, 0} gather record of the div/curl sums (EOS)
+  double* phi;            // gravitational potential (GRAVITY)
+  uint32_t* gcell_start;  // gravity octree: leaf ranges at level grav_level
+  Rec4* gmom;             // gravity octree moments, 3 records per cell, levels 0..Lt
   int32_t* nc;
   int32_t* nbr;           // [ngmax][cap] column-major: neighbour k of target i at nbr[k * cap + i]
   int32_t* nrows;         // neighbour-search scratch: row-major rows of the resident warps
@@ -236,5 +246,6 @@ void launch_update(const Fields& F, const Params& P, cudaStream_t st);
 void launch_advance_time(const Fields& F, cudaStream_t st);
 void launch_refresh_rec_m(const Fields& F, cudaStream_t st);
 void launch_stir(const Fields& F, const Params& P, const Stir& S, cudaStream_t st);
+void launch_gravity(const Fields& F, const GravParams& G, cudaStream_t st);
 int stir_modes(int32_t* n3);  // host: the fixed mode set (returns kStirModes)
 }  // namespace sph

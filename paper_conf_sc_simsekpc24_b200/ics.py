@@ -55,6 +55,11 @@ class StepParams:
     h_cap: float = 0.25
     divcurl: int = 0        # 1: IADVelocityDivCurl also computes div v, curl v
     av_switch: int = 0      # 1: Balsara switch on the AV (implies divcurl)
+    gravity: int = 0        # 1: self-gravity (GRAVITY phase, open boxes)
+    grav_G: float = 1.0
+    grav_eps: float = 0.01  # Plummer softening length
+    grav_theta: float = 0.5  # tree opening angle (0 = direct summation)
+    grav_level: int = 6     # leaf level of the gravity octree
 
     def as_dict(self):
         return asdict(self)
@@ -119,6 +124,36 @@ def noh(nside: int, u0: float = 1e-20) -> Workload:
     p = StepParams(periodic=(0, 0, 0), eos=0, gamma=5.0 / 3.0, dt_first=1e-4, h_cap=1e300)
     st = _state(x, y, z, -x * inv, -y * inv, -z * inv, h_initial(n, p.ng0), 1.0 / n, np.full(n, u0))
     return Workload(f"noh{nside}", st, p, {"nside": nside, "lattice_a": a})
+
+
+def evrard(nside: int, radius: float = 1.0, mass: float = 1.0, u_frac: float = 0.05,
+           eps: float = 0.01) -> Workload:
+    """Evrard collapse (the paper's gravity workload):
+    a gas sphere of radius R and mass M with rho = M / (2 pi R^2 r), at rest,
+    u = 0.05 G M / R, gamma 5/3, open box.  Particles: the lattice points of the
+    unit sphere (nside per diameter), stretched radially r = R r_u^(3/2) so that
+    M(<r) = M (r/R)^2; h from the local density (ng0 neighbours)."""
+    x, y, z, a = _lattice(nside)
+    x, y, z = 2 * x, 2 * y, 2 * z                       # lattice on [-1, 1]^3
+    ru = np.sqrt(x * x + y * y + z * z)
+    keep = ru < 1.0
+    x, y, z, ru = x[keep], y[keep], z[keep], ru[keep]
+    s = radius * np.sqrt(ru)                            # r / r_u = R r_u^(1/2)
+    x, y, z = x * s, y * s, z * s
+    r = ru * s
+    n = x.size
+    m = mass / n
+    rho = mass / (2.0 * math.pi * radius ** 2 * np.maximum(r, 1e-3 * radius))
+    # octree leaf level: ~4 particles per leaf on average (measured best, DESIGN.md)
+    level = int(min(8, max(3, round(math.log(max(n, 8) / 4.0, 8)))))
+    p = StepParams(box_min=(-1.0, -1.0, -1.0), box_max=(1.0, 1.0, 1.0), periodic=(0, 0, 0), eos=0,
+                   gamma=5.0 / 3.0, dt_first=1e-4, h_cap=1e300, gravity=1, grav_eps=eps,
+                   grav_level=level)
+    h = 0.5 * (3.0 * p.ng0 * m / (4.0 * math.pi * rho)) ** (1.0 / 3.0)
+    u = np.full(n, u_frac * p.grav_G * mass / radius)
+    zeros = np.zeros(n)
+    st = _state(x, y, z, zeros.copy(), zeros.copy(), zeros.copy(), h, m, u)
+    return Workload(f"evrard{nside}", st, p, {"nside": nside, "n": n})
 
 
 def _solenoidal_modes(seed: int, nmax: float = 3.0):

@@ -21,12 +21,12 @@ STATUS = {0: "OK", 1: "ERR_ARG", 2: "ERR_STATE", 3: "ERR_CUDA", 4: "ERR_NCCL", 5
           6: "ERR_NO_PERMISSION", 7: "ERR_NOT_SUPPORTED", 8: "ERR_CAPACITY", 9: "ERR_HCAP",
           10: "ERR_SINGULAR", 11: "ERR_BOX"}
 PHASES = ("keys", "sort", "cells", "neighbors", "density", "eos", "iad", "momentum_energy",
-          "timestep", "update", "stir")
+          "timestep", "update", "stir", "gravity")
 STIR_NMODES = 61
 NPHASES = len(PHASES)
 FIELDS = ("x", "y", "z", "vx", "vy", "vz", "h", "m", "u", "du_m1", "id", "key", "nc", "rho", "p",
           "c", "c11", "c12", "c13", "c22", "c23", "c33", "ax", "ay", "az", "du", "divv", "curlx",
-          "curly", "curlz", "bal")
+          "curly", "curlz", "bal", "phi")
 FIELD_ID = {name: k for k, name in enumerate(FIELDS)}
 FIELD_DTYPE = {"id": np.int64, "key": np.uint64, "nc": np.int32}
 MEM_HOST, MEM_DEVICE = 0, 1
@@ -51,7 +51,8 @@ class Config(C.Structure):
         ("av_beta", C.c_double), ("av_eps", C.c_double), ("device", C.c_int32),
         ("accounting", C.c_int32), ("rank", C.c_int32), ("nranks", C.c_int32),
         ("stir_steps", C.c_int32), ("divcurl", C.c_int32), ("av_switch", C.c_int32),
-        ("reserved", C.c_int32 * 13),
+        ("gravity", C.c_int32), ("grav_level", C.c_int32), ("grav_G", C.c_double),
+        ("grav_eps", C.c_double), ("grav_theta", C.c_double), ("reserved", C.c_int32 * 8),
     ]
 
 
@@ -63,7 +64,8 @@ class NbrStats(C.Structure):
 class StepInfo(C.Structure):
     _fields_ = [("t", C.c_double), ("dt", C.c_double), ("nbr", NbrStats),
                 ("cell_level", C.c_int32), ("reserved", C.c_int32),
-                ("phase_ms", C.c_double * NPHASES)]
+                ("phase_ms", C.c_double * NPHASES), ("grav_multipoles", C.c_int64),
+                ("grav_pairs", C.c_int64), ("grav_pops", C.c_int64)]
 
 
 class EnergyRow(C.Structure):
@@ -91,7 +93,7 @@ EXPORTS = ("sph_config_default", "sph_workspace_size", "sph_init", "sph_finalize
            "sph_set_accounting", "sph_kernel_launches", "sph_set_field",
            "sph_get_local_min_hc", "sph_set_global_min_hc", "sph_get_neighbor_rows",
            "sph_trace_start", "sph_trace_stop", "sph_stir_modes", "sph_stir_init", "sph_stir",
-           "sph_stir_get_state", "sph_supported_clocks")
+           "sph_stir_get_state", "sph_supported_clocks", "sph_gravity")
 GHOST_BIT = 1 << 62
 
 _lib = None
@@ -144,6 +146,7 @@ def load(build_if_missing: bool = True):
     L.sph_stir_modes.argtypes = [V, I]
     L.sph_stir_init.argtypes = [P, C.POINTER(StirParams), V, V, V, I64, I]
     L.sph_stir.argtypes = [P]
+    L.sph_gravity.argtypes = [P]
     L.sph_stir_get_state.argtypes = [P, V, C.POINTER(I64)]
     L.sph_supported_clocks.argtypes = [P, V, I, C.POINTER(I)]
     L.sph_trace_start.argtypes = [P, D, I64]
@@ -180,6 +183,12 @@ def config_from_params(params, n_capacity: int, device: int = 0, accounting: int
     c.stir_steps = int(stir_steps)
     c.divcurl = int(getattr(params, "divcurl", 0))
     c.av_switch = int(getattr(params, "av_switch", 0))
+    c.gravity = int(getattr(params, "gravity", 0))
+    if c.gravity:
+        c.grav_level = int(params.grav_level)
+        c.grav_G = float(params.grav_G)
+        c.grav_eps = float(params.grav_eps)
+        c.grav_theta = float(params.grav_theta)
     return c
 
 
@@ -370,7 +379,9 @@ class Simulation:
         return {"t": info.t, "dt": info.dt, "min_nc": info.nbr.min_nc, "max_nc": info.nbr.max_nc,
                 "mean_nc": info.nbr.mean_nc, "cell_level": info.cell_level,
                 "search_candidates": info.nbr.candidates, "search_passes": info.nbr.passes,
-                "phase_ms": {PHASES[p]: info.phase_ms[p] for p in range(NPHASES)}}
+                "phase_ms": {PHASES[p]: info.phase_ms[p] for p in range(NPHASES)},
+                "grav_multipoles": info.grav_multipoles, "grav_pairs": info.grav_pairs,
+                "grav_pops": info.grav_pops}
 
     # ---------------------------------------------------------------- energy / clocks
     def set_clock_policy(self, mode: int, mhz=None):
@@ -437,6 +448,10 @@ class Simulation:
 
     def stir(self):
         self._ok(self.L.sph_stir(self.ctx))
+
+    def gravity(self):
+        """sph_gravity: phase GRAVITY (cfg.gravity)."""
+        self._ok(self.L.sph_gravity(self.ctx))
 
     def stir_state(self):
         """(A[61, 6], number of STIR phases run)."""
