@@ -77,6 +77,9 @@ def lib():
         L.oracle_sinc.argtypes = [C.c_double]
         L.oracle_W.restype = C.c_double
         L.oracle_W.argtypes = [C.c_double, C.c_double, C.c_double]
+        L.oracle_dWdh.restype = C.c_double
+        L.oracle_dWdh.argtypes = [C.c_double, C.c_double, C.c_double]
+        L.oracle_timestep_vsig.restype = C.c_double
         L.oracle_morton.restype = C.c_uint64
         L.oracle_morton.argtypes = [C.c_uint64] * 3
         L.oracle_av_pi.restype = C.c_double
@@ -105,6 +108,11 @@ def sinc(x: float) -> float:
 
 def W(r: float, h: float, K: float) -> float:
     return lib().oracle_W(float(r), float(h), float(K))
+
+
+def dWdh(r: float, h: float, K: float) -> float:
+    """dW/dh at fixed r (oracle.c oracle_dWdh, reading 21)."""
+    return lib().oracle_dWdh(float(r), float(h), float(K))
 
 
 def morton(ix: int, iy: int, iz: int) -> int:
@@ -201,6 +209,23 @@ def density(x, y, z, h, m, bmin, bmax, periodic, nb: Neighbors, params):
     return rho
 
 
+def gradh(x, y, z, h, m, rho, bmin, bmax, periodic, nb: Neighbors, params):
+    """NormalizationGradh (reading 21): returns (omega, dsum, dsum_abs) with
+    dsum_i = sum_j m_j dW/dh(r_ij, h_i) (self term included)."""
+    x, y, z, h, m, rho = map(_d, (x, y, z, h, m, rho))
+    per = np.ascontiguousarray(periodic, dtype=np.int32)
+    bmin, bmax = _d(bmin), _d(bmax)
+    n = x.size
+    om, ds, da = np.zeros(n), np.zeros(n), np.zeros(n)
+    ps = params_struct(params)
+    idx = nb.idx if nb.idx.size else np.zeros(1, dtype=np.int64)
+    lib().oracle_gradh(C.c_int64(n), _p(x, _D), _p(y, _D), _p(z, _D), _p(h, _D), _p(m, _D),
+                       _p(rho, _D), _p(bmin, _D), _p(bmax, _D), _p(per, _I32),
+                       _p(nb.offsets, _I64), _p(idx, _I64), C.byref(ps), _p(om, _D), _p(ds, _D),
+                       _p(da, _D))
+    return om, ds, da
+
+
 def eos(rho, u, params):
     rho, u = _d(rho), _d(u)
     p = np.zeros(rho.size)
@@ -258,9 +283,10 @@ def balsara(divv, curl, c, h):
 
 
 def momentum_energy(x, y, z, vx, vy, vz, h, m, rho, p, c, Cm, bmin, bmax, periodic,
-                    nb: Neighbors, params, fav=None):
+                    nb: Neighbors, params, fav=None, omega=None):
     """Returns dict(ax, ay, az, du, a_abs [n,3], du_abs).  ``fav``: per-particle AV
-    switch factors (None = 1, the plain Monaghan viscosity)."""
+    switch factors (None = 1, the plain Monaghan viscosity).  ``omega``: grad-h
+    factors (None = the plain p/rho^2, reading 21)."""
     arrs = list(map(_d, (x, y, z, vx, vy, vz, h, m, rho, p, c)))
     Cm = np.ascontiguousarray(Cm, dtype=np.float64)
     per = np.ascontiguousarray(periodic, dtype=np.int32)
@@ -271,9 +297,11 @@ def momentum_energy(x, y, z, vx, vy, vz, h, m, rho, p, c, Cm, bmin, bmax, period
     ps = params_struct(params)
     idx = nb.idx if nb.idx.size else np.zeros(1, dtype=np.int64)
     fv = None if fav is None else _d(fav)
+    ov = None if omega is None else _d(omega)
     lib().oracle_momentum_energy(C.c_int64(n), *[_p(a, _D) for a in arrs], _p(Cm, _D),
                                  _p(bmin, _D), _p(bmax, _D), _p(per, _I32), _p(nb.offsets, _I64),
                                  _p(idx, _I64), C.byref(ps), None if fv is None else _p(fv, _D),
+                                 None if ov is None else _p(ov, _D),
                                  _p(ax, _D), _p(ay, _D), _p(az, _D),
                                  _p(du, _D), _p(aabs, _D), _p(dabs, _D))
     return {"ax": ax, "ay": ay, "az": az, "du": du, "a_abs": aabs, "du_abs": dabs}
@@ -286,6 +314,21 @@ def timestep(h, c, dt_prev, params) -> float:
     L.oracle_timestep.argtypes = [C.c_int64, _D, _D, C.c_double, C.POINTER(_Params)]
     return float(L.oracle_timestep(C.c_int64(h.size), _p(h, _D), _p(c, _D), C.c_double(dt_prev),
                                    C.byref(ps)))
+
+
+def timestep_vsig(x, y, z, vx, vy, vz, h, c, bmin, bmax, periodic, nb: Neighbors, dt_prev,
+                  params):
+    """Signal-velocity time step (reading 22).  Returns (dt, vsig [n])."""
+    arrs = list(map(_d, (x, y, z, vx, vy, vz, h, c)))
+    per = np.ascontiguousarray(periodic, dtype=np.int32)
+    bmin, bmax = _d(bmin), _d(bmax)
+    vs = np.zeros(arrs[0].size)
+    ps = params_struct(params)
+    idx = nb.idx if nb.idx.size else np.zeros(1, dtype=np.int64)
+    dt = lib().oracle_timestep_vsig(C.c_int64(vs.size), *[_p(a, _D) for a in arrs], _p(bmin, _D),
+                                    _p(bmax, _D), _p(per, _I32), _p(nb.offsets, _I64),
+                                    _p(idx, _I64), C.c_double(dt_prev), C.byref(ps), _p(vs, _D))
+    return float(dt), vs
 
 
 def update(state, acc, nc, dt, dt_m1, first_step, bmin, bmax, params):
@@ -401,11 +444,17 @@ def step(state: dict, params, dt_prev: float, first_step: bool, ngmax: int | Non
     rho = density(st["x"], st["y"], st["z"], st["h"], st["m"], bmin, bmax, params.periodic, nb,
                   params)
     p, c = eos(rho, st["u"], params)
+    omega = None
+    if getattr(params, "gradh", 0):
+        omega, dWsum, dWabs = gradh(st["x"], st["y"], st["z"], st["h"], st["m"], rho, bmin, bmax,
+                                    params.periodic, nb, params)
     Cm, tau, tabs, singular = iad(st["x"], st["y"], st["z"], st["h"], st["m"], rho, bmin, bmax,
                                   params.periodic, nb, params)
     if singular:
         raise ArithmeticError("IAD matrix singular")
     dc = {}
+    if omega is not None:
+        dc.update({"omega": omega, "dWdh_sum": dWsum, "dWdh_abs": dWabs})
     fav = None
     if getattr(params, "divcurl", 0) or getattr(params, "av_switch", 0):
         T, Tabs, dvv, curl = divcurl(st["x"], st["y"], st["z"], st["vx"], st["vy"], st["vz"],
@@ -416,7 +465,8 @@ def step(state: dict, params, dt_prev: float, first_step: bool, ngmax: int | Non
             fav = balsara(dvv, curl, c, st["h"])
             dc["bal"] = fav
     acc = momentum_energy(st["x"], st["y"], st["z"], st["vx"], st["vy"], st["vz"], st["h"],
-                          st["m"], rho, p, c, Cm, bmin, bmax, params.periodic, nb, params, fav)
+                          st["m"], rho, p, c, Cm, bmin, bmax, params.periodic, nb, params, fav,
+                          omega)
     acc.update(dc)
     if getattr(params, "gravity", 0):
         gr = gravity(st["x"], st["y"], st["z"], st["m"], params.grav_G, params.grav_eps)
@@ -426,7 +476,11 @@ def step(state: dict, params, dt_prev: float, first_step: bool, ngmax: int | Non
         acc["phi"] = gr["phi"]
     if stir is not None:
         acc["stir_B"] = stir_apply(stir, st["x"], st["y"], st["z"], dt_prev, bmin, bmax, acc)
-    dt = timestep(st["h"], c, dt_prev, params)
+    if getattr(params, "dt_vsig", 0):
+        dt, acc["vsig"] = timestep_vsig(st["x"], st["y"], st["z"], st["vx"], st["vy"], st["vz"],
+                                        st["h"], c, bmin, bmax, params.periodic, nb, dt_prev, params)
+    else:
+        dt = timestep(st["h"], c, dt_prev, params)
     out = {"bmin": bmin, "bmax": bmax, "keys": ks, "perm": perm, "nb": nb, "rho": rho, "p": p,
            "c": c, "C": Cm, "tau": tau, "tau_abs": tabs, "dt": dt,
            "pre": {f: st[f].copy() for f in STATE_KEYS}, **acc}
@@ -450,6 +504,8 @@ def sample_step(state: dict, params, dt_prev: float, first_step: bool, targets, 
     ``targets`` are positions in this step's sorted order.  Returns (order, out)
     with ``order`` = sorted ids (full) and ``out[name][k]`` the value at targets[k].
     """
+    if getattr(params, "gradh", 0) or getattr(params, "dt_vsig", 0):
+        raise NotImplementedError("sample_step covers the north-star step (no gradh / dt_vsig)")
     bmin, bmax = box(state["x"], state["y"], state["z"], params)
     k = keys(state["x"], state["y"], state["z"], bmin, bmax)
     perm = sort_order(k)

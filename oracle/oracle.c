@@ -66,6 +66,17 @@ double oracle_W(double r, double h, double K) {
   return K / (h * h * h) * pow(s, 6.0);
 }
 
+/* dW/dh of the same kernel at fixed r (NormalizationGradh, DESIGN.md reading
+ * 21).  With x = pi r / 2h, dx/dh = -x/h and x S'(x) = cos x - S(x):
+ *   dW/dh = -(K/h^4) S(x)^5 (6 cos x - 3 S(x))  for r < 2h,  0 for r >= 2h
+ * (at r = 0: -3K/h^4 = d/dh of K/h^3). */
+double oracle_dWdh(double r, double h, double K) {
+  if (r >= 2.0 * h) return 0.0;
+  double x = M_PI * r / (2.0 * h);
+  double s = oracle_sinc(x);
+  return -K / (h * h * h * h) * pow(s, 5.0) * (6.0 * cos(x) - 3.0 * s);
+}
+
 /* Minimum image of one coordinate difference:
  * raw difference first, then one conditional +-L. */
 static double min_image(double dx, double L, int periodic) {
@@ -231,6 +242,37 @@ void oracle_density(int64_t n, const double* x, const double* y, const double* z
 }
 
 /* ---------------------------------------------------------------------------
+ * NormalizationGradh (reading 21), optional step 5b:
+ *   Omega_i = 1 + (h_i / (3 rho_i)) * [ m_i dW/dh(0, h_i)
+ *                                       + sum_{j in N(i)} m_j dW/dh(r_ij, h_i) ]
+ * i.e. 1 - (dh/drho) drho/dh with h proportional to rho^(-1/3).  The
+ * momentum-energy step then uses p/(Omega rho^2) in place of p/rho^2.
+ * dsum_abs = m_i |dW/dh(0)| + sum_j m_j |dW/dh| (tolerance scale of the sum).
+ * ------------------------------------------------------------------------- */
+void oracle_gradh(int64_t n, const double* x, const double* y, const double* z,
+                  const double* h, const double* m, const double* rho, const double bmin[3],
+                  const double bmax[3], const int32_t per[3], const int64_t* off,
+                  const int64_t* idx, const oracle_params* P, double* omega, double* dsum,
+                  double* dsum_abs) {
+#pragma omp parallel for schedule(dynamic, 64)
+  for (int64_t i = 0; i < n; ++i) {
+    double d[3];
+    double t0 = m[i] * oracle_dWdh(0.0, h[i], P->K);
+    double sum = t0, sabs = fabs(t0);
+    for (int64_t k = off[i]; k < off[i + 1]; ++k) {
+      int64_t j = idx[k];
+      double r = sqrt(pair_d(x, y, z, i, j, bmin, bmax, per, d));
+      double t = m[j] * oracle_dWdh(r, h[i], P->K);
+      sum += t;
+      sabs += fabs(t);
+    }
+    dsum[i] = sum;
+    dsum_abs[i] = sabs;
+    omega[i] = 1.0 + h[i] / (3.0 * rho[i]) * sum;
+  }
+}
+
+/* ---------------------------------------------------------------------------
  * Step 6, equation of state.
  *   ideal:      p = (gamma-1) rho u,   c = sqrt(gamma (gamma-1) u)
  *   isothermal: p = c0^2 rho,          c = c0
@@ -326,12 +368,13 @@ void oracle_momentum_energy(int64_t n, const double* x, const double* y, const d
                             const double* c, const double* C, const double bmin[3],
                             const double bmax[3], const int32_t per[3], const int64_t* off,
                             const int64_t* idx, const oracle_params* P, const double* fav,
-                            double* ax, double* ay,
+                            const double* omega, double* ax, double* ay,
                             double* az, double* du, double* a_abs /* n x 3 */, double* du_abs) {
 #pragma omp parallel for schedule(dynamic, 64)
   for (int64_t i = 0; i < n; ++i) {
     double acc[3] = {0, 0, 0}, accabs[3] = {0, 0, 0}, e = 0, eabs = 0;
-    double pri = p[i] / (rho[i] * rho[i]);
+    /* grad-h (reading 21): p/(Omega rho^2) in place of p/rho^2 */
+    double pri = omega ? p[i] / (rho[i] * rho[i] * omega[i]) : p[i] / (rho[i] * rho[i]);
     for (int64_t k = off[i]; k < off[i + 1]; ++k) {
       int64_t j = idx[k];
       double d[3];
@@ -356,7 +399,7 @@ void oracle_momentum_energy(int64_t n, const double* x, const double* y, const d
       double rhobar = (rho[i] + rho[j]) / 2.0;
       double Pi = oracle_av_pi(rv, d2, hbar, cbar, rhobar, P);
       if (fav) Pi = Pi * ((fav[i] + fav[j]) / 2.0);  /* AV switch (reading 19) */
-      double prj = p[j] / (rho[j] * rho[j]);
+      double prj = omega ? p[j] / (rho[j] * rho[j] * omega[j]) : p[j] / (rho[j] * rho[j]);
       for (int a = 0; a < 3; ++a) {
         double t1 = pri * A[a], t2 = prj * B[a], t3 = Pi * G[a];
         acc[a] += -m[j] * (t1 + t2 + t3);
@@ -388,6 +431,39 @@ double oracle_timestep(int64_t n, const double* h, const double* c, double dt_pr
   double m = INFINITY;
   for (int64_t i = 0; i < n; ++i) {
     double q = h[i] / c[i];
+    if (q < m) m = q;
+  }
+  double a = P->k_cour * m, b = P->dt_max_growth * dt_prev;
+  return a < b ? a : b;
+}
+
+/* ---------------------------------------------------------------------------
+ * Step 9, signal-velocity variant (reading 22; optional):
+ *   w_ij = min(0, v_ij . d_ij / r_ij)     (d = x_i - x_j, v_ij = v_i - v_j)
+ *   vsig_i = max(2 c_i, max_{j in N(i)} (c_i + c_j - 3 w_ij))
+ *   dt = min(C * min_i h_i / vsig_i,  growth * dt_prev).
+ * vsig_out (may be NULL) receives vsig_i.
+ * ------------------------------------------------------------------------- */
+double oracle_timestep_vsig(int64_t n, const double* x, const double* y, const double* z,
+                            const double* vx, const double* vy, const double* vz,
+                            const double* h, const double* c, const double bmin[3],
+                            const double bmax[3], const int32_t per[3], const int64_t* off,
+                            const int64_t* idx, double dt_prev, const oracle_params* P,
+                            double* vsig_out) {
+  double m = INFINITY;
+  for (int64_t i = 0; i < n; ++i) {
+    double vs = 2.0 * c[i];
+    for (int64_t k = off[i]; k < off[i + 1]; ++k) {
+      int64_t j = idx[k];
+      double d[3];
+      double r = sqrt(pair_d(x, y, z, i, j, bmin, bmax, per, d));
+      double rv = d[0] * (vx[i] - vx[j]) + d[1] * (vy[i] - vy[j]) + d[2] * (vz[i] - vz[j]);
+      double w = rv < 0.0 ? rv / r : 0.0;
+      double v = c[i] + c[j] - 3.0 * w;
+      if (v > vs) vs = v;
+    }
+    if (vsig_out) vsig_out[i] = vs;
+    double q = h[i] / vs;
     if (q < m) m = q;
   }
   double a = P->k_cour * m, b = P->dt_max_growth * dt_prev;

@@ -60,6 +60,8 @@ class StepParams:
     grav_eps: float = 0.01  # Plummer softening length
     grav_theta: float = 0.5  # tree opening angle (0 = direct summation)
     grav_level: int = 6     # leaf level of the gravity octree
+    gradh: int = 0          # 1: NormalizationGradh, p/(Omega rho^2) in momentum (reading 21)
+    dt_vsig: int = 0        # 1: signal-velocity time step (reading 22)
 
     def as_dict(self):
         return asdict(self)
