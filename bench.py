@@ -59,6 +59,10 @@ def parse():
                     help="steps for the whole-step energy (>= ~2 s: the counter ticks every ~100 ms)")
     ap.add_argument("--av-switch", action="store_true",
                     help="IADVelocityDivCurl div/curl + Balsara AV switch (SURVEY 8(f)-1)")
+    ap.add_argument("--gradh", action="store_true",
+                    help="NormalizationGradh phase, p/(Omega rho^2) in momentum (SURVEY 8(f)-1)")
+    ap.add_argument("--dt-vsig", action="store_true",
+                    help="signal-velocity time step (SURVEY 8(f)-1)")
     ap.add_argument("--stir", action="store_true",
                     help="turbulence driving (OU stirring, SURVEY 8(f)-3) inside every step")
     ap.add_argument("--trace-seconds", type=float, default=1.5,
@@ -380,9 +384,10 @@ def main():
     torch.cuda.set_device(local)
     w = make_workload(args.workload, rank)
     n = w.n
-    if args.av_switch:
+    if args.av_switch or args.gradh or args.dt_vsig:
         import dataclasses
-        w.params = dataclasses.replace(w.params, av_switch=1)
+        w.params = dataclasses.replace(w.params, av_switch=int(args.av_switch),
+                                       gradh=int(args.gradh), dt_vsig=int(args.dt_vsig))
     stir_steps = 8192 if args.stir else 0
     sim = sph.Simulation(w.params, n_capacity=n, device=local, stir_steps=stir_steps)
     stream = sim.stream
@@ -492,7 +497,8 @@ def main():
                 "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
                 "config": {"workload": args.workload + ("+stir" if args.stir else "")
-                           + ("+balsara" if args.av_switch else ""),
+                           + ("+balsara" if args.av_switch else "")
+                           + ("+gradh" if args.gradh else "") + ("+vsig" if args.dt_vsig else ""),
                            "n_particles_per_gpu": n,
                            "n_particles_total": n * world,
                            "parallelism": "single GPU" if world == 1 else

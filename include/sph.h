@@ -92,7 +92,9 @@ typedef enum sph_phase {
                                     MOMENTUM_ENERGY, before TIMESTEP, when enabled */
   SPH_PHASE_GRAVITY = 11,        /* self-gravity; runs after
                                     MOMENTUM_ENERGY when cfg.gravity              */
-  SPH_NPHASES = 12
+  SPH_PHASE_GRADH = 12,          /* NormalizationGradh (reading 21); runs
+                                    after EOS, before IAD, when cfg.gradh          */
+  SPH_NPHASES = 13
 } sph_phase;
 
 typedef enum sph_clock_mode {
@@ -115,6 +117,8 @@ typedef enum sph_field {
   SPH_F_CURLX, SPH_F_CURLY, SPH_F_CURLZ,  /* velocity curl (cfg.divcurl)        */
   SPH_F_BAL,    /* Balsara switch factor (cfg.av_switch; valid after sph_iad)  */
   SPH_F_PHI,    /* gravitational potential (cfg.gravity; after sph_gravity)    */
+  SPH_F_OMEGA,  /* grad-h factor Omega (cfg.gradh; valid after sph_gradh)        */
+  SPH_F_VSIG,   /* signal velocity (cfg.dt_vsig; after sph_momentum_energy)    */
   SPH_NFIELDS
 } sph_field;
 
@@ -152,7 +156,11 @@ typedef struct sph_config {
   double grav_eps;          /* Plummer softening length                            */
   double grav_theta;        /* opening angle: multipole when side < theta * dist;
                                0 = direct summation                               */
-  int32_t reserved[8];
+  int32_t gradh;            /* 1: NormalizationGradh phase; momentum-energy uses
+                               p / (Omega rho^2) (reading 21)                     */
+  int32_t dt_vsig;          /* 1: signal-velocity time step (reading 22) instead of
+                               C min h/c                                          */
+  int32_t reserved[6];
 } sph_config;
 
 typedef struct sph_nbr_stats {
@@ -381,6 +389,20 @@ int sph_kernel_launches(int64_t* count);
  * so reps should make the call last >= 1 s.  Synchronises. */
 int sph_repeat_phase(sph_ctx* ctx, int phase, int reps, double* ms_per_call,
                      double* joules_per_call);
+
+/* --- NormalizationGradh and the signal-velocity time step -- */
+
+/* Phase GRADH (NormalizationGradh; reading 21 of DESIGN.md, the paper
+ * prints no formula): Omega_i = 1 + (h_i / (3 rho_i)) sum_j m_j dW(r_ij, h_i)/dh_i
+ * over the neighbour list plus the self term (dW/dh = -(K/h^4) S^5 (6 cos x - 3 S),
+ * x = pi r / 2h), i.e. 1 + (h/3rho) d rho/dh.  Writes Omega (SPH_F_OMEGA) and
+ * replaces p/rho^2 by p/(Omega rho^2) in the momentum-energy terms.  Needs
+ * cfg.gradh; after sph_eos, before sph_iad (sph_iad returns SPH_ERR_STATE while
+ * it is pending).  sph_step runs it when cfg.gradh.  With cfg.dt_vsig the
+ * momentum-energy phase also forms vsig_i = max(2 c_i, max_j (c_i + c_j - 3 w_ij)),
+ * w_ij = min(0, v_ij . d_ij / r_ij) (SPH_F_VSIG), and the time step becomes
+ * dt = min(C min_i h_i / vsig_i, growth dt_prev) (reading 22). */
+int sph_gradh(sph_ctx* ctx);
 
 /* --- self-gravity ------------------------------------------ */
 

@@ -25,7 +25,8 @@ enum Stage { S_INIT = 0, S_PART, S_TREE, S_NBR, S_DENS, S_EOS, S_IAD, S_MOM, S_D
 
 const char* kPhaseNames[SPH_NPHASES] = {"keys",    "sort",    "cells", "neighbors",
                                         "density", "eos",     "iad",   "momentum_energy",
-                                        "timestep", "update",  "stir", "gravity"};
+                                        "timestep", "update",  "stir", "gravity",
+                                        "gradh"};
 
 thread_local char g_err[512] = "";
 
@@ -65,6 +66,9 @@ struct sph_ctx {
   double *divv, *curl[3], *bal;
   Rec4* rec_iv = nullptr;
   double* phi = nullptr;
+  double* omega = nullptr;  // cfg.gradh
+  double* vsig = nullptr;   // cfg.dt_vsig
+  bool gradh_done = false;  // GRADH ran since the last EOS (cfg.gradh)
   uint32_t* gcell_start = nullptr;
   Rec4* gmom = nullptr;
   int32_t *nc, *nbr, *nrows;
@@ -149,6 +153,7 @@ Fields fields(sph_ctx* c) {
   F.ax = c->ax; F.ay = c->ay; F.az = c->az; F.du = c->du;
   F.divv = c->divv; F.bal = c->P.av_switch ? c->bal : nullptr; F.rec_iv = c->rec_iv;
   F.phi = c->phi; F.gcell_start = c->gcell_start; F.gmom = c->gmom;
+  F.omega = c->omega; F.vsig = c->vsig;
   for (int a = 0; a < 3; ++a) F.curl[a] = c->curl[a];
   F.nc = c->nc; F.nbr = c->nbr; F.ngmax = c->cfg.ngmax;
   F.nrows = c->nrows; F.nrows_ld = nrows_ld(&c->cfg);
@@ -331,7 +336,14 @@ int body_simple(sph_ctx* c, int phase, int next_stage) {
   Fields F = fields(c);
   switch (phase) {
     case SPH_PHASE_DENSITY: launch_density(F, c->P, c->st); break;
-    case SPH_PHASE_EOS: launch_eos(F, c->P, c->st); break;
+    case SPH_PHASE_EOS:
+      launch_eos(F, c->P, c->st);
+      c->gradh_done = false;
+      break;
+    case SPH_PHASE_GRADH:
+      launch_gradh(F, c->P, c->st);
+      c->gradh_done = true;
+      break;
     case SPH_PHASE_IAD: launch_iad(F, c->P, c->st); break;
     case SPH_PHASE_MOMENTUM_ENERGY:
       if (c->rec_m_dirty) {  // ghosts' C were overwritten (sph_set_field)
@@ -412,6 +424,8 @@ static int validate(const sph_config* c) {
   if (c->stir_steps < 0) return fail(nullptr, SPH_ERR_ARG, "stir_steps < 0");
   if (c->divcurl < 0 || c->divcurl > 1 || c->av_switch < 0 || c->av_switch > 1)
     return fail(nullptr, SPH_ERR_ARG, "divcurl and av_switch must be 0 or 1");
+  if (c->gradh < 0 || c->gradh > 1 || c->dt_vsig < 0 || c->dt_vsig > 1)
+    return fail(nullptr, SPH_ERR_ARG, "gradh and dt_vsig must be 0 or 1");
   if (c->gravity) {
     if (c->periodic[0] || c->periodic[1] || c->periodic[2])
       return fail(nullptr, SPH_ERR_NOT_SUPPORTED, "gravity is for isolated (fully open) boxes");
@@ -464,6 +478,12 @@ static size_t layout(const sph_config* cfg, char* base, sph_ctx* c) {
   char* rm = take(sizeof(Rec4) * kRecM * cap);
   char* riv = (cfg->divcurl || cfg->av_switch) ? take(sizeof(Rec4) * cap) : nullptr;
   if (c) c->rec_iv = (Rec4*)riv;
+  char* om = cfg->gradh ? take(D) : nullptr;
+  char* vsg = cfg->dt_vsig ? take(D) : nullptr;
+  if (c) {
+    c->omega = (double*)om;
+    c->vsig = (double*)vsg;
+  }
   if (cfg->gravity) {
     const int Lt = cfg->grav_level;
     const size_t ncells = (size_t)((((int64_t)1 << (3 * (Lt + 1))) - 1) / 7);
@@ -553,6 +573,8 @@ int sph_init(const sph_config* cfg, void* arena, size_t arena_bytes, void* strea
   c->P.av_beta = cfg->av_beta; c->P.av_eps = cfg->av_eps; c->P.max_cell_level = cfg->max_cell_level;
   c->P.av_switch = cfg->av_switch ? 1 : 0;
   c->P.divcurl = (cfg->divcurl || cfg->av_switch) ? 1 : 0;
+  c->P.gradh = cfg->gradh ? 1 : 0;
+  c->P.dt_vsig = cfg->dt_vsig ? 1 : 0;
   layout(cfg, (char*)arena, c);
   for (int p = 0; p < SPH_NPHASES; ++p) {
     c->pending[p] = false;
@@ -684,6 +706,14 @@ int sph_get_field(sph_ctx* c, int field, void* dst, int mem) {
     if (!c->phi) return fail(c, SPH_ERR_ARG, "SPH_F_PHI needs cfg.gravity");
     src = c->phi;
   }
+  else if (field == SPH_F_OMEGA) {
+    if (!c->omega) return fail(c, SPH_ERR_ARG, "SPH_F_OMEGA needs cfg.gradh");
+    src = c->omega;
+  }
+  else if (field == SPH_F_VSIG) {
+    if (!c->vsig) return fail(c, SPH_ERR_ARG, "SPH_F_VSIG needs cfg.dt_vsig");
+    src = c->vsig;
+  }
   else return fail(c, SPH_ERR_ARG, "unknown field %d", field);
   if (c->n == 0) return SPH_OK;
   const cudaMemcpyKind kind = mem == SPH_MEM_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
@@ -711,6 +741,16 @@ int sph_set_field(sph_ctx* c, int field, const void* src, int mem) {
     if (c->stage < S_IAD) return fail(c, SPH_ERR_STATE, "sph_set_field(BAL) before sph_iad");
     dst = c->bal;
     c->rec_m_dirty = true;
+  } else if (field == SPH_F_OMEGA && c->omega) {
+    // owners' Omega over the ghosts (multi-GPU halo): p/(Omega rho^2) follows
+    if (!c->gradh_done || c->stage != S_EOS)
+      return fail(c, SPH_ERR_STATE, "sph_set_field(OMEGA) must follow sph_gradh, before sph_iad");
+    if (c->n == 0) return SPH_OK;
+    const cudaMemcpyKind k2 = mem == SPH_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
+    rc = cuda_check(c, cudaMemcpyAsync(c->omega, src, sizeof(double) * c->n, k2, c->st), "set field");
+    if (rc) return rc;
+    launch_prho2(fields(c), c->st);
+    return cuda_check(c, cudaGetLastError(), "prho2");
   } else {
     return fail(c, SPH_ERR_ARG, "field %d is not settable", field);
   }
@@ -832,9 +872,18 @@ int sph_eos(sph_ctx* c) {
   return rc ? rc : body_simple(c, SPH_PHASE_EOS, S_EOS);
 }
 
+int sph_gradh(sph_ctx* c) {
+  int rc = check_ready(c, S_EOS, "sph_gradh");
+  if (rc) return rc;
+  if (!c->cfg.gradh) return fail(c, SPH_ERR_STATE, "gradh not enabled (cfg.gradh = 0)");
+  return body_simple(c, SPH_PHASE_GRADH, S_EOS);
+}
+
 int sph_iad(sph_ctx* c) {
   int rc = check_ready(c, S_EOS, "sph_iad");
-  return rc ? rc : body_simple(c, SPH_PHASE_IAD, S_IAD);
+  if (rc) return rc;
+  if (c->cfg.gradh && !c->gradh_done) return fail(c, SPH_ERR_STATE, "cfg.gradh: sph_gradh must run before sph_iad");
+  return body_simple(c, SPH_PHASE_IAD, S_IAD);
 }
 
 int sph_momentum_energy(sph_ctx* c) {
@@ -863,6 +912,7 @@ int sph_step(sph_ctx* c, sph_step_info* info) {
   if ((rc = body_neighbors(c))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_DENSITY, S_DENS))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_EOS, S_EOS))) return rc;
+  if (c->cfg.gradh && (rc = body_simple(c, SPH_PHASE_GRADH, S_EOS))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_IAD, S_IAD))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_MOMENTUM_ENERGY, S_MOM))) return rc;
   if (c->cfg.gravity && (rc = body_simple(c, SPH_PHASE_GRAVITY, S_MOM))) return rc;
@@ -994,6 +1044,10 @@ int sph_repeat_phase(sph_ctx* c, int phase, int reps, double* ms_per_call, doubl
     case SPH_PHASE_DENSITY: need = S_NBR; break;
     case SPH_PHASE_EOS: need = S_DENS; break;
     case SPH_PHASE_IAD: need = S_EOS; break;
+    case SPH_PHASE_GRADH:
+      if (!c || !c->cfg.gradh) return fail(c, SPH_ERR_STATE, "gradh not enabled (cfg.gradh = 0)");
+      need = S_EOS;
+      break;
     case SPH_PHASE_MOMENTUM_ENERGY: need = S_IAD; break;
     case SPH_PHASE_TIMESTEP: need = S_DT; break;
     default: return fail(c, SPH_ERR_ARG, "phase %d is not repeatable (it changes the state)", phase);
@@ -1038,6 +1092,7 @@ int sph_repeat_phase(sph_ctx* c, int phase, int reps, double* ms_per_call, doubl
       case SPH_PHASE_DENSITY: launch_density(F, c->P, c->st); break;
       case SPH_PHASE_EOS: launch_eos(F, c->P, c->st); break;
       case SPH_PHASE_IAD: launch_iad(F, c->P, c->st); break;
+      case SPH_PHASE_GRADH: launch_gradh(F, c->P, c->st); break;
       case SPH_PHASE_MOMENTUM_ENERGY: launch_momentum_energy(F, c->P, c->st); break;
     }
   }

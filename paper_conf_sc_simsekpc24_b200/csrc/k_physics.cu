@@ -161,6 +161,66 @@ __global__ void __launch_bounds__(256) eos_kernel(Fields F, Params P) {
   if (P.divcurl) st4(F.rec_iv + i, F.f[FVX][i], F.f[FVY][i], F.f[FVZ][i], 0.0);
 }
 
+// ------------------------------------------------------------------ GRADH
+// NormalizationGradh (reading 21): Omega_i = 1 + (h_i/(3 rho_i)) sum_j m_j dW/dh,
+// dW/dh = -(K/h^4) S^5 (6 cos x - 3 S), x = pi r/2h, self term 3 m_i inside the
+// bracket.  sin and cos of pi*r/2h come from one sincospi; then
+// p/rho^2 -> p/(Omega rho^2) for the momentum records (written by IAD).
+// Per pair: one 32-B record {x, y, z, m} (the density record).
+template <bool kWrap>
+__device__ __forceinline__ void gradh_body(const Fields& F, const Params& P, const Geom& g, int64_t i,
+                                           const Rec4& me, double hi) {
+  const int nci = min(F.nc[i], F.ngmax);
+  const double inv2h = 0.5 / hi;
+  double sum = 3.0 * me.d;  // self: S = 1, cos = 1
+  const int32_t* __restrict__ nb = F.nbr + i;
+  const Rec4* __restrict__ rec = F.rec_d;
+  const int64_t cap = F.cap;
+  int jn = nci > 0 ? __ldg(nb) : 0;
+  Rec4 ra = ldg4(rec + jn);
+  jn = nci > 1 ? __ldg(nb + cap) : 0;
+  for (int k = 0; k < nci; ++k) {
+    const Rec4 rj = ra;
+    if (k + 1 < nci) ra = ldg4(rec + jn);
+    if (k + 2 < nci) jn = __ldg(nb + (int64_t)(k + 2) * cap);
+    double dx, dy, dz;
+    pair_d<kWrap>(g, me.a, me.b, me.c, rj.a, rj.b, rj.c, dx, dy, dz);
+    const double y = sqrt(dx * dx + dy * dy + dz * dz) * inv2h;  // x = pi y
+    double sn, cs;
+    sincospi(y, &sn, &cs);
+    const double S = y > 0.0 ? sn / (kPi * y) : 1.0;
+    const double S2 = S * S;
+    sum = fma(rj.d * (S2 * S2 * S), 6.0 * cs - 3.0 * S, sum);
+  }
+  const double rho = F.rho[i];
+  const double h2 = hi * hi;
+  const double dsum = -P.K / (h2 * h2) * sum;
+  const double om = 1.0 + hi / (3.0 * rho) * dsum;
+  F.omega[i] = om;
+  F.prho2[i] = __ddiv_rn(F.p[i], __dmul_rn(__dmul_rn(rho, rho), om));
+}
+
+__global__ void __launch_bounds__(256) gradh_kernel(Fields F, Params P) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= F.n) return;
+  const Geom g = load_geom(F.ds, P);
+  const Rec4 me = F.rec_d[i];
+  const double hi = F.f[FH][i];
+  if (__any_sync(__activemask(), needs_wrap(g, me.a, me.b, me.c, hi)))
+    gradh_body<true>(F, P, g, i, me, hi);
+  else
+    gradh_body<false>(F, P, g, i, me, hi);
+}
+
+// p/(Omega rho^2) again after sph_set_field wrote the owners' Omega over the
+// ghosts (multi-GPU halo).
+__global__ void __launch_bounds__(256) prho2_kernel(Fields F) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= F.n) return;
+  const double rho = F.rho[i];
+  F.prho2[i] = __ddiv_rn(F.p[i], __dmul_rn(__dmul_rn(rho, rho), F.omega[i]));
+}
+
 // ------------------------------------------------------------------ IAD
 // tau_i = sum_j V_j W(r,h_i) Delta Delta^T, C_i = tau_i^{-1} (adjugate / det);
 // epilogue: the momentum record of particle i.  Per pair: one 32-B record
@@ -341,8 +401,8 @@ __global__ void __launch_bounds__(kIadThreads, 768 / kIadThreads) iad_kernel(Fie
 // order-preserving bit pattern of a positive double).
 // Per pair: 4 records (128 B) + 1 more (AV) for approaching pairs, 157 DP flops
 // (+ 17 and 2 divisions when approaching).
-template <bool kWrap, bool kSwitch>
-__device__ __forceinline__ void momentum_body(const Fields& F, const Params& P, const Geom& g, int64_t i) {
+template <bool kWrap, bool kSwitch, bool kVsig>
+__device__ __forceinline__ double momentum_body(const Fields& F, const Params& P, const Geom& g, int64_t i) {
   const Rec4* __restrict__ rec = F.rec_m;
   const Rec4* mi = rec + (int64_t)kRecM * i;
   const Rec4 i0 = mi[0], i1 = mi[1], i2 = mi[2], i3 = mi[3], i4 = mi[4];
@@ -354,6 +414,7 @@ __device__ __forceinline__ void momentum_body(const Fields& F, const Params& P, 
   const double alpha = P.av_alpha, beta = P.av_beta, eps = P.av_eps;
   const int nci = min(F.nc[i], F.ngmax);
   double ax = 0, ay = 0, az = 0, de = 0;
+  double vs = kVsig ? 2.0 * ci : ci;  // signal velocity (reading 22); c_i without it
   const int32_t* __restrict__ nb = F.nbr + i;
   // software pipeline: neighbour index three ahead, the position chunk (needed
   // first) two ahead; the other chunks are loaded at the top of the iteration
@@ -397,8 +458,14 @@ __device__ __forceinline__ void momentum_body(const Fields& F, const Params& P, 
     const double vx = vxi - j3.a, vy = vyi - j3.b, vz = vzi - j3.c;
     const double rv = dx * vx + dy * vy + dz * vz;
     double Pi = 0.0;
+    Rec4 j4v;
+    if (kVsig) {  // vsig_ij = c_i + c_j - 3 min(0, rv / r)
+      j4v = ldg4(rcur + 4);
+      const double w = rv < 0.0 ? rv / sqrt(r2) : 0.0;
+      vs = fmax(vs, ci + j4v.b - 3.0 * w);
+    }
     if (rv < 0.0) {
-      const Rec4 j4 = ldg4(rcur + 4);
+      const Rec4 j4 = kVsig ? j4v : ldg4(rcur + 4);
       const double hbar = 0.5 * (hi + j4.a);
       const double cbar = 0.5 * (ci + j4.b);
       const double rhobar = 0.5 * (rhoi + j4.c);
@@ -423,6 +490,8 @@ __device__ __forceinline__ void momentum_body(const Fields& F, const Params& P, 
   F.ay[i] = ay;
   F.az[i] = az;
   F.du[i] = de;
+  if (kVsig) F.vsig[i] = vs;
+  return vs;
 }
 
 __global__ void __launch_bounds__(kMomThreads, 512 / kMomThreads) momentum_energy_kernel(Fields F, Params P) {
@@ -434,14 +503,16 @@ __global__ void __launch_bounds__(kMomThreads, 512 / kMomThreads) momentum_energ
     const Rec4* mi = F.rec_m + (int64_t)kRecM * i;
     const Rec4 i0 = mi[0], i4 = mi[4];
     const bool wrap = __any_sync(__activemask(), needs_wrap(g, i0.a, i0.b, i0.c, i4.a));
-    if (P.av_switch) {
-      if (wrap) momentum_body<true, true>(F, P, g, i);
-      else momentum_body<false, true>(F, P, g, i);
+    double vs;  // c_i, or the signal velocity with cfg.dt_vsig
+    if (P.dt_vsig) {
+      if (P.av_switch) vs = wrap ? momentum_body<true, true, true>(F, P, g, i) : momentum_body<false, true, true>(F, P, g, i);
+      else vs = wrap ? momentum_body<true, false, true>(F, P, g, i) : momentum_body<false, false, true>(F, P, g, i);
+    } else if (P.av_switch) {
+      vs = wrap ? momentum_body<true, true, false>(F, P, g, i) : momentum_body<false, true, false>(F, P, g, i);
     } else {
-      if (wrap) momentum_body<true, false>(F, P, g, i);
-      else momentum_body<false, false>(F, P, g, i);
+      vs = wrap ? momentum_body<true, false, false>(F, P, g, i) : momentum_body<false, false, false>(F, P, g, i);
     }
-    hc = ord_of(__ddiv_rn(i4.a, i4.b));
+    hc = ord_of(__ddiv_rn(i4.a, vs));
   }
 #pragma unroll
   for (int off = 16; off > 0; off >>= 1) {
@@ -532,6 +603,16 @@ void launch_iad(const Fields& F, const Params& P, cudaStream_t st) {
     iad_dc_kernel<<<(unsigned)div_up(F.n, 512), 512, 0, st>>>(F, P);
   else
     iad_kernel<<<(unsigned)div_up(F.n, kIadThreads), kIadThreads, 0, st>>>(F, P);
+  note_launch();
+}
+void launch_gradh(const Fields& F, const Params& P, cudaStream_t st) {
+  if (F.n == 0) return;
+  gradh_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F, P);
+  note_launch();
+}
+void launch_prho2(const Fields& F, cudaStream_t st) {
+  if (F.n == 0) return;
+  prho2_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F);
   note_launch();
 }
 void launch_momentum_energy(const Fields& F, const Params& P, cudaStream_t st) {

@@ -110,6 +110,7 @@ struct Fields {
   double *divv, *curl[3], *bal;  // IADVelocityDivCurl extras (cfg.divcurl / av_switch)
   Rec4* rec_iv;           // {vx, vy, vz, 0} gather record of the div/curl sums (EOS)
   double* phi;            // gravitational potential (GRAVITY)
+  double *omega, *vsig;   // grad-h factor (GRADH), signal velocity (cfg.dt_vsig)
   uint32_t* gcell_start;  // gravity octree: leaf ranges at level grav_level
   Rec4* gmom;             // gravity octree moments, 3 records per cell, levels 0..Lt
   int32_t* nc;
@@ -133,6 +134,7 @@ struct Params {
   double av_alpha, av_beta, av_eps;
   int max_cell_level;
   int divcurl, av_switch;
+  int gradh, dt_vsig;
 };
 
 // Process-wide count of libsph kernel launches (sph_kernel_launches).
@@ -240,6 +242,8 @@ constexpr int kNbrSlotRows = 128;  // scratch rows per CTA (its threads)
 void launch_density(const Fields& F, const Params& P, cudaStream_t st);
 void launch_eos(const Fields& F, const Params& P, cudaStream_t st);
 void launch_iad(const Fields& F, const Params& P, cudaStream_t st);
+void launch_gradh(const Fields& F, const Params& P, cudaStream_t st);
+void launch_prho2(const Fields& F, cudaStream_t st);
 void launch_momentum_energy(const Fields& F, const Params& P, cudaStream_t st);
 void launch_timestep(const Fields& F, const Params& P, cudaStream_t st);
 void launch_update(const Fields& F, const Params& P, cudaStream_t st);

@@ -237,6 +237,9 @@ class DistributedSim:
         dst_pos = [positions_of(ids_now, g) for g in ghost_ids]       # their particles I hold
         self._halo(["rho"], src_pos, dst_pos)
         sim.eos()
+        if getattr(self.params, "gradh", 0):  # owners' Omega over the ghosts
+            sim.gradh()
+            self._halo(["omega"], src_pos, dst_pos)
         sim.iad()
         # H3: the owners' C (and Balsara factors when the AV switch is on)
         h3 = ["c11", "c12", "c13", "c22", "c23", "c33"]

@@ -21,12 +21,12 @@ STATUS = {0: "OK", 1: "ERR_ARG", 2: "ERR_STATE", 3: "ERR_CUDA", 4: "ERR_NCCL", 5
           6: "ERR_NO_PERMISSION", 7: "ERR_NOT_SUPPORTED", 8: "ERR_CAPACITY", 9: "ERR_HCAP",
           10: "ERR_SINGULAR", 11: "ERR_BOX"}
 PHASES = ("keys", "sort", "cells", "neighbors", "density", "eos", "iad", "momentum_energy",
-          "timestep", "update", "stir", "gravity")
+          "timestep", "update", "stir", "gravity", "gradh")
 STIR_NMODES = 61
 NPHASES = len(PHASES)
 FIELDS = ("x", "y", "z", "vx", "vy", "vz", "h", "m", "u", "du_m1", "id", "key", "nc", "rho", "p",
           "c", "c11", "c12", "c13", "c22", "c23", "c33", "ax", "ay", "az", "du", "divv", "curlx",
-          "curly", "curlz", "bal", "phi")
+          "curly", "curlz", "bal", "phi", "omega", "vsig")
 FIELD_ID = {name: k for k, name in enumerate(FIELDS)}
 FIELD_DTYPE = {"id": np.int64, "key": np.uint64, "nc": np.int32}
 MEM_HOST, MEM_DEVICE = 0, 1
@@ -52,7 +52,8 @@ class Config(C.Structure):
         ("accounting", C.c_int32), ("rank", C.c_int32), ("nranks", C.c_int32),
         ("stir_steps", C.c_int32), ("divcurl", C.c_int32), ("av_switch", C.c_int32),
         ("gravity", C.c_int32), ("grav_level", C.c_int32), ("grav_G", C.c_double),
-        ("grav_eps", C.c_double), ("grav_theta", C.c_double), ("reserved", C.c_int32 * 8),
+        ("grav_eps", C.c_double), ("grav_theta", C.c_double), ("gradh", C.c_int32),
+        ("dt_vsig", C.c_int32), ("reserved", C.c_int32 * 6),
     ]
 
 
@@ -93,7 +94,7 @@ EXPORTS = ("sph_config_default", "sph_workspace_size", "sph_init", "sph_finalize
            "sph_set_accounting", "sph_kernel_launches", "sph_set_field",
            "sph_get_local_min_hc", "sph_set_global_min_hc", "sph_get_neighbor_rows",
            "sph_trace_start", "sph_trace_stop", "sph_stir_modes", "sph_stir_init", "sph_stir",
-           "sph_stir_get_state", "sph_supported_clocks", "sph_gravity")
+           "sph_stir_get_state", "sph_supported_clocks", "sph_gravity", "sph_gradh")
 GHOST_BIT = 1 << 62
 
 _lib = None
@@ -147,6 +148,7 @@ def load(build_if_missing: bool = True):
     L.sph_stir_init.argtypes = [P, C.POINTER(StirParams), V, V, V, I64, I]
     L.sph_stir.argtypes = [P]
     L.sph_gravity.argtypes = [P]
+    L.sph_gradh.argtypes = [P]
     L.sph_stir_get_state.argtypes = [P, V, C.POINTER(I64)]
     L.sph_supported_clocks.argtypes = [P, V, I, C.POINTER(I)]
     L.sph_trace_start.argtypes = [P, D, I64]
@@ -184,6 +186,8 @@ def config_from_params(params, n_capacity: int, device: int = 0, accounting: int
     c.divcurl = int(getattr(params, "divcurl", 0))
     c.av_switch = int(getattr(params, "av_switch", 0))
     c.gravity = int(getattr(params, "gravity", 0))
+    c.gradh = int(getattr(params, "gradh", 0))
+    c.dt_vsig = int(getattr(params, "dt_vsig", 0))
     if c.gravity:
         c.grav_level = int(params.grav_level)
         c.grav_G = float(params.grav_G)
@@ -452,6 +456,10 @@ class Simulation:
     def gravity(self):
         """sph_gravity: phase GRAVITY (cfg.gravity)."""
         self._ok(self.L.sph_gravity(self.ctx))
+
+    def gradh(self):
+        """sph_gradh: phase GRADH, NormalizationGradh (cfg.gradh)."""
+        self._ok(self.L.sph_gradh(self.ctx))
 
     def stir_state(self):
         """(A[61, 6], number of STIR phases run)."""

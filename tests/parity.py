@@ -22,6 +22,8 @@ def gpu_pipeline(sim):
     stats = sim.find_neighbors()
     sim.density()
     sim.eos()
+    if sim.cfg.gradh:
+        sim.gradh()
     sim.iad()
     sim.momentum_energy()
     out = {k: sim.get_field(k) for k in ("id", "key", "nc", "rho", "p", "c", "ax", "ay", "az", "du",

@@ -33,9 +33,17 @@ def _sedov_balsara():
     return w
 
 
+def _random_gradh_vsig():
+    import dataclasses
+    w = ics.random_box(6000, seed=5)
+    w.params = dataclasses.replace(w.params, gradh=1, dt_vsig=1)  # halo of Omega
+    return w
+
+
 def _make(name):
     return {"turbulence16": lambda: ics.turbulence(16), "random": lambda: ics.random_box(6000, seed=5),
-            "sedov14": lambda: ics.sedov(14), "sedov14_balsara": _sedov_balsara}[name]()
+            "sedov14": lambda: ics.sedov(14), "sedov14_balsara": _sedov_balsara,
+            "random_gradh_vsig": _random_gradh_vsig}[name]()
 
 
 def _worker(rank, world, port, name, q):
@@ -69,7 +77,8 @@ def _single(name):
     return dts, {k: v[o] for k, v in st.items()}
 
 
-@pytest.mark.parametrize("name", ["turbulence16", "random", "sedov14", "sedov14_balsara"])
+@pytest.mark.parametrize("name", ["turbulence16", "random", "sedov14", "sedov14_balsara",
+                                  "random_gradh_vsig"])
 def test_two_ranks_bit_identical_to_one(name):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
