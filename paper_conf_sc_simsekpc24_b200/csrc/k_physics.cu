@@ -438,9 +438,9 @@ __device__ __forceinline__ double momentum_body(const Fields& F, const Params& P
     double dx, dy, dz;
     pair_d<kWrap>(g, xi, yi, zi, j0.a, j0.b, j0.c, dx, dy, dz);
     const double r2 = dx * dx + dy * dy + dz * dz;
-    const double wi = khi * sinc6_t(r2 * qi);
+    const double wi = khi * sinc6_t_cb(r2 * qi);
     const double tj = r2 * j0.d;
-    const double wj = tj < kPi2 ? j1.d * sinc6_t(tj) : 0.0;
+    const double wj = tj < kPi2 ? j1.d * sinc6_t_cb(tj) : 0.0;
     // Delta = -d.  With A = w_i C_i Delta, B = w_j C_j Delta, G = (A+B)/2 the
     // pair terms regroup exactly (up to rounding) as
     //   (p_i/rho_i^2) A + (p_j/rho_j^2) B + Pi G
