@@ -1,4 +1,4 @@
-"""Physics of the GPU step over many steps (SURVEY 8(c) pins 'Sedov' and
+"""Physics of the GPU step over many steps (SURVEY 8(c) pins "Sedov", "Noh" and
 'Integrator'): the Sedov blast radius follows the similarity solution
 R(t) = xi0 (E t^2 / rho0)^(1/5), xi0 = 1.1517 for gamma = 5/3, and total energy
 sum m (v^2/2 + u) is conserved to 1e-3 over the run."""
@@ -44,3 +44,45 @@ def test_sedov_blast_radius_and_energy(golden):
     assert abs(R_num - R_th) / R_th < 0.12, (R_num, R_th, t, steps)
     # strong-shock compression: the peak density is well above ambient
     assert rho[top].mean() > 2.0
+
+
+def test_noh_implosion_jumps():
+    """Noh (SURVEY 8(c) pin 'Noh'; config 4's workload, 80^3 lattice, open box):
+    at t = 0.3 the pre-shock gas follows rho = (1 + t/r)^2 with v_r = -1, the
+    shocked gas is at rest with u = 1/2 (gamma = 5/3), and the shock sits at
+    r = t/3.  Run with the signal-velocity time step (reading 22): the cold
+    inflow has c ~ 0, so the sound-speed criterion alone would not resolve it.
+    SPH smooths the jump, so the post-shock density (64 exactly) is only
+    required to exceed 0.6 of it and the shock radius to be within 30%."""
+    import dataclasses
+    from paper_conf_sc_simsekpc24_b200 import sph
+    w = ics.noh(80)
+    w.params = dataclasses.replace(w.params, dt_vsig=1, ngmax=400)
+    sim = sph.Simulation(w.params, n_capacity=w.n)
+    sim.set_particles({k: np.ascontiguousarray(v) for k, v in w.state.items()})
+    sim.set_time(0.0, w.params.dt_first, True)
+    t, steps = 0.0, 0
+    while t < 0.3 and steps < 3000:
+        t = sim.step()["t"]
+        steps += 1
+    st = sim.get_state()
+    rho = sim.get_field("rho")
+    r = np.sqrt(st["x"] ** 2 + st["y"] ** 2 + st["z"] ** 2)
+    vr = (st["vx"] * st["x"] + st["vy"] * st["y"] + st["vz"] * st["z"]) / np.maximum(r, 1e-12)
+    sim.finalize()
+    # undisturbed inflow: outside the shock (+ a smoothing length) and inside
+    # r < 0.5 - t (the cube's faces have reached r = 0.2 along the axes)
+    pre = (r > 0.145) & (r < 0.175)
+    ratio = rho[pre] / (1 + t / r[pre]) ** 2
+    assert abs(np.median(ratio) - 1) < 0.03 and abs(np.mean(ratio) - 1) < 0.06
+    assert np.abs(np.median(vr[pre]) + 1) < 0.03
+    post = (r > 0.05) & (r < 0.09)
+    assert abs(np.median(st["u"][post]) - 0.5) < 0.1
+    assert np.median(np.abs(vr[post])) < 0.05
+    assert np.median(rho[post]) > 0.6 * 64
+    # shock radius: where the median u of thin shells crosses 1/4
+    edges = np.linspace(0.02, 0.3, 57)
+    mids = 0.5 * (edges[1:] + edges[:-1])
+    umed = np.array([np.median(st["u"][(r >= a) & (r < b)]) for a, b in zip(edges[:-1], edges[1:])])
+    Rs = mids[np.argmax(umed < 0.25)]
+    assert abs(Rs - t / 3) / (t / 3) < 0.3, (Rs, t, steps)
