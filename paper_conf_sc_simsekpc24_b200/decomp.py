@@ -180,6 +180,18 @@ class DistributedSim:
         self.box_len = [float(b - a) for a, b in zip(params.box_min, params.box_max)]
         self.t, self.dt_prev, self.first = 0.0, float(params.dt_first), True
         self.stats = {}
+        self.profile = None  # dict name -> seconds when set (synchronising section timer)
+        self._t_last = None
+
+    def _mark(self, name):
+        if self.profile is None:
+            return
+        import time
+        torch.cuda.synchronize(self.dev)
+        now = time.perf_counter()
+        if self._t_last is not None and name:
+            self.profile[name] = self.profile.get(name, 0.0) + now - self._t_last
+        self._t_last = now
 
     def _field(self, name, dtype=torch.float64):
         out = torch.empty(self.sim.n, dtype=dtype, device=self.dev)
@@ -207,6 +219,7 @@ class DistributedSim:
         rows = pack(st)
         parts = [rows[own == r] for r in range(comm.world)]
         local = unpack(torch.cat(comm.alltoallv(parts), 0))
+        self._mark("migrate")
         # 2. ghosts within 2 h_max of every other rank's domain box
         x = torch.stack([local["x"], local["y"], local["z"]], 1)
         hmax = comm.all_reduce(local["h"].max().reshape(1) if local["h"].numel() else
@@ -227,14 +240,17 @@ class DistributedSim:
         held = unpack(torch.cat([lrows] + list(recv), 0))
         self.stats = {"n_local": int(local["x"].numel()),
                       "n_ghost": int(sum(r.shape[0] for r in recv))}
+        self._mark("ghosts")
         # 3. the hot path with two halo refreshes
         self._load(held)
         sim.build_tree()
         sim.find_neighbors(stats=False)
         sim.density()
+        self._mark("tree2_nbr_density")
         ids_now = self._field("id", torch.int64)
         src_pos = [positions_of(ids_now, s) for s in sent_ids]        # my particles others hold
         dst_pos = [positions_of(ids_now, g) for g in ghost_ids]       # their particles I hold
+        self._mark("halo_maps")
         self._halo(["rho"], src_pos, dst_pos)
         sim.eos()
         if getattr(self.params, "gradh", 0):  # owners' Omega over the ghosts
@@ -249,6 +265,7 @@ class DistributedSim:
         sim.momentum_energy()
         if sim.stir_enabled:  # driving: every rank holds the same OU state and noise
             sim.stir()
+        self._mark("eos_iad_mom_halos")
         # 4. global dt, update, drop ghosts
         mhc = torch.tensor([sim.get_local_min_hc()], dtype=torch.float64, device=self.dev)
         mhc = comm.all_reduce(mhc, dist.ReduceOp.MIN if comm.world > 1 else None)
@@ -259,6 +276,7 @@ class DistributedSim:
         st = self._held_state()
         keep = (st["id"] & GHOST_BIT) == 0
         self.local = {k: v[keep].contiguous() for k, v in st.items()}
+        self._mark("dt_update_drop")
         return dt
 
     def _halo(self, names, src_pos, dst_pos):
