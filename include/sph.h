@@ -119,6 +119,7 @@ typedef enum sph_field {
   SPH_F_PHI,    /* gravitational potential (cfg.gravity; after sph_gravity)    */
   SPH_F_OMEGA,  /* grad-h factor Omega (cfg.gradh; valid after sph_gradh)        */
   SPH_F_VSIG,   /* signal velocity (cfg.dt_vsig; after sph_momentum_energy)    */
+  SPH_F_ORDER,  /* int32: pre-sort index of each position (after sph_build_tree) */
   SPH_NFIELDS
 } sph_field;
 
@@ -290,6 +291,42 @@ int sph_set_field(sph_ctx* ctx, int field, const void* src, int mem);
  * the next sph_timestep instead. */
 int sph_get_local_min_hc(sph_ctx* ctx, double* min_hc);
 int sph_set_global_min_hc(sph_ctx* ctx, double min_hc);
+
+/* Device-side plumbing of the decomposed step ("domain
+ * decomposition, halo exchanges", P:216 DomainDecompAndSync).  They move and
+ * select particles; none changes a value of the method.  All pointers are
+ * DEVICE pointers on cfg.device except `boxes`; indices refer to the current
+ * particle order.  A row is SPH_ROW_DOUBLES doubles
+ * {x, y, z, vx, vy, vz, h, m, u, du_m1, id (int64 bit pattern)}.
+ *
+ * sph_compute_keys: phase KEYS alone (box + Morton keys) in the CURRENT order,
+ *   no sort; SPH_F_KEY then returns them (the SFC partition reads them).
+ * sph_compact: stable in-place compaction keeping particle i iff
+ *   (keep == NULL || keep[i] != 0) && !(drop_ghosts && (id[i] & SPH_GHOST_BIT));
+ *   *n_out = new count.  Synchronises.
+ * sph_pack_rows: rows of particles idx[0..m) into dst [m][SPH_ROW_DOUBLES],
+ *   id OR-ed with or_id (SPH_GHOST_BIT marks ghosts).
+ * sph_append_rows: m rows after the current n particles (n + m <= n_capacity,
+ *   else SPH_ERR_CAPACITY).
+ * sph_select_ghosts: mask[i] bit r (r < R <= 64, r != self) set iff particle i
+ *   is closer than `radius` (minimum image on periodic axes) to the box
+ *   boxes[6r..6r+5] = {lo_x, lo_y, lo_z, hi_x, hi_y, hi_z} (host array) of rank r;
+ *   an empty box (lo > hi) selects nothing.
+ * sph_gather_field / sph_scatter_field: dst[k] = f[idx[k]] / f[idx[k]] = src[k]
+ *   for a double field; scatter follows sph_set_field's rules (settable fields
+ *   and stages) and also accepts SPH_F_OMEGA after sph_gradh.
+ * SPH_F_ORDER (int32, via sph_get_field): after sph_build_tree, the pre-sort
+ *   index of the particle now at each position (the sort's permutation).
+ * compact / append leave the context at the "particles set" stage. */
+#define SPH_ROW_DOUBLES 11
+int sph_compute_keys(sph_ctx* ctx);
+int sph_compact(sph_ctx* ctx, const uint8_t* keep, int drop_ghosts, int64_t* n_out);
+int sph_pack_rows(sph_ctx* ctx, const int64_t* idx, int64_t m, uint64_t or_id, double* dst);
+int sph_append_rows(sph_ctx* ctx, const double* rows, int64_t m);
+int sph_select_ghosts(sph_ctx* ctx, const double* boxes, int R, int self, double radius,
+                      uint64_t* mask);
+int sph_gather_field(sph_ctx* ctx, int field, const int64_t* idx, int64_t m, double* dst);
+int sph_scatter_field(sph_ctx* ctx, int field, const int64_t* idx, int64_t m, const double* src);
 
 /* --- the hot path (each call = one accounted phase group) ------------------- */
 

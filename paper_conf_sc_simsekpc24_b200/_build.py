@@ -12,7 +12,7 @@ CSRC = os.path.join(HERE, "csrc")
 LIBDIR = os.path.join(HERE, "lib")
 LIB = os.path.join(LIBDIR, "libsph.so")
 ROOT = os.path.dirname(HERE)
-SOURCES = ["api.cu", "k_keys.cu", "k_sort.cu", "k_neighbors.cu", "k_physics.cu", "k_stir.cu", "k_gravity.cu", "nvml_dyn.cpp"]
+SOURCES = ["api.cu", "k_keys.cu", "k_sort.cu", "k_neighbors.cu", "k_physics.cu", "k_stir.cu", "k_gravity.cu", "k_decomp.cu", "nvml_dyn.cpp"]
 HEADERS = ["sph_internal.cuh", "nvml_dyn.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

@@ -96,6 +96,8 @@ struct sph_ctx {
   unsigned current_lock = 0;
   bool locked_any = false;
   bool rec_m_dirty = false;
+  uint32_t* last_perm = nullptr;  // the last sort's permutation (SPH_F_ORDER)
+  int64_t* compact_scratch = nullptr;  // per-block counts of sph_compact (+ total)
   Stir stir{};          // turbulence driving (k_stir.cu)
   bool stir_on = false;
   // DVFS trace (sph_trace_start / sph_trace_stop)
@@ -307,6 +309,7 @@ int body_tree(sph_ctx* c) {
   cudaError_t e = launch_sort(F, c->keyA, c->keyB, c->valA, c->valB, c->sort_hist, c->sort_status,
                               c->status_bytes, &perm, &ksorted, c->st);
   if ((rc = cuda_check(c, e, "sort"))) return rc;
+  c->last_perm = perm;
   const int prv = c->cur;
   c->cur ^= 1;
   c->key_sorted = ksorted;
@@ -512,6 +515,8 @@ static size_t layout(const sph_config* cfg, char* base, sph_ctx* c) {
   char* hp = take(hb);
   char* sp = take(sb);
   char* dsp = take(sizeof(DevScalars));
+  char* csc = take(sizeof(int64_t) * ((cap + 1023) / 1024 + 2));
+  if (c) c->compact_scratch = (int64_t*)csc;
   const size_t sst = (size_t)cfg->stir_steps;
   char* sA = sst ? take(sizeof(double) * kStirModes * 6) : nullptr;
   char* sB = sst ? take(sizeof(double) * kStirModes * 6) : nullptr;
@@ -714,6 +719,11 @@ int sph_get_field(sph_ctx* c, int field, void* dst, int mem) {
     if (!c->vsig) return fail(c, SPH_ERR_ARG, "SPH_F_VSIG needs cfg.dt_vsig");
     src = c->vsig;
   }
+  else if (field == SPH_F_ORDER) {
+    if (!c->last_perm || c->stage < S_TREE) return fail(c, SPH_ERR_STATE, "SPH_F_ORDER needs sph_build_tree");
+    src = c->last_perm;
+    esz = 4;
+  }
   else return fail(c, SPH_ERR_ARG, "unknown field %d", field);
   if (c->n == 0) return SPH_OK;
   const cudaMemcpyKind kind = mem == SPH_MEM_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
@@ -788,6 +798,137 @@ int sph_set_global_min_hc(sph_ctx* c, double min_hc) {
   set_minhc_kernel<<<1, 1, 0, c->st>>>(c->ds, o);
   note_launch();
   return cuda_check(c, cudaSuccess, "set_minhc");
+}
+
+// ---------------------------------------------------------------- decomposition plumbing
+int sph_compute_keys(sph_ctx* c) {
+  int rc = check_ready(c, S_PART, "sph_compute_keys");
+  if (rc) return rc;
+  if ((rc = phase_begin(c, SPH_PHASE_KEYS))) return rc;
+  launch_reset_scalars(c->ds, c->P, c->st);
+  Fields F = fields(c);
+  F.key = c->keyA;
+  launch_box_keys(F, c->P, c->st);
+  c->key_sorted = c->keyA;  // keys of the current (unsorted) order
+  if ((rc = phase_end(c, SPH_PHASE_KEYS))) return rc;
+  c->stage = S_PART;
+  return SPH_OK;
+}
+
+int sph_compact(sph_ctx* c, const uint8_t* keep, int drop_ghosts, int64_t* n_out) {
+  int rc = check_ready(c, S_PART, "sph_compact");
+  if (rc) return rc;
+  const int nxt = c->cur ^ 1;
+  int64_t* total = c->compact_scratch + (c->cfg.n_capacity + 1023) / 1024 + 1;
+  rc = cuda_check(c, launch_compact(c->n, keep, drop_ghosts ? 1 : 0, c->state[c->cur], c->ids[c->cur],
+                                    c->state[nxt], c->ids[nxt], c->compact_scratch, total, c->st),
+                  "compact");
+  if (rc) return rc;
+  int64_t n = 0;
+  rc = cuda_check(c, cudaMemcpyAsync(&n, total, sizeof(int64_t), cudaMemcpyDeviceToHost, c->st), "copy");
+  if (!rc) rc = cuda_check(c, cudaStreamSynchronize(c->st), "sync");
+  if (rc) return rc;
+  c->cur = nxt;
+  c->n = n;
+  c->stage = S_PART;
+  if (n_out) *n_out = n;
+  return SPH_OK;
+}
+
+int sph_pack_rows(sph_ctx* c, const int64_t* idx, int64_t m, uint64_t or_id, double* dst) {
+  int rc = check_ready(c, S_PART, "sph_pack_rows");
+  if (rc) return rc;
+  if (m < 0 || (m > 0 && (!idx || !dst))) return fail(c, SPH_ERR_ARG, "bad idx/dst");
+  return cuda_check(c, launch_pack_rows(m, idx, c->state[c->cur], c->ids[c->cur], or_id, dst, c->st), "pack");
+}
+
+int sph_append_rows(sph_ctx* c, const double* rows, int64_t m) {
+  int rc = check_ready(c, S_PART, "sph_append_rows");
+  if (rc) return rc;
+  if (m < 0 || (m > 0 && !rows)) return fail(c, SPH_ERR_ARG, "bad rows");
+  if (c->n + m > c->cfg.n_capacity)
+    return fail(c, SPH_ERR_CAPACITY, "n + m = %lld exceeds n_capacity %lld", (long long)(c->n + m), (long long)c->cfg.n_capacity);
+  rc = cuda_check(c, launch_append_rows(m, c->n, rows, c->state[c->cur], c->ids[c->cur], c->st), "append");
+  if (rc) return rc;
+  c->n += m;
+  c->stage = S_PART;
+  return SPH_OK;
+}
+
+int sph_select_ghosts(sph_ctx* c, const double* boxes, int R, int self, double radius, uint64_t* mask) {
+  int rc = check_ready(c, S_PART, "sph_select_ghosts");
+  if (rc) return rc;
+  if (R < 1 || R > kMaxGhostRanks || !boxes || (c->n > 0 && !mask)) return fail(c, SPH_ERR_ARG, "bad boxes/R/mask");
+  double L[3];
+  int per[3];
+  for (int a = 0; a < 3; ++a) {
+    L[a] = c->cfg.box_max[a] - c->cfg.box_min[a];
+    per[a] = c->cfg.periodic[a];
+  }
+  return cuda_check(c, launch_select_ghosts(c->n, c->state[c->cur], boxes, R, self, radius, L, per, mask, c->st),
+                    "select ghosts");
+}
+
+static double* double_field(sph_ctx* c, int field) {
+  if (field >= SPH_F_X && field <= SPH_F_DU_M1) return c->state[c->cur][field - SPH_F_X];
+  switch (field) {
+    case SPH_F_RHO: return c->rho;
+    case SPH_F_P: return c->p;
+    case SPH_F_C: return c->c;
+    case SPH_F_C11: case SPH_F_C12: case SPH_F_C13: case SPH_F_C22: case SPH_F_C23: case SPH_F_C33:
+      return c->C[field - SPH_F_C11];
+    case SPH_F_AX: return c->ax;
+    case SPH_F_AY: return c->ay;
+    case SPH_F_AZ: return c->az;
+    case SPH_F_DU: return c->du;
+    case SPH_F_DIVV: return c->divv;
+    case SPH_F_CURLX: case SPH_F_CURLY: case SPH_F_CURLZ: return c->curl[field - SPH_F_CURLX];
+    case SPH_F_BAL: return c->bal;
+    case SPH_F_PHI: return c->phi;
+    case SPH_F_OMEGA: return c->omega;
+    case SPH_F_VSIG: return c->vsig;
+    default: return nullptr;
+  }
+}
+
+int sph_gather_field(sph_ctx* c, int field, const int64_t* idx, int64_t m, double* dst) {
+  int rc = check_ready(c, S_INIT, "sph_gather_field");
+  if (rc) return rc;
+  double* f = double_field(c, field);
+  if (!f) return fail(c, SPH_ERR_ARG, "field %d is not a double field of this configuration", field);
+  if (m < 0 || (m > 0 && (!idx || !dst))) return fail(c, SPH_ERR_ARG, "bad idx/dst");
+  return cuda_check(c, launch_gather_field(m, idx, f, dst, c->st), "gather");
+}
+
+int sph_scatter_field(sph_ctx* c, int field, const int64_t* idx, int64_t m, const double* src) {
+  int rc = check_ready(c, S_INIT, "sph_scatter_field");
+  if (rc) return rc;
+  if (m < 0 || (m > 0 && (!idx || !src))) return fail(c, SPH_ERR_ARG, "bad idx/src");
+  double* f = nullptr;
+  bool prho2 = false;
+  if (field == SPH_F_RHO) {
+    if (c->stage < S_DENS) return fail(c, SPH_ERR_STATE, "scatter(RHO) before sph_density");
+    f = c->rho;
+  } else if (field >= SPH_F_C11 && field <= SPH_F_C33) {
+    if (c->stage < S_IAD) return fail(c, SPH_ERR_STATE, "scatter(C) before sph_iad");
+    f = c->C[field - SPH_F_C11];
+    c->rec_m_dirty = true;
+  } else if (field == SPH_F_BAL && c->P.av_switch) {
+    if (c->stage < S_IAD) return fail(c, SPH_ERR_STATE, "scatter(BAL) before sph_iad");
+    f = c->bal;
+    c->rec_m_dirty = true;
+  } else if (field == SPH_F_OMEGA && c->omega) {
+    if (!c->gradh_done || c->stage != S_EOS)
+      return fail(c, SPH_ERR_STATE, "scatter(OMEGA) must follow sph_gradh, before sph_iad");
+    f = c->omega;
+    prho2 = true;
+  } else {
+    return fail(c, SPH_ERR_ARG, "field %d is not settable", field);
+  }
+  rc = cuda_check(c, launch_scatter_field(m, idx, src, f, c->st), "scatter");
+  if (rc || !prho2) return rc;
+  launch_prho2(fields(c), c->st);
+  return cuda_check(c, cudaGetLastError(), "prho2");
 }
 
 int sph_build_tree(sph_ctx* c) {

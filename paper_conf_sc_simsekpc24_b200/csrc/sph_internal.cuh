@@ -262,6 +262,21 @@ void launch_density(const Fields& F, const Params& P, cudaStream_t st);
 void launch_eos(const Fields& F, const Params& P, cudaStream_t st);
 void launch_iad(const Fields& F, const Params& P, cudaStream_t st);
 void launch_gradh(const Fields& F, const Params& P, cudaStream_t st);
+// decomposition plumbing (k_decomp.cu)
+constexpr int kRowDoubles = 11;     // SPH_ROW_DOUBLES
+constexpr int kMaxGhostRanks = 64;
+cudaError_t launch_compact(int64_t n, const uint8_t* keep, int drop, double* const* src, const int64_t* id_src,
+                           double* const* dst, int64_t* id_dst, int64_t* scratch, int64_t* total,
+                           cudaStream_t st);
+cudaError_t launch_pack_rows(int64_t m, const int64_t* idx, double* const* src, const int64_t* id,
+                             uint64_t or_id, double* dst, cudaStream_t st);
+cudaError_t launch_append_rows(int64_t m, int64_t n0, const double* rows, double* const* dst, int64_t* id,
+                               cudaStream_t st);
+cudaError_t launch_select_ghosts(int64_t n, double* const* f, const double* boxes, int R, int self,
+                                 double radius, const double L[3], const int per[3], uint64_t* mask,
+                                 cudaStream_t st);
+cudaError_t launch_gather_field(int64_t m, const int64_t* idx, const double* f, double* dst, cudaStream_t st);
+cudaError_t launch_scatter_field(int64_t m, const int64_t* idx, const double* src, double* f, cudaStream_t st);
 void launch_prho2(const Fields& F, cudaStream_t st);
 void launch_momentum_energy(const Fields& F, const Params& P, cudaStream_t st);
 void launch_timestep(const Fields& F, const Params& P, cudaStream_t st);

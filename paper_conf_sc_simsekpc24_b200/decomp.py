@@ -13,7 +13,9 @@ curve; the split points come from a global histogram of the top key bits
   3. the full hot path in libsph on locals + ghosts, with two halo refreshes of
      the owners' values over the ghosts: rho after DENSITY (then EOS derives
      p, c, V) and C after IAD (H2, H3 of SURVEY 8(e));
-  4. dt = global min over ranks (all-reduce), update, ghosts dropped.
+  4. dt = global min over ranks (all-reduce), update; the ghosts are dropped
+     (sph_compact) at the start of the next step.
+The particles stay in libsph; only emigrants, ghosts and halo values move.
 
 The held set is sorted in the global Morton order and every target's
 neighbours are the same particles as in a single-GPU run, so for a periodic box
@@ -167,21 +169,43 @@ def positions_of(ids_current, query):
 # ----------------------------------------------------------------------------- stepping
 class DistributedSim:
     """One rank of the decomposed simulation.  `state` holds this rank's share of
-    the particles (torch tensors on its GPU)."""
+    the particles.  The particles stay resident in libsph between steps; only
+    emigrants, ghosts and halo values travel, packed and unpacked by libsph's
+    device plumbing (sph_compact / sph_pack_rows / sph_append_rows /
+    sph_select_ghosts / sph_gather_field / sph_scatter_field).  All torch work
+    runs on the libsph stream, so the two never need cross-stream ordering."""
 
-    def __init__(self, params, state, n_capacity: int, device: int = 0, **kw):
+    def __init__(self, params, state, n_capacity: int, device: int = 0, force_exchange: bool = False,
+                 **kw):
         from . import sph
         self.sph = sph
+        # force_exchange: run the partition / migration / ghost / halo plumbing even
+        # on one rank (it then moves nothing) -- measures its cost (tools/decomp_probe.py)
+        self.xchg = force_exchange
         self.params = params
         self.comm = Comm()
         self.dev = torch.device("cuda", device)
         self.sim = sph.Simulation(params, n_capacity=n_capacity, device=device, **kw)
-        self.local = {k: torch.as_tensor(np.ascontiguousarray(v)).to(self.dev) for k, v in state.items()}
         self.box_len = [float(b - a) for a, b in zip(params.box_min, params.box_max)]
         self.t, self.dt_prev, self.first = 0.0, float(params.dt_first), True
         self.stats = {}
         self.profile = None  # dict name -> seconds when set (synchronising section timer)
         self._t_last = None
+        self.local = {k: torch.as_tensor(np.ascontiguousarray(v)) for k, v in state.items()}
+
+    # the local (owned) particles: uploading replaces the held set
+    @property
+    def local(self):
+        st = self._held_state()
+        keep = (st["id"] & GHOST_BIT) == 0
+        return {k: v[keep].contiguous() for k, v in st.items()}
+
+    @local.setter
+    def local(self, st):
+        with torch.cuda.stream(self.sim.stream):
+            self.sim.set_particles({k: st[k].to(self.dev).contiguous() for k in STATE + ("id",)})
+        self.sim.set_time(self.t, self.dt_prev, self.first)
+        self.has_ghosts = False
 
     def _mark(self, name):
         if self.profile is None:
@@ -203,96 +227,118 @@ class DistributedSim:
         st["id"] = self._field("id", torch.int64)
         return st
 
-    def _load(self, st):
-        self.sim.set_particles({k: st[k].contiguous() for k in STATE + ("id",)})
-        self.sim.set_time(self.t, self.dt_prev, self.first)
-
     def step(self):
+        with torch.cuda.stream(self.sim.stream):
+            return self._step()
+
+    def _exchange_rows(self, idx, dest, or_id=0):
+        """Rows of the particles idx (current order) to ranks dest; returns the
+        received rows (cat, in source-rank order) and the per-source counts."""
+        world = self.comm.world
+        order = torch.argsort(dest, stable=True)
+        idx = idx[order]
+        counts = torch.bincount(dest, minlength=world).cpu().tolist()
+        rows = self.sim.pack_rows(idx, or_id)
+        recv = self.comm.alltoallv(list(torch.split(rows, counts, 0)))
+        return torch.cat(recv, 0), [int(r.shape[0]) for r in recv], idx, counts
+
+    def _step(self):
         comm, sim = self.comm, self.sim
-        # 1. keys of the locals, SFC partition, migration
-        self._load(self.local)
+        world, rank = comm.world, comm.rank
+        xchg = world > 1 or self.xchg
+        self._mark(None)
+        if xchg:
+            # 1. drop last step's ghosts; keys in the current order; SFC partition
+            if self.has_ghosts:
+                sim.compact(drop_ghosts=True)
+            sim.compute_keys()
+            keys = self._field("key", torch.int64)
+            splits = sfc_splits(keys, comm)
+            own = owners(keys, splits)
+            self._mark("keys_partition")
+            # migration: particles whose key left this rank's range
+            emig = own != rank
+            eidx = torch.nonzero(emig).flatten()
+            rows, _, _, _ = self._exchange_rows(eidx, own[eidx])
+            sim.compact(keep=~emig)
+            sim.append_rows(rows)
+            self._mark("migrate")
+            # 2. ghosts within 2 h_max of every other rank's domain box
+            x = torch.stack([self._field("x"), self._field("y"), self._field("z")], 1)
+            hl = self._field("h")
+            hmax = comm.all_reduce(hl.max().reshape(1) if hl.numel() else
+                                   torch.zeros(1, dtype=torch.float64, device=self.dev),
+                                   dist.ReduceOp.MAX if world > 1 else None)
+            boxes = domain_boxes(x, comm)
+            radius = float(2.0 * hmax.item()) * (1.0 + 1e-9)
+            mask = sim.select_ghosts(boxes.reshape(world, 6).cpu().numpy(), rank, radius)
+            gidx, gdest = [], []
+            for r in range(world):
+                if r == rank:
+                    continue
+                ir = torch.nonzero((mask >> r) & 1).flatten()
+                gidx.append(ir)
+                gdest.append(torch.full_like(ir, r))
+            e = torch.zeros(0, dtype=torch.int64, device=self.dev)
+            gidx, gdest = torch.cat(gidx + [e]), torch.cat(gdest + [e])
+            grows, gcounts, sent_idx, scounts = self._exchange_rows(gidx, gdest, GHOST_BIT)
+            n_loc = sim.n
+            sim.append_rows(grows)
+            self.has_ghosts = True
+            self.stats = {"n_local": n_loc, "n_ghost": int(sum(gcounts))}
+            self._mark("ghosts")
+        # 3. the hot path with the halo refreshes
         sim.build_tree()
-        st = self._held_state()
-        keys = self._field("key", torch.int64)
-        splits = sfc_splits(keys, comm)
-        own = owners(keys, splits)
-        rows = pack(st)
-        parts = [rows[own == r] for r in range(comm.world)]
-        local = unpack(torch.cat(comm.alltoallv(parts), 0))
-        self._mark("migrate")
-        # 2. ghosts within 2 h_max of every other rank's domain box
-        x = torch.stack([local["x"], local["y"], local["z"]], 1)
-        hmax = comm.all_reduce(local["h"].max().reshape(1) if local["h"].numel() else
-                               torch.zeros(1, dtype=torch.float64, device=self.dev),
-                               dist.ReduceOp.MAX if comm.world > 1 else None)
-        boxes = domain_boxes(x, comm)
-        radius = float(2.0 * hmax.item()) * (1.0 + 1e-9)
-        masks = ghost_masks(x, boxes, comm.rank, radius, self.box_len, self.params.periodic)
-        lrows = pack(local)
-        sent_ids = [local["id"][m] for m in masks]
-        gparts = []
-        for m in masks:
-            g = lrows[m].clone()
-            g[:, len(STATE)] = (local["id"][m] | GHOST_BIT).view(torch.float64)
-            gparts.append(g)
-        recv = comm.alltoallv(gparts)
-        ghost_ids = [unpack(r)["id"] for r in recv]
-        held = unpack(torch.cat([lrows] + list(recv), 0))
-        self.stats = {"n_local": int(local["x"].numel()),
-                      "n_ghost": int(sum(r.shape[0] for r in recv))}
-        self._mark("ghosts")
-        # 3. the hot path with two halo refreshes
-        self._load(held)
-        sim.build_tree()
+        if xchg:
+            order = self._field("order", torch.int32).to(torch.int64)
+            inv = torch.empty_like(order)
+            inv[order] = torch.arange(order.numel(), device=self.dev)
+            self._src = torch.split(inv[sent_idx], scounts, 0)              # mine others hold
+            self._dst = inv[n_loc:n_loc + sum(gcounts)]                      # theirs I hold
+            self._mark("tree_maps")
         sim.find_neighbors(stats=False)
         sim.density()
-        self._mark("tree2_nbr_density")
-        ids_now = self._field("id", torch.int64)
-        src_pos = [positions_of(ids_now, s) for s in sent_ids]        # my particles others hold
-        dst_pos = [positions_of(ids_now, g) for g in ghost_ids]       # their particles I hold
-        self._mark("halo_maps")
-        self._halo(["rho"], src_pos, dst_pos)
+        self._halo(["rho"])
         sim.eos()
         if getattr(self.params, "gradh", 0):  # owners' Omega over the ghosts
             sim.gradh()
-            self._halo(["omega"], src_pos, dst_pos)
+            self._halo(["omega"])
         sim.iad()
         # H3: the owners' C (and Balsara factors when the AV switch is on)
         h3 = ["c11", "c12", "c13", "c22", "c23", "c33"]
         if getattr(self.params, "av_switch", 0):
             h3.append("bal")
-        self._halo(h3, src_pos, dst_pos)
+        self._halo(h3)
         sim.momentum_energy()
         if sim.stir_enabled:  # driving: every rank holds the same OU state and noise
             sim.stir()
-        self._mark("eos_iad_mom_halos")
-        # 4. global dt, update, drop ghosts
-        mhc = torch.tensor([sim.get_local_min_hc()], dtype=torch.float64, device=self.dev)
-        mhc = comm.all_reduce(mhc, dist.ReduceOp.MIN if comm.world > 1 else None)
-        sim.set_global_min_hc(float(mhc.item()))
+        self._mark("physics_halos")
+        # 4. global dt, update (ghosts are dropped at the next step)
+        if xchg:
+            mhc = torch.tensor([sim.get_local_min_hc()], dtype=torch.float64, device=self.dev)
+            mhc = comm.all_reduce(mhc, dist.ReduceOp.MIN if world > 1 else None)
+            sim.set_global_min_hc(float(mhc.item()))
         dt = sim.timestep()
         sim.update()
         self.t, self.dt_prev, self.first = self.t + dt, dt, False
-        st = self._held_state()
-        keep = (st["id"] & GHOST_BIT) == 0
-        self.local = {k: v[keep].contiguous() for k, v in st.items()}
-        self._mark("dt_update_drop")
+        self._mark("dt_update")
         return dt
 
-    def _halo(self, names, src_pos, dst_pos):
-        if self.comm.world == 1:
+    def _halo(self, names):
+        if not (self.comm.world > 1 or self.xchg):
             return
-        vals = {k: self._field(k) for k in names}
-        parts = [torch.stack([vals[k][p] for k in names], 1) for p in src_pos]
-        recv = self.comm.alltoallv(parts)
-        for r, (rv, p) in enumerate(zip(recv, dst_pos)):
-            for c, k in enumerate(names):
-                vals[k][p] = rv[:, c]
-        for k in names:
-            self.sim.set_field(k, vals[k])
+        sim = self.sim
+        parts = [torch.stack([sim.gather_field(k, p) for k in names], 1) for p in self._src]
+        recv = torch.cat(self.comm.alltoallv(parts), 0)
+        for c, k in enumerate(names):
+            sim.scatter_field(k, self._dst, recv[:, c].contiguous())
 
     def gather_state(self):
         """All particles on every rank, sorted by id (host numpy) -- for tests."""
+        with torch.cuda.stream(self.sim.stream):
+            return self._gather_state()
+
+    def _gather_state(self):
         rows = pack(self.local)
         n = torch.tensor([rows.shape[0]], dtype=torch.int64, device=self.dev)
         ns = [int(v.item()) for v in self.comm.all_gather(n)]

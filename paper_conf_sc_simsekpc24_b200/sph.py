@@ -26,9 +26,10 @@ STIR_NMODES = 61
 NPHASES = len(PHASES)
 FIELDS = ("x", "y", "z", "vx", "vy", "vz", "h", "m", "u", "du_m1", "id", "key", "nc", "rho", "p",
           "c", "c11", "c12", "c13", "c22", "c23", "c33", "ax", "ay", "az", "du", "divv", "curlx",
-          "curly", "curlz", "bal", "phi", "omega", "vsig")
+          "curly", "curlz", "bal", "phi", "omega", "vsig", "order")
 FIELD_ID = {name: k for k, name in enumerate(FIELDS)}
-FIELD_DTYPE = {"id": np.int64, "key": np.uint64, "nc": np.int32}
+FIELD_DTYPE = {"id": np.int64, "key": np.uint64, "nc": np.int32, "order": np.int32}
+ROW_DOUBLES = 11  # SPH_ROW_DOUBLES: x y z vx vy vz h m u du_m1 id(bits)
 MEM_HOST, MEM_DEVICE = 0, 1
 ACCOUNTING_OFF, ACCOUNTING_PHASE = 0, 1
 CLOCK_DEFAULT, CLOCK_STATIC, CLOCK_PER_PHASE = 0, 1, 2
@@ -94,7 +95,9 @@ EXPORTS = ("sph_config_default", "sph_workspace_size", "sph_init", "sph_finalize
            "sph_set_accounting", "sph_kernel_launches", "sph_set_field",
            "sph_get_local_min_hc", "sph_set_global_min_hc", "sph_get_neighbor_rows",
            "sph_trace_start", "sph_trace_stop", "sph_stir_modes", "sph_stir_init", "sph_stir",
-           "sph_stir_get_state", "sph_supported_clocks", "sph_gravity", "sph_gradh")
+           "sph_stir_get_state", "sph_supported_clocks", "sph_gravity", "sph_gradh",
+           "sph_compute_keys", "sph_compact", "sph_pack_rows", "sph_append_rows",
+           "sph_select_ghosts", "sph_gather_field", "sph_scatter_field")
 GHOST_BIT = 1 << 62
 
 _lib = None
@@ -149,6 +152,13 @@ def load(build_if_missing: bool = True):
     L.sph_stir.argtypes = [P]
     L.sph_gravity.argtypes = [P]
     L.sph_gradh.argtypes = [P]
+    L.sph_compute_keys.argtypes = [P]
+    L.sph_compact.argtypes = [P, V, I, C.POINTER(I64)]
+    L.sph_pack_rows.argtypes = [P, V, I64, C.c_uint64, V]
+    L.sph_append_rows.argtypes = [P, V, I64]
+    L.sph_select_ghosts.argtypes = [P, V, I, I, D, V]
+    L.sph_gather_field.argtypes = [P, I, V, I64, V]
+    L.sph_scatter_field.argtypes = [P, I, V, I64, V]
     L.sph_stir_get_state.argtypes = [P, V, C.POINTER(I64)]
     L.sph_supported_clocks.argtypes = [P, V, I, C.POINTER(I)]
     L.sph_trace_start.argtypes = [P, D, I64]
@@ -316,6 +326,59 @@ class Simulation:
             self.stream.wait_stream(self.torch.cuda.current_stream(self.device))
         self._keep_field = src
         self._ok(self.L.sph_set_field(self.ctx, FIELD_ID[name], C.c_void_p(p), mem))
+
+    # ------------------------------------------------ decomposition plumbing (8(e))
+    # Device tensors in/out; callers run their torch work on self.stream (the
+    # libsph stream) so that no cross-stream ordering is needed.
+    def compute_keys(self):
+        self._ok(self.L.sph_compute_keys(self.ctx))
+
+    def compact(self, keep=None, drop_ghosts: bool = False) -> int:
+        """Stable compaction (keep: cuda uint8/bool tensor [n] or None)."""
+        n = C.c_int64()
+        kp = None if keep is None else C.c_void_p(keep.to(self.torch.uint8).contiguous().data_ptr())
+        self._keep_field = keep
+        self._ok(self.L.sph_compact(self.ctx, kp, 1 if drop_ghosts else 0, C.byref(n)))
+        self.n = int(n.value)
+        return self.n
+
+    def pack_rows(self, idx, or_id: int = 0):
+        """Rows [m, ROW_DOUBLES] (cuda float64) of the particles at idx (cuda int64)."""
+        idx = idx.to(self.torch.int64).contiguous()
+        out = self.torch.empty((idx.numel(), ROW_DOUBLES), dtype=self.torch.float64, device=self.device)
+        self._ok(self.L.sph_pack_rows(self.ctx, C.c_void_p(idx.data_ptr()), idx.numel(),
+                                      C.c_uint64(or_id), C.c_void_p(out.data_ptr())))
+        self._keep_field = (idx, out)
+        return out
+
+    def append_rows(self, rows):
+        rows = rows.contiguous()
+        self._keep_field = rows
+        self._ok(self.L.sph_append_rows(self.ctx, C.c_void_p(rows.data_ptr()), rows.shape[0]))
+        self.n += int(rows.shape[0])
+
+    def select_ghosts(self, boxes, self_rank: int, radius: float):
+        """int64 cuda tensor [n]: bit r set iff the particle is within radius of rank r's box."""
+        b = np.ascontiguousarray(boxes, dtype=np.float64).reshape(-1, 6)
+        mask = self.torch.empty(self.n, dtype=self.torch.int64, device=self.device)
+        self._ok(self.L.sph_select_ghosts(self.ctx, C.c_void_p(b.ctypes.data), b.shape[0], int(self_rank),
+                                          float(radius), C.c_void_p(mask.data_ptr())))
+        return mask
+
+    def gather_field(self, name: str, idx):
+        idx = idx.to(self.torch.int64).contiguous()
+        out = self.torch.empty(idx.numel(), dtype=self.torch.float64, device=self.device)
+        self._ok(self.L.sph_gather_field(self.ctx, FIELD_ID[name], C.c_void_p(idx.data_ptr()), idx.numel(),
+                                         C.c_void_p(out.data_ptr())))
+        self._keep_field = idx
+        return out
+
+    def scatter_field(self, name: str, idx, src):
+        idx = idx.to(self.torch.int64).contiguous()
+        src = src.to(self.torch.float64).contiguous()
+        self._keep_field = (idx, src)
+        self._ok(self.L.sph_scatter_field(self.ctx, FIELD_ID[name], C.c_void_p(idx.data_ptr()), idx.numel(),
+                                          C.c_void_p(src.data_ptr())))
 
     def get_local_min_hc(self) -> float:
         v = C.c_double()
