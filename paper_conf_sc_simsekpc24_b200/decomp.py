@@ -202,6 +202,8 @@ class DistributedSim:
 
     @local.setter
     def local(self, st):
+        # the caller may have produced st on its own stream (e.g. async H2D copies)
+        self.sim.stream.wait_stream(torch.cuda.current_stream(self.dev))
         with torch.cuda.stream(self.sim.stream):
             self.sim.set_particles({k: st[k].to(self.dev).contiguous() for k in STATE + ("id",)})
         self.sim.set_time(self.t, self.dt_prev, self.first)
@@ -228,8 +230,12 @@ class DistributedSim:
         return st
 
     def step(self):
+        caller = torch.cuda.current_stream(self.dev)
+        self.sim.stream.wait_stream(caller)
         with torch.cuda.stream(self.sim.stream):
-            return self._step()
+            dt = self._step()
+        caller.wait_stream(self.sim.stream)  # the caller's later work (events, copies) follows the step
+        return dt
 
     def _exchange_rows(self, idx, dest, or_id=0):
         """Rows of the particles idx (current order) to ranks dest; returns the
