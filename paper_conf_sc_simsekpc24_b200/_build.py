@@ -18,6 +18,8 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O2", "--expt-relaxed-constexpr",
          "-I", os.path.join(ROOT, "include")]
+# experiments only (e.g. SPH_NVCC_EXTRA="-DMOM_THREADS=384"); empty for the product build
+FLAGS += os.environ.get("SPH_NVCC_EXTRA", "").split()
 
 
 def _inputs():
