@@ -198,11 +198,13 @@ def measure_energy(sim, sph, n, args, gpu_index):
     sim.find_neighbors(stats=False)
     sim.density()
     sim.eos()
+    if sim.cfg.gradh:
+        sim.gradh()
     sim.iad()
     sim.momentum_energy()
     sim.timestep()
-    for ph in ("keys", "sort", "cells", "neighbors", "density", "eos", "iad", "momentum_energy",
-               "timestep"):
+    for ph in ("keys", "sort", "cells", "neighbors", "density", "eos") + (("gradh",) if sim.cfg.gradh else ()) + (
+            "iad", "momentum_energy", "timestep"):
         ms1, _ = sim.repeat_phase(ph, 3)
         reps = int(min(200000, max(5, 1500.0 / max(ms1, 1e-4))))
         with ClockSampler(gpu_index) as c2:
