@@ -164,33 +164,45 @@ __global__ void __launch_bounds__(256) eos_kernel(Fields F, Params P) {
 // ------------------------------------------------------------------ GRADH
 // NormalizationGradh (reading 21): Omega_i = 1 + (h_i/(3 rho_i)) sum_j m_j dW/dh,
 // dW/dh = -(K/h^4) S^5 (6 cos x - 3 S), x = pi r/2h, self term 3 m_i inside the
-// bracket.  sin and cos of pi*r/2h come from one sincospi; then
-// p/rho^2 -> p/(Omega rho^2) for the momentum records (written by IAD).
-// Per pair: one 32-B record {x, y, z, m} (the density record).
+// bracket.  S and cos x are polynomials in t = x^2 = r^2 (pi/2h)^2 (no sqrt,
+// sin or cos per pair); then p/rho^2 -> p/(Omega rho^2) for the momentum
+// records (written by IAD).  Per pair: one 32-B record {x, y, z, m} (the
+// density record), two neighbours per iteration like DENSITY.
+__device__ __forceinline__ double dwdh_term(double t) {
+  const double S = sinc_t(t), S2 = S * S;
+  return (S2 * S2 * S) * fma(6.0, cos_t(t), -3.0 * S);
+}
+
 template <bool kWrap>
 __device__ __forceinline__ void gradh_body(const Fields& F, const Params& P, const Geom& g, int64_t i,
                                            const Rec4& me, double hi) {
   const int nci = min(F.nc[i], F.ngmax);
-  const double inv2h = 0.5 / hi;
+  const double q = F.wq[i];
   double sum = 3.0 * me.d;  // self: S = 1, cos = 1
   const int32_t* __restrict__ nb = F.nbr + i;
   const Rec4* __restrict__ rec = F.rec_d;
   const int64_t cap = F.cap;
-  int jn = nci > 0 ? __ldg(nb) : 0;
-  Rec4 ra = ldg4(rec + jn);
-  jn = nci > 1 ? __ldg(nb + cap) : 0;
-  for (int k = 0; k < nci; ++k) {
-    const Rec4 rj = ra;
-    if (k + 1 < nci) ra = ldg4(rec + jn);
-    if (k + 2 < nci) jn = __ldg(nb + (int64_t)(k + 2) * cap);
+  Rec4 ra = ldg4(rec + (nci > 0 ? __ldg(nb) : 0)), rb = ldg4(rec + (nci > 1 ? __ldg(nb + cap) : 0));
+  int jc = nci > 2 ? __ldg(nb + 2 * cap) : 0, jd = nci > 3 ? __ldg(nb + 3 * cap) : 0;
+  int k = 0;
+  for (; k + 1 < nci; k += 2) {
+    const Rec4 a = ra, b = rb;
+    if (k + 2 < nci) ra = ldg4(rec + jc);
+    if (k + 3 < nci) rb = ldg4(rec + jd);
+    if (k + 4 < nci) jc = __ldg(nb + (int64_t)(k + 4) * cap);
+    if (k + 5 < nci) jd = __ldg(nb + (int64_t)(k + 5) * cap);
+    double dxa, dya, dza, dxb, dyb, dzb;
+    pair_d<kWrap>(g, me.a, me.b, me.c, a.a, a.b, a.c, dxa, dya, dza);
+    pair_d<kWrap>(g, me.a, me.b, me.c, b.a, b.b, b.c, dxb, dyb, dzb);
+    const double ta = dwdh_term((dxa * dxa + dya * dya + dza * dza) * q);
+    const double tb = dwdh_term((dxb * dxb + dyb * dyb + dzb * dzb) * q);
+    sum = fma(a.d, ta, sum);
+    sum = fma(b.d, tb, sum);
+  }
+  if (k < nci) {
     double dx, dy, dz;
-    pair_d<kWrap>(g, me.a, me.b, me.c, rj.a, rj.b, rj.c, dx, dy, dz);
-    const double y = sqrt(dx * dx + dy * dy + dz * dz) * inv2h;  // x = pi y
-    double sn, cs;
-    sincospi(y, &sn, &cs);
-    const double S = y > 0.0 ? sn / (kPi * y) : 1.0;
-    const double S2 = S * S;
-    sum = fma(rj.d * (S2 * S2 * S), 6.0 * cs - 3.0 * S, sum);
+    pair_d<kWrap>(g, me.a, me.b, me.c, ra.a, ra.b, ra.c, dx, dy, dz);
+    sum = fma(ra.d, dwdh_term((dx * dx + dy * dy + dz * dz) * q), sum);
   }
   const double rho = F.rho[i];
   const double h2 = hi * hi;
@@ -200,7 +212,7 @@ __device__ __forceinline__ void gradh_body(const Fields& F, const Params& P, con
   F.prho2[i] = __ddiv_rn(F.p[i], __dmul_rn(__dmul_rn(rho, rho), om));
 }
 
-__global__ void __launch_bounds__(256) gradh_kernel(Fields F, Params P) {
+__global__ void __launch_bounds__(kDensThreads, 1024 / kDensThreads) gradh_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= F.n) return;
   const Geom g = load_geom(F.ds, P);
@@ -607,7 +619,7 @@ void launch_iad(const Fields& F, const Params& P, cudaStream_t st) {
 }
 void launch_gradh(const Fields& F, const Params& P, cudaStream_t st) {
   if (F.n == 0) return;
-  gradh_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F, P);
+  gradh_kernel<<<(unsigned)div_up(F.n, kDensThreads), kDensThreads, 0, st>>>(F, P);
   note_launch();
 }
 void launch_prho2(const Fields& F, cudaStream_t st) {

@@ -215,6 +215,25 @@ __device__ __forceinline__ double sinc_t(double t) {
   return s;
 }
 
+// cos(x) for x^2 = t in [0, pi^2]: degree-11 polynomial in t interpolating
+// cos(sqrt t) at the 12 Chebyshev nodes (tools/sinc_fit.py); max abs error
+// 7.8e-16.  Used by the grad-h kernel derivative.
+__device__ __forceinline__ double cos_t(double t) {
+  double s = -7.989706279341135e-22;
+  s = fma(s, t, 4.087216582195389e-19);
+  s = fma(s, t, -1.561579798047433e-16);
+  s = fma(s, t, 4.779445319504966e-14);
+  s = fma(s, t, -1.1470743608679213e-11);
+  s = fma(s, t, 2.0876756905345936e-09);
+  s = fma(s, t, -2.7557319221730827e-07);
+  s = fma(s, t, 2.4801587301548223e-05);
+  s = fma(s, t, -0.0013888888888888488);
+  s = fma(s, t, 0.041666666666666644);
+  s = fma(s, t, -0.5);
+  s = fma(s, t, 1.0);
+  return s;
+}
+
 // S^6 for the kernel: W = (K/h^3) * S(pi r / 2h)^6, t = r^2 * (pi/2h)^2.
 __device__ __forceinline__ double sinc6_t(double t) {
   double s = sinc_t(t);

@@ -19,22 +19,33 @@ def S(t):
     return mp.sin(r) / r
 
 
-def fit(deg):
+def Ct(t):
+    """cos(sqrt t): the grad-h kernel derivative (k_physics.cu gradh_body)."""
+    return mp.cos(mp.sqrt(mp.mpf(t)))
+
+
+def fit(deg, f=S):
     N = deg + 1
     nodes = [T / 2 * (1 + mp.cos(mp.pi * (2 * k + 1) / (2 * N))) for k in range(N)]
     A = mp.matrix([[x ** p for p in range(N)] for x in nodes])
-    c = mp.lu_solve(A, mp.matrix([S(x) for x in nodes]))
+    c = mp.lu_solve(A, mp.matrix([f(x) for x in nodes]))
     return [float(c[p]) for p in range(N)]
 
 
-if __name__ == "__main__":
-    coef = fit(10)
+def report(coef, f):
     err = 0.0
     for t in np.linspace(0, float(T), 20001):
         s = coef[-1]
         for p in range(len(coef) - 2, -1, -1):
             s = s * t + coef[p]
-        err = max(err, abs(s - float(S(t))))
+        err = max(err, abs(s - float(f(t))))
     for p in range(len(coef) - 1, -1, -1):
         print(p, repr(coef[p]))
     print("max abs error", err)
+
+
+if __name__ == "__main__":
+    print("sin(x)/x, x^2 = t:")
+    report(fit(10), S)
+    print("cos(x), x^2 = t:")
+    report(fit(11, Ct), Ct)
