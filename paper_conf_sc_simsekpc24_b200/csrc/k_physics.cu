@@ -473,7 +473,7 @@ __device__ __forceinline__ double momentum_body(const Fields& F, const Params& P
     Rec4 j4v;
     if (kVsig) {  // vsig_ij = c_i + c_j - 3 min(0, rv / r)
       j4v = ldg4(rcur + 4);
-      const double w = rv < 0.0 ? rv / sqrt(r2) : 0.0;
+      const double w = rv < 0.0 ? rv * rsqrt(r2) : 0.0;
       vs = fmax(vs, ci + j4v.b - 3.0 * w);
     }
     if (rv < 0.0) {
