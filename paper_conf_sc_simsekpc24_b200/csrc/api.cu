@@ -90,6 +90,12 @@ struct sph_ctx {
   PhaseRow rows[SPH_NPHASES];
   unsigned long long e0 = 0;
   bool e0_ok = false;
+  // PHASE accounting: the counter read at a phase's end serves as the next
+  // phase's start read when that phase begins right after it (back-to-back
+  // phases inside sph_step); each NVML read costs milliseconds on this host.
+  unsigned long long e_last = 0;
+  bool e_last_ok = false;
+  std::chrono::steady_clock::time_point t_last_end{};
   Nvml nvml;
   int clock_mode = SPH_CLOCK_DEFAULT;
   unsigned clock_mhz[SPH_NPHASES];
@@ -217,7 +223,13 @@ int phase_begin(sph_ctx* c, int p) {
   if (c->cfg.accounting == SPH_ACCOUNTING_PHASE) {
     int rc = cuda_check(c, cudaStreamSynchronize(c->st), "phase sync");
     if (rc) return rc;
-    c->e0_ok = c->nvml.energy_mj(&c->e0);
+    const auto now = std::chrono::steady_clock::now();
+    if (c->e_last_ok && now - c->t_last_end < std::chrono::microseconds(200)) {
+      c->e0 = c->e_last;  // nothing ran since the previous phase's end read
+      c->e0_ok = true;
+    } else {
+      c->e0_ok = c->nvml.energy_mj(&c->e0);
+    }
   }
   return cuda_check(c, cudaEventRecord(c->ev[p][0], c->st), "cudaEventRecord");
 }
@@ -232,15 +244,19 @@ int phase_end(sph_ctx* c, int p) {
     rc = cuda_check(c, cudaStreamSynchronize(c->st), "phase sync");
     if (rc) return rc;
     unsigned long long e1;
+    c->e_last_ok = false;
     if (c->e0_ok && c->nvml.energy_mj(&e1)) {
       c->rows[p].joules += (double)(e1 - c->e0) * 1e-3;
       c->rows[p].avail = true;
+      c->e_last = e1;
+      c->e_last_ok = true;
     }
-    unsigned mhz;
-    if (c->nvml.sm_clock_mhz(&mhz)) {
+    unsigned mhz;  // SM clock sampled at every 8th end of each phase (NVML is slow)
+    if ((c->rows[p].calls & 7) == 1 && c->nvml.sm_clock_mhz(&mhz)) {
       c->rows[p].mhz_sum += mhz;
       c->rows[p].mhz_n++;
     }
+    c->t_last_end = std::chrono::steady_clock::now();
   }
   return SPH_OK;
 }
