@@ -46,6 +46,69 @@ FP64_PEAK_TFLOPS = 148 * 64 * 2 * 1.965e9 / 1e12
 # once, neighbour list once, outputs once): 19 doubles + nc + 4 B per neighbour + 4 doubles.
 MOM_BYTES_PER_PARTICLE = 19 * 8 + 4 + 4 * 8   # + 4 * nc
 
+# Per-phase algorithmic cost (DESIGN.md section 6 / SURVEY 8(d)): HBM bytes per
+# particle (fields read and written once), + bytes per neighbour pair (the list
+# entry), FP64 flops per pair, and the roofline that binds the phase.
+PHASE_COST = {
+    "keys": (40, 0, 0, "hbm"),
+    "sort": (196 + 224, 0, 0, "hbm"),          # 8 radix passes + the permutation
+    "cells": (8, 0, 0, "hbm"),
+    "neighbors": (52, 4, 0, "issue"),          # pos4/x/y/z/h in, nc out, list out
+    "density": (48, 4, FLOPS_PER_PAIR["density"], "fp64"),
+    "eos": (112, 0, 0, "hbm"),               # rho is L2-resident after DENSITY: frac_hbm can exceed 1
+    "gradh": (56, 4, 60, "fp64"),
+    "iad": (96, 4, FLOPS_PER_PAIR["iad"], "fp64"),
+    "momentum_energy": (MOM_BYTES_PER_PARTICLE, 4, FLOPS_PER_PAIR["momentum_energy"], "fp64"),
+    "timestep": (0, 0, 0, "latency"),
+    "update": (180, 0, 0, "hbm"),
+}
+
+
+def hbm_peak_gbs():
+    """The driver-measured copy bandwidth (MEASURED_PEAKS.json), else the
+    profiling guide's fallback."""
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return float(json.load(f)["hbm_gbs"]), "MEASURED_PEAKS.json hbm_gbs"
+    except Exception:
+        return 6540.8, "fallback (earlier measured copy bandwidth)"
+
+
+def idle_power(sim, seconds=2.0):
+    """Board power with the context alive and nothing running: NVML energy
+    counter delta over `seconds` (P:73's whole-board energy includes it)."""
+    e0 = sim.energy_counter_mj()
+    if e0 is None:
+        return None
+    time.sleep(seconds)
+    e1 = sim.energy_counter_mj()
+    return (e1 - e0) * 1e-3 / seconds
+
+
+def phase_table(phase_ms, pairs, n, energy, p_idle):
+    """SURVEY 8(d)'s per-phase record: ms, algorithmic GB/s and TF/s with their
+    roofline fractions, the binding bound, and (from the repeat-phase energy)
+    J, J above idle and EDP = J x s."""
+    peak, _ = hbm_peak_gbs()
+    out = {}
+    for name, ms in phase_ms.items():
+        if ms <= 0 or name not in PHASE_COST:
+            continue
+        b_part, b_pair, f_pair, bound = PHASE_COST[name]
+        t = ms * 1e-3
+        gbs = (b_part * n + b_pair * pairs) / t / 1e9
+        tfs = f_pair * pairs / t / 1e12
+        row = {"ms": ms, "GBps": gbs, "frac_hbm": gbs / peak, "DP_TFLOPs": tfs,
+               "frac_fp64": tfs / FP64_PEAK_TFLOPS, "bound": bound}
+        e = (energy or {}).get("phases", {}).get(name)
+        if e and e.get("J") is not None:
+            row["J"] = e["J"]
+            row["EDP_Js"] = e["J"] * e["ms"] * 1e-3
+            if p_idle is not None:
+                row["J_above_idle"] = e["J"] - p_idle * e["ms"] * 1e-3
+        out[name] = row
+    return out
+
 
 def parse():
     ap = argparse.ArgumentParser()
@@ -510,7 +573,10 @@ def main():
                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                "path": "sph_set_particles(pinned host) + sph_step + sph_get_field x11 (host)"}
 
+    p_idle = idle_power(sim) if args.energy_steps > 0 else None
     energy = measure_energy(sim, sph, n, args, local) if args.energy_steps > 0 else None
+    if energy is not None and p_idle is not None:
+        energy["idle_W"] = p_idle
     accounting = (in_situ_accounting(sim, sph, max(args.energy_steps // 2, 5), ms_max / args.steps)
                   if args.energy_steps > 0 else None)
     trace = dvfs_trace(sim, sph, args.trace_seconds) if args.trace_seconds > 0 else None
@@ -539,6 +605,7 @@ def main():
                            "search_candidates_per_target": infos[-1]["search_candidates"] / n,
                            "search_passes_per_warp": infos[-1]["search_passes"] / (n / 32)},
                 "phase_ms": phase_ms, "fp64_other": other, "roofline": roofline, "e2e": e2e,
+                "phases": phase_table(phase_ms, pairs, n, energy, p_idle),
                 "energy": energy, "accounting": accounting, "dvfs_trace": trace, "cpu_baseline": cpu, "clocks": clk.summary(),
                 "gpu_launches": launches}
         s = json.dumps(line)
