@@ -573,7 +573,9 @@ __global__ void __launch_bounds__(kNbrThreads, 6) neighbors_kernel(Fields F, Par
     wt = __shfl_sync(0xffffffffu, wt, 0);
     const int64_t i = (int64_t)wt * 32 + lane;
     if ((int64_t)wt * 32 >= F.n) break;
-    const bool active = i < F.n;
+    // ghosts (SPH_GHOST_BIT) are candidates only: no list of their own (nc = 0)
+    const bool ghost = i < F.n && (F.id[i] & SPH_GHOST_BIT);
+    const bool active = i < F.n && !ghost;
     const Target t = make_target(F, B, i, active);
     int cc[3] = {0, 0, 0};
     uint32_t ckey = 0;
@@ -616,6 +618,7 @@ __global__ void __launch_bounds__(kNbrThreads, 6) neighbors_kernel(Fields F, Par
       __syncwarp();
     }
     if (active) F.nc[i] = cnt;
+    else if (ghost) F.nc[i] = 0;
     // copy the rows to the column-major list: lane l holds row l; the store of
     // slot k by the 32 lanes is one 128-B line
     const int len = active ? min(cnt, F.ngmax) : 0;

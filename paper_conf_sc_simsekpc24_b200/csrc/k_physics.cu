@@ -124,12 +124,36 @@ __device__ __forceinline__ void density_body(const Fields& F, const Params& P, c
   F.wk[i] = kh3;
 }
 
+// Ghosts (another rank's particles, SPH_GHOST_BIT in the id) are neighbours j
+// only: their own sums would use a truncated neighbourhood and are replaced by
+// the owners' values (halo), so the neighbour sums skip them as targets and
+// write only what the j side reads (kernel factors here, the momentum record in
+// IAD).
+__device__ __forceinline__ bool is_ghost(const Fields& F, int64_t i) { return (F.id[i] & SPH_GHOST_BIT) != 0; }
+
+// The momentum record of a ghost (its C comes from the owner: halo, then
+// refresh_rec_m rewrites the C chunks).
+__device__ __forceinline__ void ghost_rec_m(const Fields& F, int64_t i, const Rec4& me) {
+  Rec4* rm = F.rec_m + (int64_t)kRecM * i;
+  st4(rm + 0, me.a, me.b, me.c, F.wq[i]);
+  st4(rm + 1, 0.0, 0.0, 0.0, F.wk[i]);
+  st4(rm + 2, 0.0, 0.0, 0.0, F.f[FM][i]);
+  st4(rm + 3, F.f[FVX][i], F.f[FVY][i], F.f[FVZ][i], F.prho2[i]);
+  st4(rm + 4, F.f[FH][i], F.c[i], F.rho[i], 1.0);
+}
+
+
 __global__ void __launch_bounds__(kDensThreads, 1024 / kDensThreads) density_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= F.n) return;
   const Geom g = load_geom(F.ds, P);
   const Rec4 me = F.rec_d[i];
   const double hi = F.f[FH][i];
+  if (is_ghost(F, i)) {
+    F.wq[i] = kPi2Over4 / (hi * hi);
+    F.wk[i] = P.K / (hi * hi * hi);
+    return;
+  }
   if (__any_sync(__activemask(), needs_wrap(g, me.a, me.b, me.c, hi)))
     density_body<true>(F, P, g, i, me, hi);
   else
@@ -218,6 +242,7 @@ __global__ void __launch_bounds__(kDensThreads, 1024 / kDensThreads) gradh_kerne
   const Geom g = load_geom(F.ds, P);
   const Rec4 me = F.rec_d[i];
   const double hi = F.f[FH][i];
+  if (is_ghost(F, i)) return;  // Omega of a ghost comes from its owner (halo)
   if (__any_sync(__activemask(), needs_wrap(g, me.a, me.b, me.c, hi)))
     gradh_body<true>(F, P, g, i, me, hi);
   else
@@ -388,6 +413,10 @@ __global__ void __launch_bounds__(512, 1) iad_dc_kernel(Fields F, Params P) {
   if (i >= F.n) return;
   const Geom g = load_geom(F.ds, P);
   const Rec4 me = F.rec_i[i];
+  if (is_ghost(F, i)) {
+    ghost_rec_m(F, i, me);
+    return;
+  }
   if (__any_sync(__activemask(), needs_wrap(g, me.a, me.b, me.c, F.f[FH][i])))
     iad_dc_body<true>(F, P, g, i, me);
   else
@@ -399,6 +428,10 @@ __global__ void __launch_bounds__(kIadThreads, 768 / kIadThreads) iad_kernel(Fie
   if (i >= F.n) return;
   const Geom g = load_geom(F.ds, P);
   const Rec4 me = F.rec_i[i];
+  if (is_ghost(F, i)) {
+    ghost_rec_m(F, i, me);
+    return;
+  }
   if (__any_sync(__activemask(), needs_wrap(g, me.a, me.b, me.c, F.f[FH][i])))
     iad_body<true>(F, g, i, me);
   else
@@ -508,7 +541,7 @@ __device__ __forceinline__ double momentum_body(const Fields& F, const Params& P
 
 __global__ void __launch_bounds__(kMomThreads, 512 / kMomThreads) momentum_energy_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  const bool active = i < F.n;
+  const bool active = i < F.n && !is_ghost(F, i);  // ghosts: no sums, not in the dt minimum
   unsigned long long hc = ~0ull;
   if (active) {
     const Geom g = load_geom(F.ds, P);
