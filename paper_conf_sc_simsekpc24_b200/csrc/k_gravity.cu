@@ -148,16 +148,16 @@ __device__ __forceinline__ void add_multipole(const double* q, double xi, double
 // per lane), the other children are pushed (in reverse: ascending pop order).
 // With theta = 0 every child of a level-(Lt-1) node is a leaf and no other node
 // has leaf children, so the direct sums run over ascending particle indices.
-__global__ void __launch_bounds__(kGravThreads) grav_walk_kernel(Fields F, GravParams G) {
-  __shared__ GravSmem s_w[kGravWarps];
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  GravSmem& S = s_w[warp];
-  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  const bool active = i < F.n;
-  if (!__any_sync(0xffffffffu, active)) return;
+// One walk for the lanes in `mine` (a group of the tile's targets): the
+// opening test uses the bounding box of the group's targets only; the other
+// lanes follow the warp-uniform walk and discard what they compute.
+__device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G, GravSmem& S, int lane,
+                                           int64_t i, bool active, bool mine, double& tax, double& tay,
+                                           double& taz, double& tphi) {
   const int64_t ii = active ? i : F.n - 1;
   const double xi = F.f[FX][ii], yi = F.f[FY][ii], zi = F.f[FZ][ii];
-  double lo[3] = {xi, yi, zi}, hi[3] = {xi, yi, zi};
+  double lo[3] = {mine ? xi : INFINITY, mine ? yi : INFINITY, mine ? zi : INFINITY};
+  double hi[3] = {mine ? xi : -INFINITY, mine ? yi : -INFINITY, mine ? zi : -INFINITY};
 #pragma unroll
   for (int a = 0; a < 3; ++a)
 #pragma unroll
@@ -233,11 +233,23 @@ __global__ void __launch_bounds__(kGravThreads) grav_walk_kernel(Fields F, GravP
     const uint32_t lm = __ballot_sync(0xffffffffu, leaf);
     const uint32_t om = __ballot_sync(0xffffffffu, open);
     __syncwarp();
-    // multipoles
+    // multipoles, two at a time into separate accumulators (independent
+    // dependency chains: the rsqrt + quadrupole chain is latency-bound)
     n_mp += __popc(am);
-    for (uint32_t m = am; m; m &= m - 1) {
-      const int k = __ffs(m) - 1;
-      add_multipole(S.mom[k], xi, yi, zi, Gc, ax, ay, az, phi);
+    {
+      double bx = 0, by = 0, bz = 0, bphi = 0;
+      uint32_t m = am;
+      for (; __popc(m) >= 2; m &= m - 1, m &= m - 1) {
+        const int k0 = __ffs(m) - 1;
+        const int k1 = __ffs(m & (m - 1)) - 1;
+        add_multipole(S.mom[k0], xi, yi, zi, Gc, ax, ay, az, phi);
+        add_multipole(S.mom[k1], xi, yi, zi, Gc, bx, by, bz, bphi);
+      }
+      if (m) add_multipole(S.mom[__ffs(m) - 1], xi, yi, zi, Gc, ax, ay, az, phi);
+      ax += bx;
+      ay += by;
+      az += bz;
+      phi += bphi;
     }
     // leaves, ascending: particles in batches of 32 through shared memory
     for (uint32_t m = lm; m; m &= m - 1) {
@@ -256,16 +268,22 @@ __global__ void __launch_bounds__(kGravThreads) grav_walk_kernel(Fields F, GravP
           S.pm[lane] = r.d;
         }
         __syncwarp();
+        // the self pair is skipped by a zero mass (branch-free, unrolled by 4
+        // for independent rsqrt chains)
+        const int64_t self = ii - (int64_t)b;
+#pragma unroll 4
         for (uint32_t t = 0; t < nb; ++t) {
-          if ((int64_t)(b + t) == ii) continue;
+          const bool me = (int64_t)t == self;
+          const double mt = me ? 0.0 : S.pm[t];
           const double dx = S.px[t] - xi, dy = S.py[t] - yi, dz = S.pz[t] - zi;
-          const double r2 = dx * dx + dy * dy + dz * dz + eps2;
+          const double r2 = me ? 1.0 : dx * dx + dy * dy + dz * dz + eps2;  // finite with eps = 0
           const double ir = rsqrt(r2);
-          const double s3 = Gc * S.pm[t] * ir * ir * ir;
+          const double gm = Gc * mt * ir;
+          const double s3 = gm * ir * ir;
           ax = fma(s3, dx, ax);
           ay = fma(s3, dy, ay);
           az = fma(s3, dz, az);
-          phi -= Gc * S.pm[t] * ir;
+          phi -= gm;
         }
       }
     }
@@ -284,6 +302,36 @@ done:
     atomicAdd(&F.ds->grav_pp, n_pp);
     atomicAdd(&F.ds->grav_pops, n_pop);
   }
+  if (mine) {
+    tax += ax;
+    tay += ay;
+    taz += az;
+    tphi += phi;
+  }
+  __syncwarp();  // the shared stack is reused by the next walk
+}
+
+// A tile of 32 Morton-consecutive targets is walked once per group of targets
+// sharing a cell of side 4 leaf cells (level Lt - 2): a tile that straddles a
+// jump of the Morton curve (e.g. across the empty corners of the box around
+// an Evrard sphere) would otherwise get a box so large that nothing is
+// accepted and its walk degenerates to the direct sum over all particles (one
+// such tile took as long as all the others together).
+__device__ __forceinline__ void walk_tile(const Fields& F, const GravParams& G, GravSmem& S, int lane,
+                                          int64_t i) {
+  const bool active = i < F.n;
+  const int Lg = max(G.level - 2, 0);
+  const unsigned long long ck =
+      active ? (unsigned long long)(F.key[i] >> (3 * (21 - Lg))) : (0xffffffff00000000ull | (unsigned)lane);
+  const uint32_t peers = __match_any_sync(0xffffffffu, ck);
+  uint32_t leaders = __ballot_sync(0xffffffffu, active && (peers & ((1u << lane) - 1u)) == 0);
+  double ax = 0, ay = 0, az = 0, phi = 0;
+  while (leaders) {
+    const int ld = __ffs(leaders) - 1;
+    leaders &= leaders - 1;
+    const uint32_t gm = __shfl_sync(0xffffffffu, peers, ld);
+    walk_group(F, G, S, lane, i, active, ((gm >> lane) & 1u) != 0, ax, ay, az, phi);
+  }
   if (active) {
     F.ax[i] += ax;
     F.ay[i] += ay;
@@ -292,9 +340,26 @@ done:
   }
 }
 
+// Persistent grid; warps take 32-target tiles from an atomic counter.  The
+// cost of a tile varies by an order of magnitude across an Evrard sphere (the
+// centre is dense), so a static one-block-per-tile grid left the SMs idle
+// half of the time waiting on the slow central blocks.
+__global__ void __launch_bounds__(kGravThreads) grav_walk_kernel(Fields F, GravParams G) {
+  __shared__ GravSmem s_w[kGravWarps];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t ntiles = div_up(F.n, 32);
+  while (true) {
+    unsigned long long t = 0;
+    if (lane == 0) t = atomicAdd(&F.ds->grav_next, 1ull);
+    t = __shfl_sync(0xffffffffu, t, 0);
+    if ((int64_t)t >= ntiles) break;
+    walk_tile(F, G, s_w[warp], lane, (int64_t)t * 32 + lane);
+  }
+}
+
 void launch_gravity(const Fields& F, const GravParams& G, cudaStream_t st) {
   if (F.n == 0) return;
-  cudaMemsetAsync(&F.ds->grav_mp, 0, 3 * sizeof(unsigned long long), st);
+  cudaMemsetAsync(&F.ds->grav_mp, 0, 4 * sizeof(unsigned long long), st);  // diagnostics + tile counter
   const int Lt = G.level;
   grav_cells_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F.n, F.key, Lt, F.gcell_start);
   grav_leaf_kernel<<<(unsigned)div_up(int64_t(1) << (3 * Lt), 256), 256, 0, st>>>(F, Lt);
@@ -303,7 +368,16 @@ void launch_gravity(const Fields& F, const GravParams& G, cudaStream_t st) {
     grav_up_kernel<<<(unsigned)div_up(int64_t(1) << (3 * l), 256), 256, 0, st>>>(F, l);
     note_launch();
   }
-  grav_walk_kernel<<<(unsigned)div_up(F.n, kGravThreads), kGravThreads, 0, st>>>(F, G);
+  static int resident = 0;  // SMs x resident CTAs of the walk
+  if (!resident) {
+    int dev = 0, sms = 0, per = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, grav_walk_kernel, kGravThreads, 0);
+    resident = std::max(1, sms * std::max(per, 1));
+  }
+  const int64_t grid = std::min<int64_t>(div_up(F.n, kGravThreads), resident);
+  grav_walk_kernel<<<(unsigned)grid, kGravThreads, 0, st>>>(F, G);
   note_launch();
 }
 

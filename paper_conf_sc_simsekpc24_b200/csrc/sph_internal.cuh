@@ -49,6 +49,7 @@ struct DevScalars {
   unsigned long long nbr_next;    // neighbour search: next 32-target tile (dynamic schedule)
   unsigned long long stir_step;   // STIR phases run since sph_stir_init
   unsigned long long grav_mp, grav_pp, grav_pops;  // gravity walk diagnostics (per warp sums)
+  unsigned long long grav_next;   // gravity walk: next 32-target tile (dynamic schedule)
 };
 
 // Self-gravity (k_gravity.cu).
