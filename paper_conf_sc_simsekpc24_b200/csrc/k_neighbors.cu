@@ -30,10 +30,9 @@
 //     difference, conditional +-L, d2 = (dx*dx + dy*dy) + dz*dz rounded per
 //     operation, d2 < (2h_i)(2h_i)).  Every decision equals the exact predicate's:
 //     the neighbour sets are bit-identical to brute force;
-//  4. hits are appended with predicated stores in candidate order.
-// Hits are appended to row-major scratch rows of the CTA slot (an owner's hits
-// of a chunk are consecutive words: a few lines per store instruction; the
-// scratch of the resident CTAs, ~70 MB, stays in L2); when a warp has finished
+//  4. each lane appends its own hits, in candidate order, to its row.
+// Hits are appended to row-major scratch rows of the CTA slot (the scratch of
+// the resident CTAs, ~70 MB, mostly stays in L2); when a warp has finished
 // its targets, every lane copies its row to the column-major list nbr[k*cap + i]
 // (one 128-B line per store instruction) that the neighbour sums read.  The
 // kernel is persistent (a grid of SMs x resident CTAs, so the scratch is indexed
@@ -193,21 +192,6 @@ __device__ __forceinline__ unsigned long long fma2(unsigned long long a, unsigne
   return d;
 }
 
-
-// Position of the r-th (0-based) set bit of m (popc binary search).
-__device__ __forceinline__ int nth_set_bit(uint32_t m, int r) {
-  int pos = 0, c;
-  c = __popc(m & 0xffffu);
-  if (r >= c) { r -= c; m >>= 16; pos += 16; }
-  c = __popc(m & 0xffu);
-  if (r >= c) { r -= c; m >>= 8; pos += 8; }
-  c = __popc(m & 0xfu);
-  if (r >= c) { r -= c; m >>= 4; pos += 4; }
-  c = __popc(m & 0x3u);
-  if (r >= c) { r -= c; m >>= 2; pos += 2; }
-  if (r >= (int)(m & 1u)) pos += 1;
-  return pos;
-}
 
 constexpr int kMaxRuns = 4 * kMaxWarpCells;  // <= 4 runs of children per cell
 
@@ -512,34 +496,22 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
     }
     // the target itself (d = 0) is not its own neighbour
     hin &= ~S.selfm[lane];
-    // cooperative append: the chunk's hits of all lanes (~100) are written by the
-    // 32 lanes together -- owner lane by binary search over the prefix of hit
-    // counts, its r-th hit by a popc search -- each list staying in candidate
-    // (= ascending index) order.  (A per-lane loop over the hit bits is slower:
-    // the warp runs the busiest lane's ~12 iterations per chunk.)
+    // append: every lane writes its own hits, in candidate (= ascending index)
+    // order, to its L2-resident row.  The warp runs the busiest lane's
+    // iterations (~8-12 per chunk), but each is 5 instructions; a cooperative
+    // append (owner by binary search over the prefix of hit counts, r-th hit by
+    // a popc search, few lines per store) was 9.85 vs 9.07 ms: its shuffle
+    // chains cost more than the scattered row stores.
     const int pc = __popc(hin);
-    int incl = pc;
-#pragma unroll
-    for (int off = 1; off < 32; off <<= 1) {
-      const int v = __shfl_up_sync(0xffffffffu, incl, off);
-      if (lane >= off) incl += v;
-    }
-    const int tot = __shfl_sync(0xffffffffu, incl, 31);
-    for (int hb = 0; hb < tot; hb += 32) {
-      const int h = hb + lane;
-      int owner = 0;
-#pragma unroll
-      for (int step = 16; step > 0; step >>= 1) {
-        const int v = __shfl_sync(0xffffffffu, incl, owner + step - 1);
-        if (v <= h) owner += step;
-      }
-      const int o_excl = __shfl_sync(0xffffffffu, incl - pc, owner);
-      const uint32_t o_mask = __shfl_sync(0xffffffffu, hin, owner);
-      const int o_cnt = __shfl_sync(0xffffffffu, cnt, owner);
-      if (h < tot) {
-        const int r = h - o_excl;
-        const int slot = o_cnt + r;
-        if (slot < ngmax) rows[owner * F.nrows_ld + slot] = (int32_t)S.cj[nth_set_bit(o_mask, r)];
+    {
+      uint32_t m = hin;
+      int slot = cnt;
+      int32_t* myrow = rows + lane * F.nrows_ld;
+      while (m) {
+        const int b = __ffs(m) - 1;
+        m &= m - 1;
+        if (slot < ngmax) myrow[slot] = (int32_t)S.cj[b];
+        ++slot;
       }
     }
     cnt += pc;
