@@ -507,11 +507,17 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
       uint32_t m = hin;
       int slot = cnt;
       int32_t* myrow = rows + lane * F.nrows_ld;
+      // two hits per iteration (the warp runs the busiest lane's count)
       while (m) {
-        const int b = __ffs(m) - 1;
+        const int b0 = __ffs(m) - 1;
         m &= m - 1;
-        if (slot < ngmax) myrow[slot] = (int32_t)S.cj[b];
-        ++slot;
+        const int b1 = m ? __ffs(m) - 1 : b0;
+        const bool two = m != 0;
+        m &= m - 1;
+        const int32_t v0 = (int32_t)S.cj[b0], v1 = (int32_t)S.cj[b1];
+        if (slot < ngmax) myrow[slot] = v0;
+        if (two && slot + 1 < ngmax) myrow[slot + 1] = v1;
+        slot += two ? 2 : 1;
       }
     }
     cnt += pc;
