@@ -284,11 +284,26 @@ __device__ __forceinline__ GroupBox build_cells(const Box& B, const int (&cc)[3]
   __syncwarp();
   uint32_t rank[kMaxWarpCells / 32] = {0, 0, 0, 0};
   const int E = D * 27;
-  for (int u = 0; u < E; ++u) {
-    const unsigned long long w = sk[u];
+  // only the registers that hold entries are ranked (E = 27 for the common
+  // one-cell group: one compare per entry instead of four)
+  if (E <= 32) {
+    for (int u = 0; u < E; ++u) {
+      const unsigned long long w = sk[u];
+      rank[0] += (w < v[0] || (w == v[0] && u < lane)) ? 1u : 0u;
+    }
+  } else if (E <= 64) {
+    for (int u = 0; u < E; ++u) {
+      const unsigned long long w = sk[u];
 #pragma unroll
-    for (int r = 0; r < kMaxWarpCells / 32; ++r)
-      rank[r] += (w < v[r] || (w == v[r] && u < r * 32 + lane)) ? 1u : 0u;
+      for (int r = 0; r < 2; ++r) rank[r] += (w < v[r] || (w == v[r] && u < r * 32 + lane)) ? 1u : 0u;
+    }
+  } else {
+    for (int u = 0; u < E; ++u) {
+      const unsigned long long w = sk[u];
+#pragma unroll
+      for (int r = 0; r < kMaxWarpCells / 32; ++r)
+        rank[r] += (w < v[r] || (w == v[r] && u < r * 32 + lane)) ? 1u : 0u;
+    }
   }
   __syncwarp();
 #pragma unroll
