@@ -464,16 +464,21 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
   const int64_t wbase = i - lane;  // the warp's first target
   S.selfm[lane] = 0u;
   if (nchunks) load(0);
+  // candidate c is staged at slot sigma(c) = 4 (c & 7) + (c >> 3): the sign-bit
+  // gathering below then yields bit c for candidate c
+  const int sg = 4 * (lane & 7) + (lane >> 3);
+  const unsigned long long rin2x2 = pack2(t.r_in2, t.r_in2), rout2x2 = pack2(t.r_out2, t.r_out2);
   for (uint32_t c = 0; c < nchunks; ++c) {
-    S.cx[lane] = q.x + sx;
-    S.cy[lane] = q.y + sy;
-    S.cz[lane] = q.z + sz;
+    S.cx[sg] = q.x + sx;
+    S.cy[sg] = q.y + sy;
+    S.cz[sg] = q.z + sz;
     S.cj[lane] = qj;
     if (c * 32 + (uint32_t)lane < ncand && (uint64_t)((int64_t)qj - wbase) < 32u)
       atomicOr(&S.selfm[(int64_t)qj - wbase], 1u << lane);  // candidate is a target of this warp
     __syncwarp();
     if (c + 1 < nchunks) load(c + 1);
     uint32_t hin = 0, hout = 0;
+    uint32_t pin_prev = 0, pout_prev = 0;
 #pragma unroll
     for (int k = 0; k < 32; k += 2) {
       const unsigned long long px = *reinterpret_cast<const unsigned long long*>(&S.cx[k]);
@@ -493,12 +498,20 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
         dz = pack2(a0, a1);
       }
       const unsigned long long d2 = fma2(dx, dx, fma2(dy, dy, mul2(dz, dz)));
-      float e0, e1;
-      unpack2(d2, e0, e1);
-      hin |= (e0 < t.r_in2 ? 1u : 0u) << k;
-      hin |= (e1 < t.r_in2 ? 1u : 0u) << (k + 1);
-      hout |= (e0 < t.r_out2 ? 1u : 0u) << k;
-      hout |= (e1 < t.r_out2 ? 1u : 0u) << (k + 1);
+      // d2 < r  <=>  sign(fl(d2 - r)) (exact: a rounded difference keeps the sign
+      // and is +0 only for d2 == r; canonical NaN is positive).  The sign bytes
+      // of 4 slots are gathered by PRMT, then shifted into bit positions.
+      const unsigned long long din = sub2(d2, rin2x2), dout = sub2(d2, rout2x2);
+      const uint32_t pin = __byte_perm((uint32_t)din, (uint32_t)(din >> 32), 0x0073);
+      const uint32_t pout = __byte_perm((uint32_t)dout, (uint32_t)(dout >> 32), 0x0073);
+      if ((k & 2) == 0) {
+        pin_prev = pin;
+        pout_prev = pout;
+      } else {
+        const int gq = k >> 2;
+        hin |= (__byte_perm(pin_prev, pin, 0x5410) >> (7 - gq)) & (0x01010101u << gq);
+        hout |= (__byte_perm(pout_prev, pout, 0x5410) >> (7 - gq)) & (0x01010101u << gq);
+      }
     }
     // thin shell: the exact fp64 predicate decides (rare)
     uint32_t shell = hout & ~hin;
