@@ -443,16 +443,29 @@ def step(state: dict, params, dt_prev: float, first_step: bool, ngmax: int | Non
         raise OverflowError(f"neighbour count {int(nb.nc.max())} exceeds capacity {ngmax}")
     rho = density(st["x"], st["y"], st["z"], st["h"], st["m"], bmin, bmax, params.periodic, nb,
                   params)
-    p, c = eos(rho, st["u"], params)
     omega = None
-    if getattr(params, "gradh", 0):
+    ve = {}
+    if getattr(params, "ve", 0):
+        # generalized volume elements (reading 23): X = m / rho0, the
+        # normalisation kx = (K/h^3)[X_i + sum_j X_j S^6] (the density sum with X
+        # in place of m), rho = kx m / X; grad-h with X and kx
+        rho0 = rho
+        X = st["m"] / rho0
+        kx = density(st["x"], st["y"], st["z"], st["h"], X, bmin, bmax, params.periodic, nb, params)
+        rho = kx * st["m"] / X
+        ve = {"rho0": rho0, "X": X, "kx": kx}
+        if getattr(params, "gradh", 0):
+            omega, dWsum, dWabs = gradh(st["x"], st["y"], st["z"], st["h"], X, kx, bmin, bmax,
+                                        params.periodic, nb, params)
+    elif getattr(params, "gradh", 0):
         omega, dWsum, dWabs = gradh(st["x"], st["y"], st["z"], st["h"], st["m"], rho, bmin, bmax,
                                     params.periodic, nb, params)
+    p, c = eos(rho, st["u"], params)
     Cm, tau, tabs, singular = iad(st["x"], st["y"], st["z"], st["h"], st["m"], rho, bmin, bmax,
                                   params.periodic, nb, params)
     if singular:
         raise ArithmeticError("IAD matrix singular")
-    dc = {}
+    dc = dict(ve)
     if omega is not None:
         dc.update({"omega": omega, "dWdh_sum": dWsum, "dWdh_abs": dWabs})
     fav = None
@@ -504,8 +517,8 @@ def sample_step(state: dict, params, dt_prev: float, first_step: bool, targets, 
     ``targets`` are positions in this step's sorted order.  Returns (order, out)
     with ``order`` = sorted ids (full) and ``out[name][k]`` the value at targets[k].
     """
-    if getattr(params, "gradh", 0) or getattr(params, "dt_vsig", 0):
-        raise NotImplementedError("sample_step covers the north-star step (no gradh / dt_vsig)")
+    if getattr(params, "gradh", 0) or getattr(params, "dt_vsig", 0) or getattr(params, "ve", 0):
+        raise NotImplementedError("sample_step covers the north-star step (no gradh / dt_vsig / ve)")
     bmin, bmax = box(state["x"], state["y"], state["z"], params)
     k = keys(state["x"], state["y"], state["z"], bmin, bmax)
     perm = sort_order(k)

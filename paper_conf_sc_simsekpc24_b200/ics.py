@@ -62,6 +62,7 @@ class StepParams:
     grav_level: int = 6     # leaf level of the gravity octree
     gradh: int = 0          # 1: NormalizationGradh, p/(Omega rho^2) in momentum (reading 21)
     dt_vsig: int = 0        # 1: signal-velocity time step (reading 22)
+    ve: int = 0             # 1: generalized volume elements X = m/rho0 (reading 23)
 
     def as_dict(self):
         return asdict(self)

@@ -7,7 +7,10 @@ a central difference of the density in h -- Omega_i = 1 + h_i/(3 rho_i)
 d rho_i/d h_i is the definition, the analytic sum is what the oracle computes.
 Omega = 1 must reproduce the plain step bit for bit, and the Omega-weighted
 pressure terms must keep momentum and energy conserved for symmetric pairs.
-vsig: closed forms on two particles and on a lattice at rest."""
+vsig: closed forms on two particles and on a lattice at rest.
+Volume elements (reading 23): kx = 1 on a perfect lattice, mass scaling, a
+loose partition of unity, Omega_VE against a central difference of kx(h), and
+conservation with the VE density."""
 import math
 
 import numpy as np
@@ -181,3 +184,75 @@ def test_step_with_gradh_and_vsig_runs_and_conserves_mass():
     assert "omega" in o and "vsig" in o
     assert np.all(np.isfinite(st["u"])) and st["m"].sum() == pytest.approx(w.state["m"].sum(),
                                                                            rel=1e-15)
+
+
+# ----------------------------------------------------------------- volume elements
+def _ve_parts(w):
+    s, P = w.state, w.params
+    bmin, bmax = oracle.box(s["x"], s["y"], s["z"], P)
+    nb = oracle.neighbors(s["x"], s["y"], s["z"], s["h"], bmin, bmax, P.periodic)
+    import dataclasses
+    P2 = dataclasses.replace(P, ve=1, gradh=1)
+    st, o = oracle.step({k: v.copy() for k, v in s.items()}, P2, P2.dt_first, True)
+    return o, nb
+
+
+def test_ve_lattice_normalisation_is_one():
+    """Perfect lattice, uniform masses: X = m/rho0 is uniform, so the
+    normalisation kx = sum_j X_j W_ij = X rho0 / m = 1 and rho = rho0."""
+    o, _ = _ve_parts(ics.sedov(12))
+    assert np.allclose(o["kx"], 1.0, rtol=1e-13, atol=0)
+    assert np.allclose(o["rho"], o["rho0"], rtol=1e-13, atol=0)
+
+
+def test_ve_mass_scaling_and_partition_of_unity():
+    """Doubling every mass doubles rho0 and rho and leaves X, kx unchanged; on
+    a disordered set kx stays a partition of unity to within the kernel's
+    accuracy (a few %)."""
+    w = _jittered()
+    o1, _ = _ve_parts(w)
+    w.state["m"] = 2.0 * w.state["m"]
+    o2, _ = _ve_parts(w)
+    assert np.allclose(o2["kx"], o1["kx"], rtol=1e-13, atol=0)
+    assert np.allclose(o2["rho"], 2 * o1["rho"], rtol=1e-13, atol=0)
+    # (h varies by +-10% and m by +-50% here: the sum is a loose partition of unity)
+    assert np.all(np.abs(o1["kx"] - 1) < 0.3) and abs(np.mean(o1["kx"]) - 1) < 0.05
+    assert np.std(o1["kx"]) > 1e-4
+
+
+def test_ve_omega_is_the_h_derivative_of_kx():
+    """Omega_VE = 1 + (h/(3 kx)) d kx/dh with X held fixed (central difference
+    of the normalisation sum, lists recomputed at each h)."""
+    w = _jittered(seed=8)
+    s, P = w.state, w.params
+    o, nb = _ve_parts(w)
+    X, h = o["X"], o["pre"]["h"]
+    pre = o["pre"]
+    bmin, bmax = o["bmin"], o["bmax"]
+
+    def kx_at(hh):
+        nbh = oracle.neighbors(pre["x"], pre["y"], pre["z"], hh, bmin, bmax, P.periodic)
+        return oracle.density(pre["x"], pre["y"], pre["z"], hh, X, bmin, bmax, P.periodic, nbh, P)
+    d = 1e-4
+    dk = (kx_at(h * (1 + d)) - kx_at(h * (1 - d))) / (2 * d * h)
+    assert np.all(np.abs(o["dWdh_sum"] - dk) <= 1e-6 * o["dWdh_abs"])
+    assert np.allclose(o["omega"], 1 + h / (3 * o["kx"]) * dk, rtol=1e-6, atol=0)
+
+
+def test_ve_conserves_momentum_and_energy_uniform_h():
+    import dataclasses
+    w = ics.turbulence(10)
+    s = w.state
+    rng = np.random.default_rng(9)
+    s["u"] = rng.uniform(0.5, 2.0, s["x"].size)
+    w.params = dataclasses.replace(w.params, eos=0, ve=1, gradh=1)
+    st, r = oracle.step({k: v.copy() for k, v in s.items()}, w.params, w.params.dt_first, True)
+    pre = r["pre"]
+    m = pre["m"]
+    scale = (m[:, None] * r["a_abs"]).sum(0)
+    mom = np.array([(m * r["ax"]).sum(), (m * r["ay"]).sum(), (m * r["az"]).sum()])
+    assert np.all(np.abs(mom) < 1e-14 * scale)
+    power = (m * (pre["vx"] * r["ax"] + pre["vy"] * r["ay"] + pre["vz"] * r["az"] + r["du"])).sum()
+    pscale = (m * (np.abs(pre["vx"]) * r["a_abs"][:, 0] + np.abs(pre["vy"]) * r["a_abs"][:, 1]
+                   + np.abs(pre["vz"]) * r["a_abs"][:, 2] + r["du_abs"])).sum()
+    assert abs(power) < 1e-14 * pscale
