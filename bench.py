@@ -124,6 +124,8 @@ def parse():
                     help="IADVelocityDivCurl div/curl + Balsara AV switch (SURVEY 8(f)-1)")
     ap.add_argument("--gradh", action="store_true",
                     help="NormalizationGradh phase, p/(Omega rho^2) in momentum (SURVEY 8(f)-1)")
+    ap.add_argument("--ve", action="store_true",
+                    help="generalized volume elements X = m/rho0 in XMass/NormalizationGradh (SURVEY 8(f)-1)")
     ap.add_argument("--dt-vsig", action="store_true",
                     help="signal-velocity time step (SURVEY 8(f)-1)")
     ap.add_argument("--stir", action="store_true",
@@ -261,12 +263,12 @@ def measure_energy(sim, sph, n, args, gpu_index):
     sim.find_neighbors(stats=False)
     sim.density()
     sim.eos()
-    if sim.cfg.gradh:
+    if sim.cfg.gradh or sim.cfg.ve:
         sim.gradh()
     sim.iad()
     sim.momentum_energy()
     sim.timestep()
-    for ph in ("keys", "sort", "cells", "neighbors", "density", "eos") + (("gradh",) if sim.cfg.gradh else ()) + (
+    for ph in ("keys", "sort", "cells", "neighbors", "density", "eos") + (("gradh",) if sim.cfg.gradh and not sim.cfg.ve else ()) + (
             "iad", "momentum_energy", "timestep"):
         ms1, _ = sim.repeat_phase(ph, 3)
         reps = int(min(200000, max(5, 1500.0 / max(ms1, 1e-4))))
@@ -475,9 +477,9 @@ def main():
     torch.cuda.set_device(local)
     w = make_workload(args.workload, rank)
     n = w.n
-    if args.av_switch or args.gradh or args.dt_vsig:
+    if args.av_switch or args.gradh or args.dt_vsig or args.ve:
         import dataclasses
-        w.params = dataclasses.replace(w.params, av_switch=int(args.av_switch),
+        w.params = dataclasses.replace(w.params, av_switch=int(args.av_switch), ve=int(args.ve),
                                        gradh=int(args.gradh), dt_vsig=int(args.dt_vsig))
     stir_steps = 8192 if args.stir else 0
     sim = sph.Simulation(w.params, n_capacity=n, device=local, stir_steps=stir_steps)
@@ -594,7 +596,8 @@ def main():
                 "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
                 "config": {"workload": args.workload + ("+stir" if args.stir else "")
                            + ("+balsara" if args.av_switch else "")
-                           + ("+gradh" if args.gradh else "") + ("+vsig" if args.dt_vsig else ""),
+                           + ("+gradh" if args.gradh else "") + ("+vsig" if args.dt_vsig else "")
+                           + ("+ve" if args.ve else ""),
                            "n_particles_per_gpu": n,
                            "n_particles_total": n * world,
                            "parallelism": "single GPU" if world == 1 else

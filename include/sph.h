@@ -161,7 +161,9 @@ typedef struct sph_config {
                                p / (Omega rho^2) (reading 21)                     */
   int32_t dt_vsig;          /* 1: signal-velocity time step (reading 22) instead of
                                C min h/c                                          */
-  int32_t reserved[6];
+  int32_t ve;               /* 1: generalized volume elements X = m/rho0 (reading
+                               23): GRADH normalises the density                  */
+  int32_t reserved[5];
 } sph_config;
 
 typedef struct sph_nbr_stats {
@@ -438,7 +440,13 @@ int sph_repeat_phase(sph_ctx* ctx, int phase, int reps, double* ms_per_call,
  * it is pending).  sph_step runs it when cfg.gradh.  With cfg.dt_vsig the
  * momentum-energy phase also forms vsig_i = max(2 c_i, max_j (c_i + c_j - 3 w_ij)),
  * w_ij = min(0, v_ij . d_ij / r_ij) (SPH_F_VSIG), and the time step becomes
- * dt = min(C min_i h_i / vsig_i, growth dt_prev) (reading 22). */
+ * dt = min(C min_i h_i / vsig_i, growth dt_prev) (reading 22).
+ * With cfg.ve (generalized volume elements, reading 23) the same phase first
+ * forms X_i = m_i / rho0_i (rho0 = the density of sph_density), the
+ * normalisation kx_i = (K/h_i^3)[X_i + sum_j X_j S^6] and rho_i = kx_i m_i / X_i,
+ * Omega with X and kx in place of m and rho, and re-runs the EOS on the new
+ * density (p / (Omega rho^2) when cfg.gradh).  sph_step runs it when cfg.gradh
+ * or cfg.ve. */
 int sph_gradh(sph_ctx* ctx);
 
 /* --- self-gravity ------------------------------------------ */

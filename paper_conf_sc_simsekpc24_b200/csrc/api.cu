@@ -361,6 +361,7 @@ int body_simple(sph_ctx* c, int phase, int next_stage) {
       break;
     case SPH_PHASE_GRADH:
       launch_gradh(F, c->P, c->st);
+      if (c->P.ve) launch_eos(F, c->P, c->st, c->P.gradh != 0);  // EOS of the normalised density
       c->gradh_done = true;
       break;
     case SPH_PHASE_IAD: launch_iad(F, c->P, c->st); break;
@@ -443,8 +444,8 @@ static int validate(const sph_config* c) {
   if (c->stir_steps < 0) return fail(nullptr, SPH_ERR_ARG, "stir_steps < 0");
   if (c->divcurl < 0 || c->divcurl > 1 || c->av_switch < 0 || c->av_switch > 1)
     return fail(nullptr, SPH_ERR_ARG, "divcurl and av_switch must be 0 or 1");
-  if (c->gradh < 0 || c->gradh > 1 || c->dt_vsig < 0 || c->dt_vsig > 1)
-    return fail(nullptr, SPH_ERR_ARG, "gradh and dt_vsig must be 0 or 1");
+  if (c->gradh < 0 || c->gradh > 1 || c->dt_vsig < 0 || c->dt_vsig > 1 || c->ve < 0 || c->ve > 1)
+    return fail(nullptr, SPH_ERR_ARG, "gradh, dt_vsig and ve must be 0 or 1");
   if (c->gravity) {
     if (c->periodic[0] || c->periodic[1] || c->periodic[2])
       return fail(nullptr, SPH_ERR_NOT_SUPPORTED, "gravity is for isolated (fully open) boxes");
@@ -595,6 +596,7 @@ int sph_init(const sph_config* cfg, void* arena, size_t arena_bytes, void* strea
   c->P.av_switch = cfg->av_switch ? 1 : 0;
   c->P.divcurl = (cfg->divcurl || cfg->av_switch) ? 1 : 0;
   c->P.gradh = cfg->gradh ? 1 : 0;
+  c->P.ve = cfg->ve ? 1 : 0;
   c->P.dt_vsig = cfg->dt_vsig ? 1 : 0;
   layout(cfg, (char*)arena, c);
   for (int p = 0; p < SPH_NPHASES; ++p) {
@@ -782,7 +784,10 @@ int sph_set_field(sph_ctx* c, int field, const void* src, int mem) {
   }
   if (c->n == 0) return SPH_OK;
   const cudaMemcpyKind kind = mem == SPH_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
-  return cuda_check(c, cudaMemcpyAsync(dst, src, sizeof(double) * c->n, kind, c->st), "set field");
+  rc = cuda_check(c, cudaMemcpyAsync(dst, src, sizeof(double) * c->n, kind, c->st), "set field");
+  if (rc || !(field == SPH_F_RHO && c->P.ve && c->gradh_done && c->stage == S_EOS)) return rc;
+  launch_eos(fields(c), c->P, c->st, c->P.gradh != 0);  // owners' normalised rho (reading 23)
+  return cuda_check(c, cudaGetLastError(), "eos refresh");
 }
 
 int sph_get_local_min_hc(sph_ctx* c, double* min_hc) {
@@ -922,9 +927,13 @@ int sph_scatter_field(sph_ctx* c, int field, const int64_t* idx, int64_t m, cons
   if (m < 0 || (m > 0 && (!idx || !src))) return fail(c, SPH_ERR_ARG, "bad idx/src");
   double* f = nullptr;
   bool prho2 = false;
+  bool eos_refresh = false;
   if (field == SPH_F_RHO) {
     if (c->stage < S_DENS) return fail(c, SPH_ERR_STATE, "scatter(RHO) before sph_density");
     f = c->rho;
+    // after a volume-element GRADH the EOS already ran: run it again on the
+    // owners' normalised densities (reading 23)
+    eos_refresh = c->P.ve && c->gradh_done && c->stage == S_EOS;
   } else if (field >= SPH_F_C11 && field <= SPH_F_C33) {
     if (c->stage < S_IAD) return fail(c, SPH_ERR_STATE, "scatter(C) before sph_iad");
     f = c->C[field - SPH_F_C11];
@@ -942,7 +951,12 @@ int sph_scatter_field(sph_ctx* c, int field, const int64_t* idx, int64_t m, cons
     return fail(c, SPH_ERR_ARG, "field %d is not settable", field);
   }
   rc = cuda_check(c, launch_scatter_field(m, idx, src, f, c->st), "scatter");
-  if (rc || !prho2) return rc;
+  if (rc) return rc;
+  if (eos_refresh) {
+    launch_eos(fields(c), c->P, c->st, c->P.gradh != 0);
+    return cuda_check(c, cudaGetLastError(), "eos refresh");
+  }
+  if (!prho2) return rc;
   launch_prho2(fields(c), c->st);
   return cuda_check(c, cudaGetLastError(), "prho2");
 }
@@ -1032,14 +1046,15 @@ int sph_eos(sph_ctx* c) {
 int sph_gradh(sph_ctx* c) {
   int rc = check_ready(c, S_EOS, "sph_gradh");
   if (rc) return rc;
-  if (!c->cfg.gradh) return fail(c, SPH_ERR_STATE, "gradh not enabled (cfg.gradh = 0)");
+  if (!c->cfg.gradh && !c->cfg.ve) return fail(c, SPH_ERR_STATE, "gradh not enabled (cfg.gradh = cfg.ve = 0)");
   return body_simple(c, SPH_PHASE_GRADH, S_EOS);
 }
 
 int sph_iad(sph_ctx* c) {
   int rc = check_ready(c, S_EOS, "sph_iad");
   if (rc) return rc;
-  if (c->cfg.gradh && !c->gradh_done) return fail(c, SPH_ERR_STATE, "cfg.gradh: sph_gradh must run before sph_iad");
+  if ((c->cfg.gradh || c->cfg.ve) && !c->gradh_done)
+    return fail(c, SPH_ERR_STATE, "cfg.gradh / cfg.ve: sph_gradh must run before sph_iad");
   return body_simple(c, SPH_PHASE_IAD, S_IAD);
 }
 
@@ -1069,7 +1084,7 @@ int sph_step(sph_ctx* c, sph_step_info* info) {
   if ((rc = body_neighbors(c))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_DENSITY, S_DENS))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_EOS, S_EOS))) return rc;
-  if (c->cfg.gradh && (rc = body_simple(c, SPH_PHASE_GRADH, S_EOS))) return rc;
+  if ((c->cfg.gradh || c->cfg.ve) && (rc = body_simple(c, SPH_PHASE_GRADH, S_EOS))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_IAD, S_IAD))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_MOMENTUM_ENERGY, S_MOM))) return rc;
   if (c->cfg.gravity && (rc = body_simple(c, SPH_PHASE_GRAVITY, S_MOM))) return rc;
@@ -1202,7 +1217,8 @@ int sph_repeat_phase(sph_ctx* c, int phase, int reps, double* ms_per_call, doubl
     case SPH_PHASE_EOS: need = S_DENS; break;
     case SPH_PHASE_IAD: need = S_EOS; break;
     case SPH_PHASE_GRADH:
-      if (!c || !c->cfg.gradh) return fail(c, SPH_ERR_STATE, "gradh not enabled (cfg.gradh = 0)");
+      // (with cfg.ve the phase rewrites rho from itself: not repeatable)
+      if (!c || !c->cfg.gradh || c->cfg.ve) return fail(c, SPH_ERR_STATE, "GRADH repeatable only with cfg.gradh and no cfg.ve");
       need = S_EOS;
       break;
     case SPH_PHASE_MOMENTUM_ENERGY: need = S_IAD; break;

@@ -163,7 +163,7 @@ __global__ void __launch_bounds__(kDensThreads, 1024 / kDensThreads) density_ker
 // ------------------------------------------------------------------ EOS
 // Bit-exact vs the oracle (same operation order, IEEE sqrt/div): p, c; plus the
 // derived V = m/rho, p/rho^2 and the IAD record {x, y, z, V}.
-__global__ void __launch_bounds__(256) eos_kernel(Fields F, Params P) {
+__global__ void __launch_bounds__(256) eos_kernel(Fields F, Params P, bool apply_omega) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= F.n) return;
   const double rho = F.rho[i], u = F.f[FU][i];
@@ -180,7 +180,9 @@ __global__ void __launch_bounds__(256) eos_kernel(Fields F, Params P) {
   F.p[i] = p;
   F.c[i] = c;
   F.vol[i] = V;
-  F.prho2[i] = __ddiv_rn(p, __dmul_rn(rho, rho));
+  // after a volume-element GRADH (reading 23) the grad-h factor is already known
+  F.prho2[i] = apply_omega ? __ddiv_rn(p, __dmul_rn(__dmul_rn(rho, rho), F.omega[i]))
+                           : __ddiv_rn(p, __dmul_rn(rho, rho));
   st4(F.rec_i + i, rd.a, rd.b, rd.c, V);
   if (P.divcurl) st4(F.rec_iv + i, F.f[FVX][i], F.f[FVY][i], F.f[FVZ][i], 0.0);
 }
@@ -197,15 +199,23 @@ __device__ __forceinline__ double dwdh_term(double t) {
   return (S2 * S2 * S) * fma(6.0, cos_t(t), -3.0 * S);
 }
 
-template <bool kWrap>
+template <bool kWrap, bool kVE>
 __device__ __forceinline__ void gradh_body(const Fields& F, const Params& P, const Geom& g, int64_t i,
                                            const Rec4& me, double hi) {
+  // records {x, y, z, w}: w = m (plain) or X = V0 = m/rho0 (volume elements,
+  // the EOS's IAD record, reading 23)
   const int nci = min(F.nc[i], F.ngmax);
   const double q = F.wq[i];
-  double sum = 3.0 * me.d;  // self: S = 1, cos = 1
+  double sum = 3.0 * me.d;  // dW/dh bracket, self: S = 1, cos = 1
+  double sw = me.d;         // normalisation sum (kVE), self: S^6 = 1
   const int32_t* __restrict__ nb = F.nbr + i;
-  const Rec4* __restrict__ rec = F.rec_d;
+  const Rec4* __restrict__ rec = kVE ? F.rec_i : F.rec_d;
   const int64_t cap = F.cap;
+  auto add = [&](const Rec4& rj, double t) {
+    const double S = sinc_t(t), S2 = S * S, S5 = S2 * S2 * S;
+    sum = fma(rj.d * S5, fma(6.0, cos_t(t), -3.0 * S), sum);
+    if (kVE) sw = fma(rj.d, S5 * S, sw);
+  };
   Rec4 ra = ldg4(rec + (nci > 0 ? __ldg(nb) : 0)), rb = ldg4(rec + (nci > 1 ? __ldg(nb + cap) : 0));
   int jc = nci > 2 ? __ldg(nb + 2 * cap) : 0, jd = nci > 3 ? __ldg(nb + 3 * cap) : 0;
   int k = 0;
@@ -218,35 +228,48 @@ __device__ __forceinline__ void gradh_body(const Fields& F, const Params& P, con
     double dxa, dya, dza, dxb, dyb, dzb;
     pair_d<kWrap>(g, me.a, me.b, me.c, a.a, a.b, a.c, dxa, dya, dza);
     pair_d<kWrap>(g, me.a, me.b, me.c, b.a, b.b, b.c, dxb, dyb, dzb);
-    const double ta = dwdh_term((dxa * dxa + dya * dya + dza * dza) * q);
-    const double tb = dwdh_term((dxb * dxb + dyb * dyb + dzb * dzb) * q);
-    sum = fma(a.d, ta, sum);
-    sum = fma(b.d, tb, sum);
+    add(a, (dxa * dxa + dya * dya + dza * dza) * q);
+    add(b, (dxb * dxb + dyb * dyb + dzb * dzb) * q);
   }
   if (k < nci) {
     double dx, dy, dz;
     pair_d<kWrap>(g, me.a, me.b, me.c, ra.a, ra.b, ra.c, dx, dy, dz);
-    sum = fma(ra.d, dwdh_term((dx * dx + dy * dy + dz * dz) * q), sum);
+    add(ra, (dx * dx + dy * dy + dz * dz) * q);
   }
-  const double rho = F.rho[i];
+  double rho = F.rho[i];
   const double h2 = hi * hi;
-  const double dsum = -P.K / (h2 * h2) * sum;
-  const double om = 1.0 + hi / (3.0 * rho) * dsum;
-  F.omega[i] = om;
-  F.prho2[i] = __ddiv_rn(F.p[i], __dmul_rn(__dmul_rn(rho, rho), om));
+  if (kVE) {
+    const double kx = P.K / (h2 * hi) * sw;
+    F.rho[i] = kx * F.f[FM][i] / me.d;  // rho = kx m / X
+    rho = kx;                            // Omega uses kx in place of rho
+  }
+  if (P.gradh) {
+    const double dsum = -P.K / (h2 * h2) * sum;
+    const double om = 1.0 + hi / (3.0 * rho) * dsum;
+    F.omega[i] = om;
+    if (!kVE) F.prho2[i] = __ddiv_rn(F.p[i], __dmul_rn(__dmul_rn(rho, rho), om));
+  }
 }
 
 __global__ void __launch_bounds__(kDensThreads, 1024 / kDensThreads) gradh_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= F.n) return;
   const Geom g = load_geom(F.ds, P);
-  const Rec4 me = F.rec_d[i];
   const double hi = F.f[FH][i];
-  if (is_ghost(F, i)) return;  // Omega of a ghost comes from its owner (halo)
-  if (__any_sync(__activemask(), needs_wrap(g, me.a, me.b, me.c, hi)))
-    gradh_body<true>(F, P, g, i, me, hi);
-  else
-    gradh_body<false>(F, P, g, i, me, hi);
+  if (is_ghost(F, i)) return;  // rho and Omega of a ghost come from its owner (halo)
+  if (P.ve) {
+    const Rec4 me = F.rec_i[i];
+    if (__any_sync(__activemask(), needs_wrap(g, me.a, me.b, me.c, hi)))
+      gradh_body<true, true>(F, P, g, i, me, hi);
+    else
+      gradh_body<false, true>(F, P, g, i, me, hi);
+  } else {
+    const Rec4 me = F.rec_d[i];
+    if (__any_sync(__activemask(), needs_wrap(g, me.a, me.b, me.c, hi)))
+      gradh_body<true, false>(F, P, g, i, me, hi);
+    else
+      gradh_body<false, false>(F, P, g, i, me, hi);
+  }
 }
 
 // p/(Omega rho^2) again after sph_set_field wrote the owners' Omega over the
@@ -637,9 +660,9 @@ void launch_density(const Fields& F, const Params& P, cudaStream_t st) {
   density_kernel<<<(unsigned)div_up(F.n, kDensThreads), kDensThreads, 0, st>>>(F, P);
   note_launch();
 }
-void launch_eos(const Fields& F, const Params& P, cudaStream_t st) {
+void launch_eos(const Fields& F, const Params& P, cudaStream_t st, bool apply_omega) {
   if (F.n == 0) return;
-  eos_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F, P);
+  eos_kernel<<<(unsigned)div_up(F.n, 256), 256, 0, st>>>(F, P, apply_omega);
   note_launch();
 }
 void launch_iad(const Fields& F, const Params& P, cudaStream_t st) {

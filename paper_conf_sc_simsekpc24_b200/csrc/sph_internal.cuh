@@ -135,7 +135,7 @@ struct Params {
   double av_alpha, av_beta, av_eps;
   int max_cell_level;
   int divcurl, av_switch;
-  int gradh, dt_vsig;
+  int gradh, dt_vsig, ve;
 };
 
 // Process-wide count of libsph kernel launches (sph_kernel_launches).
@@ -279,7 +279,7 @@ void launch_neighbors(const Fields& F, const Params& P, cudaStream_t st);
 constexpr int kNbrSlots = 1024;    // neighbour-search CTAs in flight (>= SMs x resident CTAs)
 constexpr int kNbrSlotRows = 128;  // scratch rows per CTA (its threads)
 void launch_density(const Fields& F, const Params& P, cudaStream_t st);
-void launch_eos(const Fields& F, const Params& P, cudaStream_t st);
+void launch_eos(const Fields& F, const Params& P, cudaStream_t st, bool apply_omega = false);
 void launch_iad(const Fields& F, const Params& P, cudaStream_t st);
 void launch_gradh(const Fields& F, const Params& P, cudaStream_t st);
 // decomposition plumbing (k_decomp.cu)

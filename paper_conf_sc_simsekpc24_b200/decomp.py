@@ -306,9 +306,10 @@ class DistributedSim:
         sim.density()
         self._halo(["rho"])
         sim.eos()
-        if getattr(self.params, "gradh", 0):  # owners' Omega over the ghosts
-            sim.gradh()
-            self._halo(["omega"])
+        if getattr(self.params, "gradh", 0) or getattr(self.params, "ve", 0):
+            sim.gradh()  # owners' normalised rho (volume elements) and Omega over the ghosts
+            self._halo((["rho"] if getattr(self.params, "ve", 0) else [])
+                       + (["omega"] if getattr(self.params, "gradh", 0) else []))
         sim.iad()
         # H3: the owners' C (and Balsara factors when the AV switch is on)
         h3 = ["c11", "c12", "c13", "c22", "c23", "c33"]

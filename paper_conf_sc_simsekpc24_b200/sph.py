@@ -54,7 +54,7 @@ class Config(C.Structure):
         ("stir_steps", C.c_int32), ("divcurl", C.c_int32), ("av_switch", C.c_int32),
         ("gravity", C.c_int32), ("grav_level", C.c_int32), ("grav_G", C.c_double),
         ("grav_eps", C.c_double), ("grav_theta", C.c_double), ("gradh", C.c_int32),
-        ("dt_vsig", C.c_int32), ("reserved", C.c_int32 * 6),
+        ("dt_vsig", C.c_int32), ("ve", C.c_int32), ("reserved", C.c_int32 * 5),
     ]
 
 
@@ -198,6 +198,7 @@ def config_from_params(params, n_capacity: int, device: int = 0, accounting: int
     c.gravity = int(getattr(params, "gravity", 0))
     c.gradh = int(getattr(params, "gradh", 0))
     c.dt_vsig = int(getattr(params, "dt_vsig", 0))
+    c.ve = int(getattr(params, "ve", 0))
     if c.gravity:
         c.grav_level = int(params.grav_level)
         c.grav_G = float(params.grav_G)

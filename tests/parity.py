@@ -22,7 +22,7 @@ def gpu_pipeline(sim):
     stats = sim.find_neighbors()
     sim.density()
     sim.eos()
-    if sim.cfg.gradh:
+    if sim.cfg.gradh or sim.cfg.ve:
         sim.gradh()
     sim.iad()
     sim.momentum_energy()

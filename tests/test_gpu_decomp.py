@@ -40,10 +40,17 @@ def _random_gradh_vsig():
     return w
 
 
+def _random_ve():
+    import dataclasses
+    w = ics.random_box(6000, seed=5)
+    w.params = dataclasses.replace(w.params, ve=1, gradh=1)  # halo of the normalised rho and Omega
+    return w
+
+
 def _make(name):
     return {"turbulence16": lambda: ics.turbulence(16), "random": lambda: ics.random_box(6000, seed=5),
             "sedov14": lambda: ics.sedov(14), "sedov14_balsara": _sedov_balsara,
-            "random_gradh_vsig": _random_gradh_vsig}[name]()
+            "random_gradh_vsig": _random_gradh_vsig, "random_ve": _random_ve}[name]()
 
 
 def _worker(rank, world, port, name, q):
@@ -78,7 +85,7 @@ def _single(name):
 
 
 @pytest.mark.parametrize("name", ["turbulence16", "random", "sedov14", "sedov14_balsara",
-                                  "random_gradh_vsig"])
+                                  "random_gradh_vsig", "random_ve"])
 def test_two_ranks_bit_identical_to_one(name):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()

@@ -1,5 +1,5 @@
-"""GPU parity of NormalizationGradh (reading 21) and of the
-signal-velocity time step (reading 22): libsph's GRADH phase (sincospi per
+"""GPU parity of NormalizationGradh (reading 21), its volume-element
+form (reading 23) and of the signal-velocity time step (reading 22): libsph's GRADH phase (sincospi per
 pair) and the vsig maximum inside MOMENTUM_ENERGY against the oracle's plain
 sums, on the tolerance metric of DESIGN.md section 3 (scale = sum of |terms|),
 one step and ten steps."""
@@ -18,6 +18,9 @@ CASES = {
     "sedov16_gradh_vsig": lambda: (ics.sedov(16), dict(gradh=1, dt_vsig=1)),
     "random_gradh": lambda: (ics.random_box(6000, seed=7), dict(gradh=1)),
     "turbulence16_vsig": lambda: (ics.turbulence(16), dict(dt_vsig=1)),
+    "turbulence16_ve": lambda: (ics.turbulence(16), dict(ve=1)),
+    "sedov16_ve_gradh": lambda: (ics.sedov(16), dict(ve=1, gradh=1)),
+    "random_ve_gradh": lambda: (ics.random_box(6000, seed=7), dict(ve=1, gradh=1, dt_vsig=1)),
 }
 
 
@@ -42,10 +45,22 @@ def test_omega(case):
     name, w, sim, g, st, o = case
     if not w.params.gradh:
         pytest.skip("gradh off")
-    h, rho = g["h"], o["rho"]
+    h = g["h"]
+    rho = o["kx"] if w.params.ve else o["rho"]   # volume elements: kx in place of rho
     scale = h / (3 * rho) * o["dWdh_abs"]
     assert_sum_close(g["omega"], o["omega"], scale, TOL_1STEP, "omega")
     assert np.max(np.abs(o["omega"] - 1)) > 1e-4   # the factor is not trivially 1
+
+
+def test_ve_density(case):
+    """Volume elements (reading 23): the normalised density against the
+    oracle's kx m / X (rho0 from the plain density sum)."""
+    from parity import TOL_1STEP, assert_rel_close
+    name, w, sim, g, st, o = case
+    if not w.params.ve:
+        pytest.skip("ve off")
+    assert_rel_close(g["rho"], o["rho"], TOL_1STEP, "rho (volume elements)")
+    assert np.max(np.abs(o["kx"] - 1)) > 1e-6 or name.startswith("sedov")
 
 
 def test_vsig(case):
