@@ -362,16 +362,7 @@ __device__ __forceinline__ void iad_dc_body(const Fields& F, const Params& P, co
   const Rec4* __restrict__ rec = F.rec_i;
   const Rec4* __restrict__ rv = F.rec_iv;
   const int64_t cap = F.cap;
-  int jn = nci > 0 ? __ldg(nb) : 0;
-  Rec4 ra = ldg4(rec + jn), va = ldg4(rv + jn);
-  jn = nci > 1 ? __ldg(nb + cap) : 0;
-  for (int k = 0; k < nci; ++k) {
-    const Rec4 rj = ra, vj = va;
-    if (k + 1 < nci) {
-      ra = ldg4(rec + jn);
-      va = ldg4(rv + jn);
-    }
-    if (k + 2 < nci) jn = __ldg(nb + (int64_t)(k + 2) * cap);
+  auto add = [&](const Rec4& rj, const Rec4& vj) {
     double dx, dy, dz;
     pair_d<kWrap>(g, me.a, me.b, me.c, rj.a, rj.b, rj.c, dx, dy, dz);
     const double r2 = dx * dx + dy * dy + dz * dz;
@@ -390,7 +381,29 @@ __device__ __forceinline__ void iad_dc_body(const Fields& F, const Params& P, co
     for (int a = 0; a < 3; ++a)
 #pragma unroll
       for (int b = 0; b < 3; ++b) M[a][b] = fma(-aw[a], dv[b], M[a][b]);
+  };
+  // two neighbours per iteration (as iad_body), records one pair ahead,
+  // indices two ahead; the sums still run in list order
+  int j0 = nci > 0 ? __ldg(nb) : 0, j1 = nci > 1 ? __ldg(nb + cap) : 0;
+  Rec4 ra = ldg4(rec + j0), va = ldg4(rv + j0), rb = ldg4(rec + j1), vb = ldg4(rv + j1);
+  int jc = nci > 2 ? __ldg(nb + 2 * cap) : 0, jd = nci > 3 ? __ldg(nb + 3 * cap) : 0;
+  int k = 0;
+  for (; k + 1 < nci; k += 2) {
+    const Rec4 a = ra, av = va, b = rb, bv = vb;
+    if (k + 2 < nci) {
+      ra = ldg4(rec + jc);
+      va = ldg4(rv + jc);
+    }
+    if (k + 3 < nci) {
+      rb = ldg4(rec + jd);
+      vb = ldg4(rv + jd);
+    }
+    if (k + 4 < nci) jc = __ldg(nb + (int64_t)(k + 4) * cap);
+    if (k + 5 < nci) jd = __ldg(nb + (int64_t)(k + 5) * cap);
+    add(a, av);
+    add(b, bv);
   }
+  if (k < nci) add(ra, va);
   const double det = t11 * (t22 * t33 - t23 * t23) - t12 * (t12 * t33 - t23 * t13) +
                      t13 * (t12 * t23 - t22 * t13);
   const double inv = 1.0 / det;
@@ -431,7 +444,10 @@ __device__ __forceinline__ void iad_dc_body(const Fields& F, const Params& P, co
   st4(rm + 4, F.f[FH][i], F.c[i], F.rho[i], f);
 }
 
-__global__ void __launch_bounds__(512, 1) iad_dc_kernel(Fields F, Params P) {
+// 512 threads x 128 registers (640 x 102 spills with the two-pair loop;
+// one pair per iteration: 512 -> 6.02, 640 -> 5.53 ms; two pairs at 512: 4.78)
+constexpr int kIadDcThreads = 512;
+__global__ void __launch_bounds__(kIadDcThreads, 1) iad_dc_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= F.n) return;
   const Geom g = load_geom(F.ds, P);
@@ -668,7 +684,7 @@ void launch_eos(const Fields& F, const Params& P, cudaStream_t st, bool apply_om
 void launch_iad(const Fields& F, const Params& P, cudaStream_t st) {
   if (F.n == 0) return;
   if (P.divcurl)
-    iad_dc_kernel<<<(unsigned)div_up(F.n, 512), 512, 0, st>>>(F, P);
+    iad_dc_kernel<<<(unsigned)div_up(F.n, kIadDcThreads), kIadDcThreads, 0, st>>>(F, P);
   else
     iad_kernel<<<(unsigned)div_up(F.n, kIadThreads), kIadThreads, 0, st>>>(F, P);
   note_launch();
