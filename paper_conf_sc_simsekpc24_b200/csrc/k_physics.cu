@@ -548,18 +548,22 @@ __device__ __forceinline__ double momentum_body(const Fields& F, const Params& P
       const double w = rv < 0.0 ? rv * rsqrt(r2) : 0.0;
       vs = fmax(vs, ci + j4v.b - 3.0 * w);
     }
-    if (rv < 0.0) {
-      const Rec4 j4 = kVsig ? j4v : ldg4(rcur + 4);
+    {
+      // branch-free AV: the AV chunk is loaded by approaching lanes only (a
+      // predicated load; receding lanes use their own values, finite), Pi is
+      // formed by every lane and zeroed for receding pairs
+      Rec4 j4;
+      if (kVsig) j4 = j4v; else { j4.a = hi; j4.b = ci; j4.c = rhoi; j4.d = fi; }
+      if (!kVsig && rv < 0.0) j4 = ldg4(rcur + 4);
       const double hbar = 0.5 * (hi + j4.a);
       const double cbar = 0.5 * (ci + j4.b);
       const double rhobar = 0.5 * (rhoi + j4.c);
-      // mu = hbar rv / D, Pi = (-alpha cbar mu + beta mu^2) / rhobar with one
-      // division: q = 1 / (D rhobar), 1/D = rhobar q, 1/rhobar = D q
       const double D = fma(eps * hbar, hbar, r2);
       const double q = 1.0 / (D * rhobar);
       const double mu = hbar * rv * (rhobar * q);
-      Pi = (fma(beta, mu, -alpha * cbar) * mu) * (D * q);
-      if (kSwitch) Pi *= 0.5 * (fi + j4.d);  // Balsara switch (reading 19)
+      double pv = (fma(beta, mu, -alpha * cbar) * mu) * (D * q);
+      if (kSwitch) pv *= 0.5 * (fi + j4.d);
+      Pi = rv < 0.0 ? pv : 0.0;
     }
     const double mj = j2.d, prj = j3.d;
     const double ka = (pri + 0.5 * Pi) * wi, kb = (prj + 0.5 * Pi) * wj;
