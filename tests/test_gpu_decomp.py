@@ -172,3 +172,30 @@ def test_device_plumbing_matches_host_logic():
         g = sim.gather_field("h", torch.tensor([2, 0, 1], device=dev))
         assert g.cpu().tolist() == st2["h"][[2, 0, 1]].tolist()
     sim.finalize()
+
+
+def test_device_plumbing_edge_cases():
+    """Empty compaction, append past the capacity (SPH_ERR_CAPACITY, state
+    unchanged), too many ranks for the ghost mask (SPH_ERR_ARG), empty packs."""
+    from paper_conf_sc_simsekpc24_b200 import sph
+    w = ics.random_box(500, seed=3)
+    sim = sph.Simulation(w.params, n_capacity=600)
+    sim.set_particles({k: np.ascontiguousarray(v) for k, v in w.state.items()})
+    dev = torch.device("cuda", 0)
+    with torch.cuda.stream(sim.stream):
+        rows = sim.pack_rows(torch.arange(200, device=dev))
+        with pytest.raises(sph.SphError) as e:
+            sim.append_rows(rows)                 # 500 + 200 > 600
+        assert "CAPACITY" in str(e.value)
+        assert sim.n == 500
+        sim.append_rows(rows[:100])
+        assert sim.n == 600
+        assert sim.pack_rows(torch.zeros(0, dtype=torch.int64, device=dev)).shape == (0, sph.ROW_DOUBLES)
+        with pytest.raises(sph.SphError):
+            sim.select_ghosts(np.zeros((65, 6)), 0, 0.1)
+        assert sim.compact(keep=torch.zeros(600, dtype=torch.bool, device=dev)) == 0
+        assert sim.n == 0
+        sim.append_rows(rows[:10])
+        st = sim.get_state()
+        assert np.array_equal(st["x"], w.state["x"][:10])
+    sim.finalize()
