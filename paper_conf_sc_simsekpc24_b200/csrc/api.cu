@@ -145,8 +145,9 @@ int check_ready(sph_ctx* c, int min_stage, const char* what) {
   return SPH_OK;
 }
 
-// Row stride of the neighbour-search scratch rows: ngmax rounded up to 8.
-int64_t nrows_ld(const sph_config* cfg) { return ((int64_t)cfg->ngmax + 7) / 8 * 8; }
+// Row stride of the neighbour-search scratch rows: ngmax + 1 (a spare word for
+// the branch-free append) rounded up to 8.
+int64_t nrows_ld(const sph_config* cfg) { return ((int64_t)cfg->ngmax + 8) / 8 * 8; }
 
 Fields fields(sph_ctx* c) {
   Fields F;

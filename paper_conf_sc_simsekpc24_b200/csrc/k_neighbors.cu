@@ -543,8 +543,10 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
         const bool two = m != 0;
         m &= m - 1;
         const int32_t v0 = (int32_t)S.cj[b0], v1 = (int32_t)S.cj[b1];
-        if (slot < ngmax) myrow[slot] = v0;
-        if (two && slot + 1 < ngmax) myrow[slot + 1] = v1;
+        // branch-free: past the capacity (or for a missing second hit) the
+        // store goes to the row's spare word ngmax (nrows_ld > ngmax), never read
+        myrow[min(slot, ngmax)] = v0;
+        myrow[two ? min(slot + 1, ngmax) : ngmax] = v1;
         slot += two ? 2 : 1;
       }
     }

@@ -117,7 +117,7 @@ struct Fields {
   int32_t* nc;
   int32_t* nbr;           // [ngmax][cap] column-major: neighbour k of target i at nbr[k * cap + i]
   int32_t* nrows;         // neighbour-search scratch: row-major rows of the resident warps
-  int64_t nrows_ld;       // their row stride (ngmax rounded up to 8: 32-B aligned rows)
+  int64_t nrows_ld;       // their row stride (ngmax + 1 rounded up to 8: 32-B aligned rows, a spare word)
   int32_t ngmax;
   uint32_t* cell_start;   // [8^L + 1], L = fine cell level
   float4* pos4;           // fp32 (x, y, z) - box_min: neighbour-search prefilter
