@@ -585,7 +585,7 @@ def main():
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        k = args.cpu_sample or 160  # ~10 s of oracle work on the host cores
+        k = args.cpu_sample or 240  # ~10 s of oracle work on the host cores
         v, sec, threads = cpu_baseline(w, k)
         cpu = {"value": v, "unit": UNIT, "cores": threads, "kind": "oracle",
                "sample": f"{k} random targets of {args.workload}, one step (oracle sampled mode), {sec:.1f} s"}
