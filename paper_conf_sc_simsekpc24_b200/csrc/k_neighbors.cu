@@ -24,15 +24,19 @@
 //     load per lane, prefetched one chunk ahead, staged in shared memory) and every
 //     lane tests every candidate two at a time with packed f32x2 arithmetic
 //     (FADD2/FFMA2) against an outer and an inner radius that bracket 2h_i by a
-//     rigorous bound on the fp32 rounding (reading 14):
+//     rigorous bound on the fp32 rounding (reading 14),
+//     the two comparisons taken as the sign bits of packed differences gathered
+//     four at a time by PRMT (candidates staged in a permuted slot order so
+//     that bit c of the masks is candidate c):
 //     outside -> rejected, inside -> accepted; only the thin shell in between
 //     (~1e-4 of candidates) runs the oracle's exact fp64 predicate (raw
 //     difference, conditional +-L, d2 = (dx*dx + dy*dy) + dz*dz rounded per
 //     operation, d2 < (2h_i)(2h_i)).  Every decision equals the exact predicate's:
 //     the neighbour sets are bit-identical to brute force;
-//  4. each lane appends its own hits, in candidate order, to its row.
-// Hits are appended to row-major scratch rows of the CTA slot (the scratch of
-// the resident CTAs, ~70 MB, mostly stays in L2); when a warp has finished
+//  4. each lane appends its own hits, in candidate order, two per iteration and
+//     branch-free (a spare word past ngmax absorbs over-capacity stores), to its
+//     row-major scratch row (the scratch of the resident CTAs, ~70 MB, mostly
+//     stays in L2); when a warp has finished
 // its targets, every lane copies its row to the column-major list nbr[k*cap + i]
 // (one 128-B line per store instruction) that the neighbour sums read.  The
 // kernel is persistent (a grid of SMs x resident CTAs, so the scratch is indexed
