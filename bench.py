@@ -439,7 +439,7 @@ def run_decomposed(args, rank, world, local):
                 "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
                 "config": {"workload": f"turbulence{nside}", "n_particles_total": n_total,
                            "n_particles_per_gpu": n_total / world,
-                           "parallelism": f"SFC domain decomposition over {world} GPUs, halo exchange (NCCL)",
+                           "parallelism": f"SFC domain decomposition over {world} GPUs, halo exchange ({dist.get_backend().upper()})",
                            "ghost_fraction": float(ghosts[0] / ghosts[1]),
                            "l2": "inputs >> 126 MB L2; no flush"},
                 "phase_ms_rank0": phase_ms, "roofline": None,
