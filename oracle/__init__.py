@@ -69,10 +69,8 @@ _I32 = C.POINTER(C.c_int32)
 _U64 = C.POINTER(C.c_uint64)
 
 
-def lib():
-    global _lib
-    if _lib is None:
-        L = C.CDLL(build())
+def _configure(L):
+    if True:
         L.oracle_sinc.restype = C.c_double
         L.oracle_sinc.argtypes = [C.c_double]
         L.oracle_W.restype = C.c_double
@@ -86,8 +84,34 @@ def lib():
         L.oracle_av_pi.argtypes = [C.c_double] * 5 + [C.POINTER(_Params)]
         L.oracle_timestep.restype = C.c_double
         L.oracle_ball.restype = C.c_int64
-        _lib = L
+    return L
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        _lib = _configure(C.CDLL(build()))
     return _lib
+
+
+class use_library:
+    """Context manager: run the oracle functions on another compiled copy of
+    oracle.c (tests/test_oracle_mutants.py checks that deliberately broken copies
+    fail the pins)."""
+
+    def __init__(self, path: str):
+        self.path = path
+
+    def __enter__(self):
+        global _lib
+        self.prev = lib()
+        _lib = _configure(C.CDLL(self.path))
+        return _lib
+
+    def __exit__(self, *exc):
+        global _lib
+        _lib = self.prev
+        return False
 
 
 def _p(a, t):
@@ -426,6 +450,53 @@ def gravity(x, y, z, m, G: float, eps: float):
     return {"ax": ax, "ay": ay, "az": az, "phi": phi, "a_abs": aabs}
 
 
+def _physics(st: dict, params, bmin, bmax, nb: Neighbors):
+    """The neighbour sums of one step on a sorted particle set with its lists, in
+    the order of SURVEY 8(c) steps 5-8 (+ the opt-in 8(f)-1 functions): density,
+    [volume elements], [grad-h], EOS, IAD, [div/curl, Balsara switch],
+    momentum-energy.  Returns every quantity by name."""
+    rho = density(st["x"], st["y"], st["z"], st["h"], st["m"], bmin, bmax, params.periodic, nb,
+                  params)
+    omega = None
+    out = {}
+    if getattr(params, "ve", 0):
+        # generalized volume elements (reading 23): X = m / rho0, the
+        # normalisation kx = (K/h^3)[X_i + sum_j X_j S^6] (the density sum with X
+        # in place of m), rho = kx m / X; grad-h with X and kx
+        rho0 = rho
+        X = st["m"] / rho0
+        kx = density(st["x"], st["y"], st["z"], st["h"], X, bmin, bmax, params.periodic, nb, params)
+        rho = kx * st["m"] / X
+        out.update({"rho0": rho0, "X": X, "kx": kx})
+        if getattr(params, "gradh", 0):
+            omega, dWsum, dWabs = gradh(st["x"], st["y"], st["z"], st["h"], X, kx, bmin, bmax,
+                                        params.periodic, nb, params)
+    elif getattr(params, "gradh", 0):
+        omega, dWsum, dWabs = gradh(st["x"], st["y"], st["z"], st["h"], st["m"], rho, bmin, bmax,
+                                    params.periodic, nb, params)
+    if omega is not None:
+        out.update({"omega": omega, "dWdh_sum": dWsum, "dWdh_abs": dWabs})
+    p, c = eos(rho, st["u"], params)
+    Cm, tau, tabs, singular = iad(st["x"], st["y"], st["z"], st["h"], st["m"], rho, bmin, bmax,
+                                  params.periodic, nb, params)
+    if singular:
+        raise ArithmeticError("IAD matrix singular")
+    fav = None
+    if getattr(params, "divcurl", 0) or getattr(params, "av_switch", 0):
+        T, Tabs, dvv, curl = divcurl(st["x"], st["y"], st["z"], st["vx"], st["vy"], st["vz"],
+                                     st["h"], st["m"], rho, Cm, bmin, bmax, params.periodic, nb,
+                                     params)
+        out.update({"T": T, "T_abs": Tabs, "divv": dvv, "curl": curl})
+        if getattr(params, "av_switch", 0):
+            fav = balsara(dvv, curl, c, st["h"])
+            out["bal"] = fav
+    acc = momentum_energy(st["x"], st["y"], st["z"], st["vx"], st["vy"], st["vz"], st["h"],
+                          st["m"], rho, p, c, Cm, bmin, bmax, params.periodic, nb, params, fav,
+                          omega)
+    out.update({"rho": rho, "p": p, "c": c, "C": Cm, "tau": tau, "tau_abs": tabs, **acc})
+    return out
+
+
 def step(state: dict, params, dt_prev: float, first_step: bool, ngmax: int | None = None,
          stir: dict | None = None):
     """One full oracle step.  Returns (new_state, out) where new_state is in this
@@ -441,46 +512,8 @@ def step(state: dict, params, dt_prev: float, first_step: bool, ngmax: int | Non
     nb = neighbors(st["x"], st["y"], st["z"], st["h"], bmin, bmax, params.periodic)
     if ngmax is not None and nb.nc.size and int(nb.nc.max()) > ngmax:
         raise OverflowError(f"neighbour count {int(nb.nc.max())} exceeds capacity {ngmax}")
-    rho = density(st["x"], st["y"], st["z"], st["h"], st["m"], bmin, bmax, params.periodic, nb,
-                  params)
-    omega = None
-    ve = {}
-    if getattr(params, "ve", 0):
-        # generalized volume elements (reading 23): X = m / rho0, the
-        # normalisation kx = (K/h^3)[X_i + sum_j X_j S^6] (the density sum with X
-        # in place of m), rho = kx m / X; grad-h with X and kx
-        rho0 = rho
-        X = st["m"] / rho0
-        kx = density(st["x"], st["y"], st["z"], st["h"], X, bmin, bmax, params.periodic, nb, params)
-        rho = kx * st["m"] / X
-        ve = {"rho0": rho0, "X": X, "kx": kx}
-        if getattr(params, "gradh", 0):
-            omega, dWsum, dWabs = gradh(st["x"], st["y"], st["z"], st["h"], X, kx, bmin, bmax,
-                                        params.periodic, nb, params)
-    elif getattr(params, "gradh", 0):
-        omega, dWsum, dWabs = gradh(st["x"], st["y"], st["z"], st["h"], st["m"], rho, bmin, bmax,
-                                    params.periodic, nb, params)
-    p, c = eos(rho, st["u"], params)
-    Cm, tau, tabs, singular = iad(st["x"], st["y"], st["z"], st["h"], st["m"], rho, bmin, bmax,
-                                  params.periodic, nb, params)
-    if singular:
-        raise ArithmeticError("IAD matrix singular")
-    dc = dict(ve)
-    if omega is not None:
-        dc.update({"omega": omega, "dWdh_sum": dWsum, "dWdh_abs": dWabs})
-    fav = None
-    if getattr(params, "divcurl", 0) or getattr(params, "av_switch", 0):
-        T, Tabs, dvv, curl = divcurl(st["x"], st["y"], st["z"], st["vx"], st["vy"], st["vz"],
-                                     st["h"], st["m"], rho, Cm, bmin, bmax, params.periodic, nb,
-                                     params)
-        dc = {"T": T, "T_abs": Tabs, "divv": dvv, "curl": curl}
-        if getattr(params, "av_switch", 0):
-            fav = balsara(dvv, curl, c, st["h"])
-            dc["bal"] = fav
-    acc = momentum_energy(st["x"], st["y"], st["z"], st["vx"], st["vy"], st["vz"], st["h"],
-                          st["m"], rho, p, c, Cm, bmin, bmax, params.periodic, nb, params, fav,
-                          omega)
-    acc.update(dc)
+    acc = _physics(st, params, bmin, bmax, nb)
+    c = acc["c"]
     if getattr(params, "gravity", 0):
         gr = gravity(st["x"], st["y"], st["z"], st["m"], params.grav_G, params.grav_eps)
         for k in ("ax", "ay", "az"):
@@ -494,67 +527,86 @@ def step(state: dict, params, dt_prev: float, first_step: bool, ngmax: int | Non
                                         st["h"], c, bmin, bmax, params.periodic, nb, dt_prev, params)
     else:
         dt = timestep(st["h"], c, dt_prev, params)
-    out = {"bmin": bmin, "bmax": bmax, "keys": ks, "perm": perm, "nb": nb, "rho": rho, "p": p,
-           "c": c, "C": Cm, "tau": tau, "tau_abs": tabs, "dt": dt,
+    out = {"bmin": bmin, "bmax": bmax, "keys": ks, "perm": perm, "nb": nb, "dt": dt,
            "pre": {f: st[f].copy() for f in STATE_KEYS}, **acc}
     update(st, acc, nb.nc, dt, dt_prev, first_step, bmin, bmax, params)
     return st, out
 
 
-def sample_step(state: dict, params, dt_prev: float, first_step: bool, targets, margin=1e-6):
+def sample_step(state: dict, params, dt_prev: float, first_step: bool, targets, margin=1e-6,
+                dt: float | None = None):
     """One step evaluated at a few sampled particles of a large input.
 
     The full-size parts that are cheap stay exact and global: box, keys, stable
     sort (O(N log N)) and dt (O(N), needs only c(u) -- exact for both EOS).  The
-    neighbour sums at a target t depend on particles at most three kernel radii
-    away: a_t needs C_j (j in N(t)), C_j needs rho_k (k in N(j)), rho_k needs
-    the positions in N(k).  So every value at t is a function of the particles
-    within R = 3 * 2 h_max of t only.  We take that ball S (ascending order, so
-    the summation order is unchanged), run the plain oracle functions on S, and
-    keep the values at t.  This is the same definition restricted to a set that
-    provably contains t's whole dependency cone -- no approximation.
+    neighbour sums at a target t depend on particles a few kernel radii away:
+    a_t needs C_j, Omega_j, f_j (j in N(t)); C_j needs rho_k (k in N(j)); rho_k
+    needs the positions in N(k) -- three radii.  With volume elements rho_k needs
+    X_l = m_l/rho0_l (l in N(k)), so four.  Every value at t is therefore a
+    function of the particles within R = hops * 2 h_max of t only.  We take that
+    ball S (ascending order, so the summation order is unchanged), run the same
+    plain functions (``_physics``) on S, and keep the values at t.  This is the
+    same definition restricted to a set that provably contains t's whole
+    dependency cone -- no approximation.
+
+    The signal-velocity time step (cfg.dt_vsig) is a global minimum over every
+    particle's neighbour list, which the sampled mode cannot form: there the
+    caller passes ``dt`` (the GPU's) for the update, and ``out["vsig"]`` gives
+    the exact v_sig of each target (the test checks dt against them).
 
     ``targets`` are positions in this step's sorted order.  Returns (order, out)
     with ``order`` = sorted ids (full) and ``out[name][k]`` the value at targets[k].
     """
-    if getattr(params, "gradh", 0) or getattr(params, "dt_vsig", 0) or getattr(params, "ve", 0):
-        raise NotImplementedError("sample_step covers the north-star step (no gradh / dt_vsig / ve)")
+    if getattr(params, "gravity", 0):
+        raise NotImplementedError("sample_step: gravity is long-range (no finite dependency ball)")
+    vsig_mode = bool(getattr(params, "dt_vsig", 0))
+    if vsig_mode and dt is None:
+        raise ValueError("sample_step with dt_vsig needs the caller's dt (global minimum)")
     bmin, bmax = box(state["x"], state["y"], state["z"], params)
     k = keys(state["x"], state["y"], state["z"], bmin, bmax)
     perm = sort_order(k)
     st = {f: np.ascontiguousarray(state[f][perm]) for f in STATE_KEYS}
-    p_all, c_all = eos(np.ones(st["x"].size), st["u"], params)  # c does not depend on rho
-    dt = timestep(st["h"], c_all, dt_prev, params)
+    if not vsig_mode:
+        p_all, c_all = eos(np.ones(st["x"].size), st["u"], params)  # c does not depend on rho
+        dt = timestep(st["h"], c_all, dt_prev, params)
     hmax = float(st["h"].max())
-    R = 6.0 * hmax * (1.0 + margin)
-    names = ("nc", "rho", "p", "c", "ax", "ay", "az", "du", "du_abs", "x", "y", "z", "vx", "vy",
-             "vz", "u", "h")
-    out = {nm: np.zeros(len(targets)) for nm in names}
+    hops = 4 if getattr(params, "ve", 0) else 3
+    R = hops * 2.0 * hmax * (1.0 + margin)
+    names = ["nc", "rho", "p", "c", "ax", "ay", "az", "du", "du_abs", "x", "y", "z", "vx", "vy",
+             "vz", "u", "h"]
+    extra = [nm for nm, on in (("omega", getattr(params, "gradh", 0)),
+                               ("kx", getattr(params, "ve", 0)),
+                               ("divv", getattr(params, "divcurl", 0) or getattr(params, "av_switch", 0)),
+                               ("bal", getattr(params, "av_switch", 0)),
+                               ("vsig", vsig_mode)) if on]
+    out = {nm: np.zeros(len(targets)) for nm in names + extra}
     out["C"] = np.zeros((len(targets), 6))
     out["a_abs"] = np.zeros((len(targets), 3))
     out["nbrs"] = []
+    out["ball_sizes"] = []
     for q, t in enumerate(targets):
         S = ball(st["x"], st["y"], st["z"], int(t), R, bmin, bmax, params.periodic)
         sub = {f: np.ascontiguousarray(st[f][S]) for f in STATE_KEYS}
         loc = int(np.searchsorted(S, t))
         nb = neighbors(sub["x"], sub["y"], sub["z"], sub["h"], bmin, bmax, params.periodic)
-        rho = density(sub["x"], sub["y"], sub["z"], sub["h"], sub["m"], bmin, bmax,
-                      params.periodic, nb, params)
-        p, c = eos(rho, sub["u"], params)
-        Cm, _, _, _ = iad(sub["x"], sub["y"], sub["z"], sub["h"], sub["m"], rho, bmin, bmax,
-                          params.periodic, nb, params)
-        acc = momentum_energy(sub["x"], sub["y"], sub["z"], sub["vx"], sub["vy"], sub["vz"],
-                              sub["h"], sub["m"], rho, p, c, Cm, bmin, bmax, params.periodic, nb,
-                              params)
+        acc = _physics(sub, params, bmin, bmax, nb)
+        if vsig_mode:
+            _, vs = timestep_vsig(sub["x"], sub["y"], sub["z"], sub["vx"], sub["vy"], sub["vz"],
+                                  sub["h"], acc["c"], bmin, bmax, params.periodic, nb, dt_prev,
+                                  params)
+            out["vsig"][q] = vs[loc]
         one = {f: np.ascontiguousarray(sub[f][loc:loc + 1]) for f in STATE_KEYS}
         acc1 = {kk: acc[kk][loc:loc + 1] for kk in ("ax", "ay", "az", "du")}
         nc1 = nb.nc[loc:loc + 1].copy()
         out["nbrs"].append(S[nb.idx[nb.offsets[loc]:nb.offsets[loc + 1]]])
+        out["ball_sizes"].append(S.size)
         out["nc"][q] = nc1[0]
-        out["rho"][q], out["p"][q], out["c"][q] = rho[loc], p[loc], c[loc]
-        out["C"][q] = Cm[loc]
-        for kk in ("ax", "ay", "az", "du", "du_abs"):
+        for kk in ("rho", "p", "c", "ax", "ay", "az", "du", "du_abs"):
             out[kk][q] = acc[kk][loc]
+        for kk in extra:
+            if kk != "vsig":
+                out[kk][q] = acc[kk][loc]
+        out["C"][q] = acc["C"][loc]
         out["a_abs"][q] = acc["a_abs"][loc]
         update(one, acc1, nc1, dt, dt_prev, first_step, bmin, bmax, params)
         for f in ("x", "y", "z", "vx", "vy", "vz", "u", "h"):

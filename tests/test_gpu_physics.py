@@ -30,9 +30,14 @@ def test_sedov_blast_radius_and_energy(golden):
     E1 = _energy(st)
     # The scheme of the readings (no grad-h terms with variable h, a sound-speed
     # Courant condition) does not conserve energy through a strong shock: the
-    # ORACLE drifts +5.4% on Sedov 16^3 by t = 0.05 (reading 16), so the
-    # SURVEY's heuristic 1e-3 gate is replaced by 10%.
-    assert abs(E1 - E0) / E0 < 0.10, (E0, E1)
+    # ORACLE drifts +5.39% on Sedov 16^3 by t = 0.05 (measured,
+    # tests/golden/sedov16_drift.json; the GPU reproduces it to 1e-6 in
+    # test_sedov16_drift_matches_oracle).  At 40^3 the shock is resolved better
+    # and the drift is smaller; the gate is the oracle's 16^3 drift (not the
+    # SURVEY's heuristic 1e-3, which the scheme cannot meet).
+    import json, os
+    ref = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "sedov16_drift.json")))
+    assert abs(E1 - E0) / E0 < ref["drift"], (E0, E1, ref["drift"])
     rho = sim.get_field("rho")  # density of the last step's (pre-update) positions, same order
     r = np.sqrt(st["x"] ** 2 + st["y"] ** 2 + st["z"] ** 2)
     # shock position: the radius of the density peak, averaged over the shell of
@@ -44,6 +49,32 @@ def test_sedov_blast_radius_and_energy(golden):
     assert abs(R_num - R_th) / R_th < 0.12, (R_num, R_th, t, steps)
     # strong-shock compression: the peak density is well above ambient
     assert rho[top].mean() > 2.0
+
+
+def test_sedov16_drift_matches_oracle():
+    """The GPU Sedov 16^3 trajectory to t = 0.05 (89 steps) has the oracle's energy
+    drift (tests/golden/sedov16_drift.json, written by tools/golden_sedov_drift.py
+    from the oracle alone): same step count, t_end to 1e-9, drift to 1e-6."""
+    import json, os
+    from paper_conf_sc_simsekpc24_b200 import sph
+    ref = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "sedov16_drift.json")))
+    w = ics.sedov(16)
+    sim = sph.Simulation(w.params, n_capacity=w.n)
+    sim.set_particles({k: np.ascontiguousarray(v) for k, v in w.state.items()})
+    sim.set_time(0.0, w.params.dt_first, True)
+    E0 = _energy(w.state)
+    Es = [E0]
+    t = 0.0
+    for k in range(ref["steps"]):
+        t = sim.step()["t"]
+        Es.append(_energy(sim.get_state()))
+    sim.finalize()
+    assert abs(t / ref["t_end"] - 1) < 1e-9, (t, ref["t_end"])
+    assert abs(E0 / ref["E0"] - 1) < 1e-15
+    drift = Es[-1] / E0 - 1
+    assert abs(drift - ref["drift"]) < 1e-6, (drift, ref["drift"])
+    for a, b in zip(Es[::10], ref["E_every_10"]):
+        assert abs(a / b - 1) < 1e-6
 
 
 def test_noh_implosion_jumps():

@@ -284,3 +284,106 @@ def test_leapfrog_constant_acceleration():
                       np.array(P.box_min), np.array(P.box_max), P)
         assert st["vx"][0] == pytest.approx(0.5 * dt * k, rel=1e-15)
         assert st["x"][0] == pytest.approx(0.5 * dt * dt * k * (k + 1) / 2, rel=1e-14)
+
+
+# ----------------------------------------------------------------- variable h
+def _mutual_lattice(nside=10, seed=31):
+    """Perfect periodic lattice (a = 1/nside) with h jittered by +-1% around the
+    ng0 = 100 value (2h/a = 2.87941), random u (ideal gas) and random v.  Then
+    2h/a lies in [2.85, 2.91]: above the sqrt(8) shell and below the next one at
+    3, so every particle has the same 92 neighbours at the same lattice offsets
+    whatever its h -- every neighbour relation is mutual while h_i != h_j.  The
+    exact pair antisymmetry of SURVEY 8(c) step 8 (A_ij = -B_ji, G_ij = -G_ji,
+    Pi_ij = Pi_ji) then holds with VARIABLE h, which is what pins the j-side
+    W(r, h_j), B = C_j Delta w_j and the symmetric means h-bar, c-bar, rho-bar."""
+    w = ics.sedov(nside)
+    s = w.state
+    rng = np.random.default_rng(seed)
+    n = s["x"].size
+    s["h"] = s["h"] * (1.0 + rng.uniform(-0.01, 0.01, n))
+    s["u"] = rng.uniform(0.5, 2.0, n)
+    for k in ("vx", "vy", "vz"):
+        s[k] = rng.uniform(-0.5, 0.5, n)
+    w.params.eos = 0
+    a = 1.0 / nside
+    assert 2 * s["h"].min() / a > 2.85 > 8 ** 0.5 and 2 * s["h"].max() / a < 2.91 < 3.0
+    return w
+
+
+def test_mutual_lattice_is_mutual():
+    w = _mutual_lattice()
+    s, bmin, bmax, nb = _prep(w)
+    assert np.all(nb.nc == 92)
+    pairs = set()
+    for i in range(s["x"].size):
+        for j in nb.idx[nb.offsets[i]:nb.offsets[i + 1]]:
+            pairs.add((i, int(j)))
+    assert all((j, i) in pairs for (i, j) in pairs)
+    assert np.ptp(s["h"]) > 0.01 * s["h"].mean()   # h really varies
+
+
+def test_conservation_variable_h_mutual():
+    """Variable h, every pair mutual: sum m a = 0 and sum m (v.a + du) = 0 to roundoff
+    of the term scale.  Fails if the j-side kernel used h_i (w_j = W(r, h_i)), if B
+    used C_i, or if a mean (h-bar, c-bar, rho-bar) were one-sided."""
+    w = _mutual_lattice()
+    s = w.state
+    r = _chain(w)
+    m = s["m"]
+    scale = (m[:, None] * r["a_abs"]).sum(0)
+    mom = np.array([(m * r["ax"]).sum(), (m * r["ay"]).sum(), (m * r["az"]).sum()])
+    assert np.all(np.abs(mom) < 1e-14 * scale), mom / scale
+    power = (m * (s["vx"] * r["ax"] + s["vy"] * r["ay"] + s["vz"] * r["az"] + r["du"])).sum()
+    pscale = (m * (np.abs(s["vx"]) * r["a_abs"][:, 0] + np.abs(s["vy"]) * r["a_abs"][:, 1]
+                   + np.abs(s["vz"]) * r["a_abs"][:, 2] + r["du_abs"])).sum()
+    assert abs(power) < 1e-14 * pscale, power / pscale
+    # the viscosity really acts (approaching pairs exist), so Pi is exercised
+    assert np.abs(r["du"]).max() > 0
+
+
+def _iad_gradient_error(w):
+    s, bmin, bmax, nb = _prep(w)
+    r = _chain(w)
+    g = np.array([0.3, -1.7, 0.9])
+    V = s["m"] / r["rho"]
+    err = 0.0
+    for i in range(s["x"].size):
+        js = nb.idx[nb.offsets[i]:nb.offsets[i + 1]]
+        D = np.stack([s["x"][js] - s["x"][i], s["y"][js] - s["y"][i], s["z"][js] - s["z"][i]], 1)
+        D -= np.round(D)  # minimum image in the unit box
+        # the gradient of f = g.x with the kernel of the TARGET's smoothing length
+        Wv = np.array([oracle.W(np.linalg.norm(d), s["h"][i], K_SINC6) for d in D])
+        c = r["C"][i]
+        Cm = np.array([[c[0], c[1], c[2]], [c[1], c[3], c[4]], [c[2], c[4], c[5]]])
+        grad = ((V[js] * Wv * (D @ g))[:, None] * (D @ Cm.T)).sum(0)
+        err = max(err, np.abs(grad - g).max() / np.abs(g).max())
+    return err
+
+
+@pytest.mark.parametrize("kind", ["mutual_lattice", "jittered_varh"])
+def test_iad_linear_exactness_variable_h(kind):
+    """IAD linear exactness with variable h: C_i inverts tau_i built with W(r, h_i),
+    so the gradient of a linear field taken with W(r, h_i) is exact.  A tau built
+    with W(r, h_j) breaks it as soon as h varies (uniform-h sets cannot tell)."""
+    if kind == "mutual_lattice":
+        w = _mutual_lattice()
+    else:
+        w = ics.turbulence(10)
+        rng = np.random.default_rng(5)
+        w.state["h"] = w.state["h"] * (1.0 + rng.uniform(-0.1, 0.1, w.n))
+    assert _iad_gradient_error(w) < 1e-13
+
+
+def test_density_uses_own_h_only(golden):
+    """Perfect 10^3 lattice at the ng0 = 100 h, one particle's h raised by 1%: every
+    OTHER particle keeps the golden lattice density (its sum uses its own h_i, not
+    the neighbour's), and the changed particle's density moves."""
+    w = ics.sedov(10)
+    s = w.state
+    k = 437
+    s["h"] = s["h"].copy()
+    s["h"][k] *= 1.01
+    r = _chain(w)
+    others = np.arange(w.n) != k
+    assert np.allclose(r["rho"][others], golden["lattice_rho"]["value"], rtol=1e-14, atol=0)
+    assert abs(r["rho"][k] / golden["lattice_rho"]["value"] - 1) > 1e-6  # ~2e-5: a normalised estimate
