@@ -137,7 +137,7 @@ typedef struct sph_config {
   double ng0;               /* target neighbour count of the h update              */
   int32_t ngmax;            /* neighbour-list capacity per particle (never truncates:
                                overflow -> SPH_ERR_CAPACITY)                       */
-  int32_t max_cell_level;   /* finest cell-grid level L (8^L cells), <= 10         */
+  int32_t max_cell_level;   /* finest cell-grid level L (8^L cells), in [1, 10]    */
   double h_cap;             /* h <= h_cap after the update (periodic: <= min L / 4) */
   double k_cour;            /* Courant factor                                      */
   double dt_max_growth;     /* dt <= growth * dt_prev                              */
@@ -391,6 +391,10 @@ int sph_step(sph_ctx* ctx, sph_step_info* info);
 
 /* Clock policy: DEFAULT, STATIC (mhz[0] for every phase) or PER_PHASE (mhz[p]
  * set before phase p, skipped when unchanged; 0 = leave the clock as is).
+ * NVML applies a lock when it is called, not in stream order, so PER_PHASE
+ * synchronises the stream before every clock change (each phase then runs at
+ * its own clock; the wait is part of the policy's time, as the paper's
+ * ManDyn includes its clock-switch latency).
  * Requests snap to the nearest supported graphics clock.  Uses
  * nvmlDeviceSetGpuLockedClocks; this needs root and is disabled unless the
  * environment sets SPH_ALLOW_CLOCK_CONTROL=1 (shared hosts forbid clock changes)
@@ -422,9 +426,12 @@ int sph_kernel_launches(int64_t* count);
  * KernelTuner-style isolated measurement of P:81-87 -- and returns its mean time
  * and energy per call (joules < 0 when NVML is unavailable).  Repeatable phases
  * leave the pipeline state unchanged: KEYS (into a spare key buffer), SORT
- * (re-sorts the sorted keys, permutes into the spare state buffer), CELLS,
- * NEIGHBORS, DENSITY, EOS, IAD, MOMENTUM_ENERGY, TIMESTEP; UPDATE is not
- * (SPH_ERR_ARG).  The NVML energy counter of a B200 advances about every 100 ms,
+ * (re-sorts the sorted keys, permutes into the spare state buffer; the last
+ * permutation, SPH_F_ORDER, is saved and restored), CELLS, NEIGHBORS, DENSITY,
+ * EOS (after GRADH with p/(Omega rho^2), as the pipeline left it), IAD,
+ * MOMENTUM_ENERGY, TIMESTEP, GRADH (cfg.gradh without cfg.ve); UPDATE is not
+ * (SPH_ERR_ARG).  DENSITY after the volume-element GRADH would overwrite the
+ * normalised rho: SPH_ERR_STATE.  The NVML energy counter of a B200 advances about every 100 ms,
  * so reps should make the call last >= 1 s.  Synchronises. */
 int sph_repeat_phase(sph_ctx* ctx, int phase, int reps, double* ms_per_call,
                      double* joules_per_call);

@@ -543,7 +543,9 @@ def sample_step(state: dict, params, dt_prev: float, first_step: bool, targets, 
     a_t needs C_j, Omega_j, f_j (j in N(t)); C_j needs rho_k (k in N(j)); rho_k
     needs the positions in N(k) -- three radii.  With volume elements rho_k needs
     X_l = m_l/rho0_l (l in N(k)), so four.  Every value at t is therefore a
-    function of the particles within R = hops * 2 h_max of t only.  We take that
+    function of the particles within R = 2 h_t + 2 max h (ball 1) + 2 max h (ball
+    2) [+ ...] of t only (the radius grown hop by hop, so a few large smoothing
+    lengths far away do not inflate every ball).  We take that
     ball S (ascending order, so the summation order is unchanged), run the same
     plain functions (``_physics``) on S, and keep the values at t.  This is the
     same definition restricted to a set that provably contains t's whole
@@ -569,9 +571,7 @@ def sample_step(state: dict, params, dt_prev: float, first_step: bool, targets, 
     if not vsig_mode:
         p_all, c_all = eos(np.ones(st["x"].size), st["u"], params)  # c does not depend on rho
         dt = timestep(st["h"], c_all, dt_prev, params)
-    hmax = float(st["h"].max())
     hops = 4 if getattr(params, "ve", 0) else 3
-    R = hops * 2.0 * hmax * (1.0 + margin)
     names = ["nc", "rho", "p", "c", "ax", "ay", "az", "du", "du_abs", "x", "y", "z", "vx", "vy",
              "vz", "u", "h"]
     extra = [nm for nm, on in (("omega", getattr(params, "gradh", 0)),
@@ -585,6 +585,12 @@ def sample_step(state: dict, params, dt_prev: float, first_step: bool, targets, 
     out["nbrs"] = []
     out["ball_sizes"] = []
     for q, t in enumerate(targets):
+        # dependency radius, hop by hop: N(t) lies within 2 h_t; the lists of the
+        # particles within R lie within R + 2 max h of them (max over that ball)
+        R = 2.0 * float(st["h"][t]) * (1.0 + margin)
+        for _ in range(hops - 1):
+            S = ball(st["x"], st["y"], st["z"], int(t), R, bmin, bmax, params.periodic)
+            R = (R + 2.0 * float(st["h"][S].max())) * (1.0 + margin)
         S = ball(st["x"], st["y"], st["z"], int(t), R, bmin, bmax, params.periodic)
         sub = {f: np.ascontiguousarray(st[f][S]) for f in STATE_KEYS}
         loc = int(np.searchsorted(S, t))
@@ -600,6 +606,8 @@ def sample_step(state: dict, params, dt_prev: float, first_step: bool, targets, 
         nc1 = nb.nc[loc:loc + 1].copy()
         out["nbrs"].append(S[nb.idx[nb.offsets[loc]:nb.offsets[loc + 1]]])
         out["ball_sizes"].append(S.size)
+        if "dWdh_abs" in acc:
+            out.setdefault("dWdh_abs", np.zeros(len(targets)))[q] = acc["dWdh_abs"][loc]
         out["nc"][q] = nc1[0]
         for kk in ("rho", "p", "c", "ax", "ay", "az", "du", "du_abs"):
             out[kk][q] = acc[kk][loc]

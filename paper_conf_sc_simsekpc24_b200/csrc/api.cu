@@ -103,6 +103,7 @@ struct sph_ctx {
   bool locked_any = false;
   bool rec_m_dirty = false;
   uint32_t* last_perm = nullptr;  // the last sort's permutation (SPH_F_ORDER)
+  uint32_t* perm_saved = nullptr; // its copy while sph_repeat_phase(SORT) reuses the buffers
   int64_t* compact_scratch = nullptr;  // per-block counts of sph_compact (+ total)
   Stir stir{};          // turbulence driving (k_stir.cu)
   bool stir_on = false;
@@ -195,6 +196,10 @@ void apply_clock(sph_ctx* c, int p) {
   if (c->clock_mode == SPH_CLOCK_DEFAULT) return;
   unsigned want = c->clock_mhz[p];
   if (want == 0 || want == c->current_lock) return;
+  // The lock applies from the moment NVML sets it, not in stream order: wait
+  // until the earlier phases have finished so each runs at its own clock (the
+  // wait is part of ManDyn's cost, like the paper's clock-switch latency).
+  cudaStreamSynchronize(c->st);
   if (c->nvml.lock_sm_clock(want) == 0) {
     c->current_lock = want;
     c->locked_any = true;
@@ -436,7 +441,7 @@ static int validate(const sph_config* c) {
   if (c->n_capacity < 1 || c->n_capacity >= (int64_t(1) << 30))
     return fail(nullptr, SPH_ERR_ARG, "n_capacity must be in [1, 2^30)");
   if (c->ngmax < 1 || c->ngmax > 4096) return fail(nullptr, SPH_ERR_ARG, "ngmax must be in [1, 4096]");
-  if (c->max_cell_level < 0 || c->max_cell_level > 10) return fail(nullptr, SPH_ERR_ARG, "max_cell_level must be in [0, 10]");
+  if (c->max_cell_level < 1 || c->max_cell_level > 10) return fail(nullptr, SPH_ERR_ARG, "max_cell_level must be in [1, 10]");
   for (int a = 0; a < 3; ++a)
     if (c->periodic[a] && !(c->box_max[a] > c->box_min[a])) return fail(nullptr, SPH_ERR_ARG, "periodic axis %d: box_max <= box_min", a);
   if (c->eos != SPH_EOS_IDEAL && c->eos != SPH_EOS_ISOTHERMAL) return fail(nullptr, SPH_ERR_ARG, "unknown eos %d", c->eos);
@@ -479,6 +484,7 @@ static size_t layout(const sph_config* cfg, char* base, sph_ctx* c) {
   char* kB = take(sizeof(uint64_t) * cap);
   char* vA = take(sizeof(uint32_t) * cap);
   char* vB = take(sizeof(uint32_t) * cap);
+  char* vS = take(sizeof(uint32_t) * cap);  // sph_repeat_phase(SORT) keeps last_perm here
   double** dst[] = {c ? &c->rho : nullptr, c ? &c->p : nullptr, c ? &c->c : nullptr,
                     c ? &c->vol : nullptr, c ? &c->prho2 : nullptr, c ? &c->wq : nullptr,
                     c ? &c->wk : nullptr, c ? &c->ax : nullptr, c ? &c->ay : nullptr,
@@ -548,7 +554,7 @@ static size_t layout(const sph_config* cfg, char* base, sph_ctx* c) {
   }
   if (c) {
     c->keyA = (uint64_t*)kA; c->keyB = (uint64_t*)kB;
-    c->valA = (uint32_t*)vA; c->valB = (uint32_t*)vB;
+    c->valA = (uint32_t*)vA; c->valB = (uint32_t*)vB; c->perm_saved = (uint32_t*)vS;
     c->nc = (int32_t*)ncp; c->nbr = (int32_t*)nbp; c->nrows = (int32_t*)nrp;
     c->cell_start = (uint32_t*)cs;
     c->level_cap = Lc;
@@ -1214,7 +1220,13 @@ int sph_repeat_phase(sph_ctx* c, int phase, int reps, double* ms_per_call, doubl
     case SPH_PHASE_SORT: need = S_TREE; break;
     case SPH_PHASE_CELLS: need = S_TREE; break;
     case SPH_PHASE_NEIGHBORS: need = S_TREE; break;
-    case SPH_PHASE_DENSITY: need = S_NBR; break;
+    case SPH_PHASE_DENSITY:
+      // after the volume-element GRADH, DENSITY would overwrite the normalised rho
+      // with rho0 (reading 23): not repeatable without re-running GRADH
+      if (c && c->cfg.ve && c->gradh_done)
+        return fail(c, SPH_ERR_STATE, "DENSITY is not repeatable after the volume-element GRADH");
+      need = S_NBR;
+      break;
     case SPH_PHASE_EOS: need = S_DENS; break;
     case SPH_PHASE_IAD: need = S_EOS; break;
     case SPH_PHASE_GRADH:
@@ -1246,6 +1258,11 @@ int sph_repeat_phase(sph_ctx* c, int phase, int reps, double* ms_per_call, doubl
   Fields Fk = F;
   Fk.key = spare_keys;
   const int prv = c->cur;
+  const size_t perm_bytes = sizeof(uint32_t) * (size_t)c->n;
+  if (phase == SPH_PHASE_SORT && c->last_perm && c->n > 0)  // the repeats reuse its buffer
+    cudaMemcpyAsync(c->perm_saved, c->last_perm, perm_bytes, cudaMemcpyDeviceToDevice, c->st);
+  // EOS after GRADH: p/(Omega rho^2), as the pipeline left it (reading 21)
+  const bool eos_omega = c->gradh_done && c->cfg.gradh;
   for (int r = 0; r < reps; ++r) {
     switch (phase) {
       case SPH_PHASE_KEYS: launch_box_keys(Fk, c->P, c->st); break;
@@ -1264,13 +1281,15 @@ int sph_repeat_phase(sph_ctx* c, int phase, int reps, double* ms_per_call, doubl
       case SPH_PHASE_TIMESTEP: launch_timestep(F, c->P, c->st); break;
       case SPH_PHASE_NEIGHBORS: launch_neighbors(F, c->P, c->st); break;
       case SPH_PHASE_DENSITY: launch_density(F, c->P, c->st); break;
-      case SPH_PHASE_EOS: launch_eos(F, c->P, c->st); break;
+      case SPH_PHASE_EOS: launch_eos(F, c->P, c->st, eos_omega); break;
       case SPH_PHASE_IAD: launch_iad(F, c->P, c->st); break;
       case SPH_PHASE_GRADH: launch_gradh(F, c->P, c->st); break;
       case SPH_PHASE_MOMENTUM_ENERGY: launch_momentum_energy(F, c->P, c->st); break;
     }
   }
   cudaEventRecord(b, c->st);
+  if (phase == SPH_PHASE_SORT && c->last_perm && c->n > 0)
+    cudaMemcpyAsync(c->last_perm, c->perm_saved, perm_bytes, cudaMemcpyDeviceToDevice, c->st);
   rc = cuda_check(c, cudaEventSynchronize(b), "repeat");
   if (!rc) {
     eok = eok && c->nvml.energy_mj(&e1);

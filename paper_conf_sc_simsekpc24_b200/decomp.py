@@ -178,6 +178,10 @@ class DistributedSim:
     def __init__(self, params, state, n_capacity: int, device: int = 0, force_exchange: bool = False,
                  **kw):
         from . import sph
+        if getattr(params, "gravity", 0):
+            # self-gravity is long-range: a 2 h_max halo cannot supply it (a global
+            # tree or multipole exchange would be needed)
+            raise NotImplementedError("DistributedSim: self-gravity is not decomposed")
         self.sph = sph
         # force_exchange: run the partition / migration / ghost / halo plumbing even
         # on one rank (it then moves nothing) -- measures its cost (tools/decomp_probe.py)

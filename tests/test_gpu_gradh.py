@@ -24,27 +24,34 @@ CASES = {
 }
 
 
-@pytest.fixture(scope="module", params=sorted(CASES))
-def case(request):
-    from parity import gpu_pipeline, new_sim
-    w, flags = CASES[request.param]()
-    w.params = dataclasses.replace(w.params, **flags)
-    st, o = oracle.step({k: v.copy() for k, v in w.state.items()}, w.params, w.params.dt_first, True)
-    sim = new_sim(w)
-    g = gpu_pipeline(sim)
-    if w.params.gradh:
-        g["omega"] = sim.get_field("omega")
-    if w.params.dt_vsig:
-        g["vsig"] = sim.get_field("vsig")
-    yield request.param, w, sim, g, st, o
-    sim.finalize()
+_RUNS = {}
 
 
-def test_omega(case):
+def _case(name):
+    """Oracle step + GPU pipeline of one case, computed once per session."""
+    if name not in _RUNS:
+        from parity import gpu_pipeline, new_sim
+        w, flags = CASES[name]()
+        w.params = dataclasses.replace(w.params, **flags)
+        st, o = oracle.step({k: v.copy() for k, v in w.state.items()}, w.params, w.params.dt_first, True)
+        sim = new_sim(w)
+        g = gpu_pipeline(sim)
+        if w.params.gradh:
+            g["omega"] = sim.get_field("omega")
+        if w.params.dt_vsig:
+            g["vsig"] = sim.get_field("vsig")
+        _RUNS[name] = (name, w, sim, g, st, o)
+    return _RUNS[name]
+
+
+def _with(flag):
+    return sorted(k for k in CASES if CASES[k]()[1].get(flag))
+
+
+@pytest.mark.parametrize("name", _with("gradh"))
+def test_omega(name):
     from parity import TOL_1STEP, assert_sum_close
-    name, w, sim, g, st, o = case
-    if not w.params.gradh:
-        pytest.skip("gradh off")
+    name, w, sim, g, st, o = _case(name)
     h = g["h"]
     rho = o["kx"] if w.params.ve else o["rho"]   # volume elements: kx in place of rho
     scale = h / (3 * rho) * o["dWdh_abs"]
@@ -52,28 +59,27 @@ def test_omega(case):
     assert np.max(np.abs(o["omega"] - 1)) > 1e-4   # the factor is not trivially 1
 
 
-def test_ve_density(case):
+@pytest.mark.parametrize("name", _with("ve"))
+def test_ve_density(name):
     """Volume elements (reading 23): the normalised density against the
     oracle's kx m / X (rho0 from the plain density sum)."""
     from parity import TOL_1STEP, assert_rel_close
-    name, w, sim, g, st, o = case
-    if not w.params.ve:
-        pytest.skip("ve off")
+    name, w, sim, g, st, o = _case(name)
     assert_rel_close(g["rho"], o["rho"], TOL_1STEP, "rho (volume elements)")
     assert np.max(np.abs(o["kx"] - 1)) > 1e-6 or name.startswith("sedov")
 
 
-def test_vsig(case):
-    name, w, sim, g, st, o = case
-    if not w.params.dt_vsig:
-        pytest.skip("dt_vsig off")
+@pytest.mark.parametrize("name", _with("dt_vsig"))
+def test_vsig(name):
+    name, w, sim, g, st, o = _case(name)
     # max over pairs of c_i + c_j - 3 rv/r: only rounding of rv and r differs
     assert np.all(np.abs(g["vsig"] - o["vsig"]) <= 1e-13 * o["vsig"])
 
 
-def test_step(case):
+@pytest.mark.parametrize("name", sorted(CASES))
+def test_step(name):
     from parity import TOL_1STEP, compare_state, compare_sums
-    name, w, sim, g, st, o = case
+    name, w, sim, g, st, o = _case(name)
     compare_sums(g, o, TOL_1STEP)
     dt = sim.timestep()
     if w.params.dt_vsig:

@@ -1,7 +1,9 @@
 """Physics of the GPU step over many steps (SURVEY 8(c) pins "Sedov", "Noh" and
 'Integrator'): the Sedov blast radius follows the similarity solution
-R(t) = xi0 (E t^2 / rho0)^(1/5), xi0 = 1.1517 for gamma = 5/3, and total energy
-sum m (v^2/2 + u) is conserved to 1e-3 over the run."""
+R(t) = xi0 (E t^2 / rho0)^(1/5), xi0 = 1.1517 for gamma = 5/3, and the total
+energy sum m (v^2/2 + u) follows the ORACLE's measured curve (the scheme drifts
++5-7% through the shock, reading 16, so SURVEY's heuristic 1e-3 gate
+is replaced by agreement with the oracle's own trajectory)."""
 import numpy as np
 import pytest
 
@@ -14,31 +16,64 @@ def _energy(st):
     return float((st["m"] * (0.5 * (st["vx"] ** 2 + st["vy"] ** 2 + st["vz"] ** 2) + st["u"])).sum())
 
 
-def test_sedov_blast_radius_and_energy(golden):
+def _gpu_sedov(nside, steps):
+    """GPU Sedov nside^3 for `steps` sph_step calls: (t, energies per step, state, rho)."""
+    from paper_conf_sc_simsekpc24_b200 import sph
+    w = ics.sedov(nside)
+    sim = sph.Simulation(w.params, n_capacity=w.n)
+    sim.set_particles({k: np.ascontiguousarray(v) for k, v in w.state.items()})
+    sim.set_time(0.0, w.params.dt_first, True)
+    Es = [_energy(w.state)]
+    t = 0.0
+    for _ in range(steps):
+        t = sim.step()["t"]
+        Es.append(_energy(sim.get_state()))
+    st = sim.get_state()
+    rho = sim.get_field("rho")  # density of the last step's (pre-update) positions, same order
+    sim.finalize()
+    return t, Es, st, rho
+
+
+def _golden_drift(nside):
+    import json, os
+    return json.load(open(os.path.join(os.path.dirname(__file__), "golden", f"sedov{nside}_drift.json")))
+
+
+@pytest.mark.parametrize("nside", [16, 32])
+def test_sedov_drift_matches_oracle(nside):
+    """The scheme of the readings (no grad-h terms with variable h, a sound-speed
+    Courant step) does not conserve energy through a strong shock: the ORACLE
+    gains 5.39% (16^3) and 6.85% (32^3) of total energy by t = 0.05
+    (tests/golden/sedov{16,32}_drift.json, written by tools/golden_sedov_drift.py
+    from the oracle alone; reading 16).  The GPU trajectory has the same
+    step count, t_end to 1e-9, and the oracle's energy curve to 1e-6."""
+    ref = _golden_drift(nside)
+    t, Es, st, rho = _gpu_sedov(nside, ref["steps"])
+    assert abs(t / ref["t_end"] - 1) < 1e-9, (t, ref["t_end"])
+    assert abs(Es[0] / ref["E0"] - 1) < 1e-15
+    drift = Es[-1] / Es[0] - 1
+    assert abs(drift - ref["drift"]) < 1e-6, (drift, ref["drift"])
+    for a, b in zip(Es[::10], ref["E_every_10"]):
+        assert abs(a / b - 1) < 1e-6
+
+
+def test_sedov_blast_radius(golden):
+    """Sedov 40^3 to t = 0.05: the shock sits at the similarity radius
+    R(t) = xi0 (E t^2 / rho0)^(1/5), xi0 = 1.1517 (gamma = 5/3), within 12%, and
+    the shell is compressed.  (Its energy is the oracle's, checked at 16^3 and
+    32^3 in test_sedov_drift_matches_oracle; the oracle is too slow at 40^3.)"""
     from paper_conf_sc_simsekpc24_b200 import sph
     w = ics.sedov(40)
     sim = sph.Simulation(w.params, n_capacity=w.n)
     sim.set_particles({k: np.ascontiguousarray(v) for k, v in w.state.items()})
     sim.set_time(0.0, w.params.dt_first, True)
-    E0 = _energy(w.state)
-    t = 0.0
-    steps = 0
+    t, steps = 0.0, 0
     while t < 0.05 and steps < 2000:
         t = sim.step()["t"]
         steps += 1
     st = sim.get_state()
-    E1 = _energy(st)
-    # The scheme of the readings (no grad-h terms with variable h, a sound-speed
-    # Courant condition) does not conserve energy through a strong shock: the
-    # ORACLE drifts +5.39% on Sedov 16^3 by t = 0.05 (measured,
-    # tests/golden/sedov16_drift.json; the GPU reproduces it to 1e-6 in
-    # test_sedov16_drift_matches_oracle).  At 40^3 the shock is resolved better
-    # and the drift is smaller; the gate is the oracle's 16^3 drift (not the
-    # SURVEY's heuristic 1e-3, which the scheme cannot meet).
-    import json, os
-    ref = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "sedov16_drift.json")))
-    assert abs(E1 - E0) / E0 < ref["drift"], (E0, E1, ref["drift"])
-    rho = sim.get_field("rho")  # density of the last step's (pre-update) positions, same order
+    rho = sim.get_field("rho")
+    sim.finalize()
     r = np.sqrt(st["x"] ** 2 + st["y"] ** 2 + st["z"] ** 2)
     # shock position: the radius of the density peak, averaged over the shell of
     # the 200 densest particles
@@ -46,35 +81,9 @@ def test_sedov_blast_radius_and_energy(golden):
     R_num = float(np.median(r[top]))
     xi0 = golden["sedov_xi0_gamma53"]["value"]
     R_th = xi0 * (1.0 * t * t / 1.0) ** 0.2
-    assert abs(R_num - R_th) / R_th < 0.12, (R_num, R_th, t, steps)
+    assert abs(R_num - R_th) / R_th < 0.12, (R_num, R_th, t)
     # strong-shock compression: the peak density is well above ambient
     assert rho[top].mean() > 2.0
-
-
-def test_sedov16_drift_matches_oracle():
-    """The GPU Sedov 16^3 trajectory to t = 0.05 (89 steps) has the oracle's energy
-    drift (tests/golden/sedov16_drift.json, written by tools/golden_sedov_drift.py
-    from the oracle alone): same step count, t_end to 1e-9, drift to 1e-6."""
-    import json, os
-    from paper_conf_sc_simsekpc24_b200 import sph
-    ref = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "sedov16_drift.json")))
-    w = ics.sedov(16)
-    sim = sph.Simulation(w.params, n_capacity=w.n)
-    sim.set_particles({k: np.ascontiguousarray(v) for k, v in w.state.items()})
-    sim.set_time(0.0, w.params.dt_first, True)
-    E0 = _energy(w.state)
-    Es = [E0]
-    t = 0.0
-    for k in range(ref["steps"]):
-        t = sim.step()["t"]
-        Es.append(_energy(sim.get_state()))
-    sim.finalize()
-    assert abs(t / ref["t_end"] - 1) < 1e-9, (t, ref["t_end"])
-    assert abs(E0 / ref["E0"] - 1) < 1e-15
-    drift = Es[-1] / E0 - 1
-    assert abs(drift - ref["drift"]) < 1e-6, (drift, ref["drift"])
-    for a, b in zip(Es[::10], ref["E_every_10"]):
-        assert abs(a / b - 1) < 1e-6
 
 
 def test_noh_implosion_jumps():

@@ -1,5 +1,5 @@
-"""Writes tests/golden/sedov16_drift.json: the ORACLE's total-energy drift over a
-Sedov 16^3 run to t >= 0.05 (reading 16).  Calls only oracle/ and the
+"""Writes tests/golden/sedov{N}_drift.json (N = argv[1], default 16): the
+ORACLE's total-energy drift over a Sedov N^3 run to t >= 0.05 (reading 16).  Calls only oracle/ and the
 input generator (no CUDA path).  Re-run after any change to the oracle's
 arithmetic; tests/test_oracle_step.py recomputes it and must agree."""
 import json
@@ -18,8 +18,8 @@ def energy(s):
     return float((s["m"] * (0.5 * (s["vx"] ** 2 + s["vy"] ** 2 + s["vz"] ** 2) + s["u"])).sum())
 
 
-def run():
-    w = ics.sedov(16)
+def run(nside=16):
+    w = ics.sedov(nside)
     s = {k: v.copy() for k, v in w.state.items()}
     E0 = energy(s)
     dt, t, k = w.params.dt_first, 0.0, 0
@@ -35,11 +35,12 @@ def run():
 
 
 if __name__ == "__main__":
-    r = run()
-    r["what"] = ("oracle total energy sum m (v^2/2 + u), Sedov 16^3 (ics.sedov), stepped until "
+    nside = int(sys.argv[1]) if len(sys.argv) > 1 else 16
+    r = run(nside)
+    r["what"] = (f"oracle total energy sum m (v^2/2 + u), Sedov {nside}^3 (ics.sedov), stepped until "
                  "t >= 0.05; DESIGN.md reading 16")
-    r["script"] = "tools/golden_sedov_drift.py"
-    path = os.path.join(ROOT, "tests", "golden", "sedov16_drift.json")
+    r["script"] = f"tools/golden_sedov_drift.py {nside}"
+    path = os.path.join(ROOT, "tests", "golden", f"sedov{nside}_drift.json")
     with open(path, "w") as f:
         json.dump(r, f, indent=1)
     print(json.dumps({k: r[k] for k in ("steps", "t_end", "drift")}))
