@@ -35,13 +35,19 @@ sys.path.insert(0, ROOT)
 METRIC = "particle-updates/s per SPH step"
 UNIT = "particle-updates/s"
 
-# Algorithmic FP64 flops per neighbour pair, counting
-# add/sub/mul as 1 and fma as 2, sinc as its 10-FMA polynomial; the artificial
-# viscosity's flops (approaching pairs only) are NOT counted (lower bound).
-FLOPS_PER_PAIR = {"density": 34, "iad": 49, "momentum_energy": 145}
-# FP64 peak: 148 SMs x 64 FP64 FMA/clk x 2 flop x 1.965 GHz (guide's SM count and
-# max SM clock; DFMA microbenchmark measured 34.1 TF, tools/probe_fp64.cu).
+# Algorithmic FP64 flops per neighbour pair: SURVEY.md 8(d)'s counts (density
+# 44, IAD 60, momentum-energy 171 incl. the artificial viscosity), the figures
+# the roofline fractions are quoted against.  The DP
+# instructions the kernels actually execute are counted by ncu
+# (profiles/r02_dp_counts.json, 2 x DFMA + DMUL + DADD per pair) and reported
+# beside them.
+FLOPS_PER_PAIR = {"density": 44, "iad": 60, "momentum_energy": 171}
+# FP64 peak: 148 SMs x 64 FP64 FMA/clk x 2 flop x 1.965 GHz, DERIVED from the
+# guide's SM count and max SM clock (B200_PROFILING.md; MEASURED_PEAKS.json has
+# no FP64 figure).  A DFMA microbenchmark on this B200 measured 34.1 TF/s
+# (tools/probe_fp64.cu, profiles/r01_probe_fp64.json).
 FP64_PEAK_TFLOPS = 148 * 64 * 2 * 1.965e9 / 1e12
+FP64_PEAK_MEASURED_TFLOPS = 34.082
 # Algorithmic HBM bytes per particle of the momentum-energy launch (i-side fields
 # once, neighbour list once, outputs once): 19 doubles + nc + 4 B per neighbour + 4 doubles.
 MOM_BYTES_PER_PARTICLE = 19 * 8 + 4 + 4 * 8   # + 4 * nc
@@ -118,8 +124,13 @@ def parse():
     ap.add_argument("--workload", default="turbulence200")
     ap.add_argument("--impl", default="libsph", choices=["libsph", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
-    ap.add_argument("--energy-steps", type=int, default=60,
-                    help="steps for the whole-step energy (>= ~2 s: the counter ticks every ~100 ms)")
+    ap.add_argument("--energy-seconds", type=float, default=10.0,
+                    help="length of each energy window (the NVML counter ticks every ~100 ms / "
+                         "~99 J on a B200: >= 10 s keeps a window within ~1%%); 0 = no energy")
+    ap.add_argument("--energy-repeats", type=int, default=3,
+                    help="whole-step energy windows (median and CV)")
+    ap.add_argument("--timing-repeats", type=int, default=3,
+                    help="extra blocks of --steps timed steps after the contract's block (median, CV)")
     ap.add_argument("--av-switch", action="store_true",
                     help="IADVelocityDivCurl div/curl + Balsara AV switch (SURVEY 8(f)-1)")
     ap.add_argument("--gradh", action="store_true",
@@ -225,39 +236,103 @@ def cpu_baseline(w, n_targets: int, seed: int = 3):
     return n_targets / dt, dt, threads
 
 
-def measure_energy(sim, sph, n, args, gpu_index):
-    """Per-step and per-phase energy from the NVML total-energy counter.
+def _cv(xs):
+    return statistics.pstdev(xs) / statistics.mean(xs) if len(xs) > 1 and statistics.mean(xs) else 0.0
 
-    The B200 counter advances about every 100 ms (tools/probe_nvml.py), far
-    coarser than a phase (0.01-14 ms), so energy is never read at phase edges:
-      * step: counter delta over `energy_steps` back-to-back steps (no syncs);
-      * phase: the KernelTuner-style isolated repetition of P:81-87 -- each
-        repeatable phase re-run on the same inputs for ~1.5 s (sph_repeat_phase),
-        with the SM clock sampled meanwhile (the DVFS clock of Fig. 9, P:208-220);
-      * update (not repeatable: it advances the state): time x step-average power.
+
+def cpu_physics_only(w, m: int = 32768):
+    """SURVEY 8(d)'s fair per-kernel CPU baseline: the oracle's physics only
+    (density, EOS, IAD, momentum-energy), GIVEN the neighbour lists, per
+    particle -- on the first m particles of the workload in Morton order (a
+    compact block; lists from the oracle's brute force, not timed)."""
+    import numpy as np
+    import oracle
+    s = w.state
+    bmin, bmax = oracle.box(s["x"], s["y"], s["z"], w.params)
+    k = oracle.keys(s["x"], s["y"], s["z"], bmin, bmax)
+    sel = oracle.sort_order(k)[:min(m, w.n)]
+    st = {f: np.ascontiguousarray(s[f][sel]) for f in oracle.STATE_KEYS}
+    nb = oracle.neighbors(st["x"], st["y"], st["z"], st["h"], bmin, bmax, w.params.periodic)
+    P = w.params
+    t0 = time.perf_counter()
+    rho = oracle.density(st["x"], st["y"], st["z"], st["h"], st["m"], bmin, bmax, P.periodic, nb, P)
+    p, c = oracle.eos(rho, st["u"], P)
+    Cm, _, _, _ = oracle.iad(st["x"], st["y"], st["z"], st["h"], st["m"], rho, bmin, bmax, P.periodic, nb, P)
+    oracle.momentum_energy(st["x"], st["y"], st["z"], st["vx"], st["vy"], st["vz"], st["h"], st["m"], rho, p, c,
+                           Cm, bmin, bmax, P.periodic, nb, P)
+    dt = time.perf_counter() - t0
+    return {"s_per_particle": dt / sel.size, "particle_updates_per_s": sel.size / dt, "particles": int(sel.size),
+            "mean_nc": float(nb.nc.mean()), "seconds": dt,
+            "what": "oracle density+EOS+IAD+momentum-energy given the neighbour lists (C, OpenMP over targets)"}
+
+
+def measure_energy(sim, sph, n, args, gpu_index, ms_off):
+    """Per-step and per-phase energy at default DVFS clocks.
+
+    * Whole step, in situ: `energy_repeats` windows of >= `energy_seconds` of
+      back-to-back steps with PHASE accounting on (no phase-edge syncs: a host
+      thread integrates the NVML instant power per device-tagged phase).  Per
+      window: J/step from the NVML total-energy counter, the sampled integral of
+      P dt (the accounting's self-check: counter vs integral), the sum of the
+      per-phase joules, and the accounting's time overhead vs OFF.  The instant
+      power refreshes every ~100 ms on a B200, so in-situ per-phase joules are
+      TIME-APPORTIONED (each phase's device time at the power around it).
+    * Per phase, isolated: the KernelTuner-style repetition of P:81-87 -- each
+      repeatable phase re-run on the same inputs for >= `energy_seconds`
+      (sph_repeat_phase; counter delta / reps), with the SM clock sampled
+      meanwhile (Fig. 9's DVFS clock).  UPDATE (not repeatable: it advances the
+      state) takes time x the step's average power.
     """
     import torch
     torch.cuda.synchronize()
-    e0 = sim.energy_counter_mj()
-    if e0 is None:
+    if sim.energy_counter_mj() is None:
         return {"available": False, "why": "NVML energy counter unavailable"}
-    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    k = args.energy_steps
-    with ClockSampler(gpu_index) as clk:
-        ev0.record(sim.stream)
-        for _ in range(k):
-            sim.step()
-        ev1.record(sim.stream)
-        torch.cuda.synchronize()
-    e1 = sim.energy_counter_mj()
-    step_ms = ev0.elapsed_time(ev1) / k
-    step_J = (e1 - e0) * 1e-3 / k
-    out = {"available": True, "counter": "nvmlDeviceGetTotalEnergyConsumption (mJ, ~100 ms update)",
+    T = args.energy_seconds
+    windows = []
+    insitu = None
+    for r in range(max(args.energy_repeats, 1)):
+        sim.set_accounting(sph.ACCOUNTING_PHASE)
+        sim.energy_reset()
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with ClockSampler(gpu_index) as clk:
+            t0 = time.perf_counter()
+            ev0.record(sim.stream)
+            k = 0
+            while time.perf_counter() - t0 < T:
+                sim.step()
+                k += 1
+            ev1.record(sim.stream)
+            torch.cuda.synchronize()
+        tot = sim.energy_totals()
+        rows = sim.energy_report()
+        sim.set_accounting(sph.ACCOUNTING_OFF)
+        ms = ev0.elapsed_time(ev1) / k
+        cj = tot["counter_joules"]
+        ph = {x["name"]: x["joules"] / k for x in rows if x["calls"] and x["joules"] is not None}
+        windows.append({"steps": k, "seconds": tot["wall_seconds"], "ms_per_step": ms,
+                        "J_per_step_counter": cj / k if cj is not None else None,
+                        "J_per_step_sampled": tot["sampled_joules"] / k,
+                        "counter_over_sampled": (cj / tot["sampled_joules"]) if cj and tot["sampled_joules"] else None,
+                        "phase_J_sum_over_step": (sum(ph.values()) / (cj / k)) if cj else None,
+                        "between_phases_J_per_step": tot["between_joules"] / k,
+                        "overhead_pct_vs_off": 100.0 * (ms / ms_off - 1.0),
+                        "clocks": clk.summary()})
+        if r == 0:
+            insitu = ph
+    step_J = [w["J_per_step_counter"] for w in windows if w["J_per_step_counter"] is not None]
+    step_ms = [w["ms_per_step"] for w in windows]
+    J = statistics.median(step_J)
+    out = {"available": True,
+           "counter": "nvmlDeviceGetTotalEnergyConsumption (mJ, ~100 ms / ~99 J update)",
+           "power_sensor": "NVML_FI_DEV_POWER_INSTANT, refreshed ~every 100 ms (profiles/r02_probe_nvml_instant.json)",
            "clock_policy": ("default DVFS: SM clock locking is implemented (sph_set_clock_policy) but "
                             "not exercised -- this shared host forbids clock changes"),
-           "step": {"steps": k, "J": step_J, "ms": step_ms, "W": step_J / (step_ms * 1e-3),
-                    "clocks": clk.summary()},
-           "uJ_per_particle_update": step_J / n * 1e6, "phases": {}}
+           "step": {"windows": windows, "J_median": J, "J_cv": _cv(step_J), "ms_median": statistics.median(step_ms),
+                    "W": J / (statistics.median(step_ms) * 1e-3)},
+           "uJ_per_particle_update": J / n * 1e6,
+           "in_situ_phase_J_per_step": {"kind": "time-apportioned (PHASE accounting, sampled P dt per device-tagged phase)",
+                                        "J": insitu},
+           "phases": {}}
     # one more step, stopped before the update so every repeatable phase has its inputs
     sim.build_tree()
     sim.find_neighbors(stats=False)
@@ -271,43 +346,18 @@ def measure_energy(sim, sph, n, args, gpu_index):
     for ph in ("keys", "sort", "cells", "neighbors", "density", "eos") + (("gradh",) if sim.cfg.gradh and not sim.cfg.ve else ()) + (
             "iad", "momentum_energy", "timestep"):
         ms1, _ = sim.repeat_phase(ph, 3)
-        reps = int(min(200000, max(5, 1500.0 / max(ms1, 1e-4))))
+        reps = int(min(2000000, max(5, 1e3 * T / max(ms1, 1e-4))))
         with ClockSampler(gpu_index) as c2:
-            ms, J = sim.repeat_phase(ph, reps)
-        out["phases"][ph] = {"ms": ms, "J": J, "W": (J / (ms * 1e-3)) if J else None, "reps": reps,
-                             "sm_mhz": c2.summary().get("sm_mhz")}
+            ms, Jp = sim.repeat_phase(ph, reps)
+        out["phases"][ph] = {"ms": ms, "J": Jp, "W": (Jp / (ms * 1e-3)) if Jp else None, "reps": reps,
+                             "window_s": ms * reps * 1e-3, "sm_mhz": c2.summary().get("sm_mhz")}
     sim.update()
     ms_upd = sim.step()["phase_ms"]["update"]
-    out["phases"]["update"] = {"ms": ms_upd, "J": ms_upd * 1e-3 * out["step"]["W"], "W": out["step"]["W"],
+    W = out["step"]["W"]
+    out["phases"]["update"] = {"ms": ms_upd, "J": ms_upd * 1e-3 * W, "W": W,
                                "reps": 0, "note": "not repeatable; step-average power x time"}
-    out["phase_J_sum_vs_step"] = (sum(p["J"] or 0.0 for p in out["phases"].values()) / step_J)
+    out["repeat_phase_J_sum_over_step"] = sum(p["J"] or 0.0 for p in out["phases"].values()) / J
     return out
-
-
-def in_situ_accounting(sim, sph, steps, ms_off):
-    """The paper's in-situ instrumentation (energy "from the start of each
-    function call until its completion"): SPH_ACCOUNTING_PHASE syncs the stream
-    and reads the NVML counter at every phase edge.  Reports the step time it
-    costs against accounting OFF and the per-phase joules it apportions -- with
-    a ~100 ms counter tick these are coarse (reading 12); the
-    KernelTuner-style numbers of measure_energy are the clean ones."""
-    import torch
-    sim.set_accounting(sph.ACCOUNTING_PHASE)
-    sim.energy_reset()
-    torch.cuda.synchronize()
-    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    ev0.record(sim.stream)
-    for _ in range(steps):
-        sim.step()
-    ev1.record(sim.stream)
-    torch.cuda.synchronize()
-    rows = sim.energy_report()
-    sim.set_accounting(sph.ACCOUNTING_OFF)
-    ms = ev0.elapsed_time(ev1) / steps
-    ph = {r["name"]: (r["joules"] / steps if r["joules"] is not None else None) for r in rows if r["calls"]}
-    tot = sum(v for v in ph.values() if v) if ph else None
-    return {"mode": "phase", "steps": steps, "ms_per_step": ms, "ms_per_step_off": ms_off,
-            "overhead_pct": 100.0 * (ms / ms_off - 1.0), "J_per_step": tot, "phase_J_per_step": ph}
 
 
 def dvfs_trace(sim, sph, seconds):
@@ -517,6 +567,20 @@ def main():
         barrier()
     launches = sph.kernel_launches() - launches0
     ms = ev0.elapsed_time(ev1)
+    # >= 3 repeats, median and CV (extra blocks of K steps, after
+    # the contract's timed block, which alone gives `value`)
+    rep_ms = [ms / args.steps]
+    for _ in range(max(args.timing_repeats, 0)):
+        r0, r1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        barrier()
+        r0.record(stream)
+        for _ in range(args.steps):
+            sim.step()
+        r1.record(stream)
+        barrier()
+        rep_ms.append(r0.elapsed_time(r1) / args.steps)
+    repeats = {"blocks": len(rep_ms), "steps_per_block": args.steps, "ms_per_step": rep_ms,
+               "median": statistics.median(rep_ms), "cv": _cv(rep_ms)}
     ms_t = torch.tensor([ms], device="cuda")
     if world > 1:
         dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
@@ -535,19 +599,40 @@ def main():
             traffic = json.load(f)["momentum_energy_kernel"]["dram_bytes_per_launch"]
     except (OSError, KeyError, ValueError):
         pass
+    dp = {}
+    try:
+        with open(os.path.join(ROOT, "profiles", "r02_dp_counts.json")) as f:
+            dp = json.load(f)["kernels"]
+    except (OSError, KeyError, ValueError):
+        pass
+
+    def counted(kernel, t):
+        c = dp.get(kernel)
+        if not c:
+            return None
+        fl = c["dp_flops_per_pair"] * pairs / t / 1e12
+        return {"dp_flops_per_pair": c["dp_flops_per_pair"], "tflops": fl, "frac": fl / FP64_PEAK_TFLOPS,
+                "source": "ncu sm__sass_thread_inst_executed_op_{dfma,dmul,dadd}_pred_on (profiles/r02_dp_counts.json)"}
+
     roofline = {"bound": "alu", "achieved": achieved, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
                 "frac": achieved / FP64_PEAK_TFLOPS, "traffic": traffic,
                 "traffic_unit": "DRAM bytes per launch (ncu --set full, profiles/ncu_traffic.json)",
                 "algorithmic_bytes_per_launch": (MOM_BYTES_PER_PARTICLE + 4 * mean_nc) * n,
                 "kernel": "momentum_energy_kernel",
-                "peak_source": "148 SM x 64 DFMA/clk x 2 x 1.965 GHz (FP64 pipe; DESIGN.md 6)",
+                "flops_per_pair": FLOPS_PER_PAIR["momentum_energy"],
+                "flops_source": "SURVEY.md 8(d) algorithmic count (171 per pair incl. the AV)",
+                "peak_source": "derived: 148 SM x 64 DFMA/clk x 2 x 1.965 GHz (guide's unit counts and max clock)",
+                "peak_measured_dfma_probe": FP64_PEAK_MEASURED_TFLOPS,
+                "frac_of_measured_peak": achieved / FP64_PEAK_MEASURED_TFLOPS,
+                "counted": counted("momentum_energy_kernel", mom_s),
                 "hbm_GBps_algorithmic": (MOM_BYTES_PER_PARTICLE + 4 * mean_nc) * n / mom_s / 1e9,
                 "share_of_step": statistics.mean(mom_ms) / (ms_max / args.steps)}
     other = {}
-    for p in ("density", "iad"):
+    for p, kname in (("density", "density_kernel"), ("iad", "iad_kernel")):
         t = phase_ms[p] * 1e-3
-        other[p] = {"tflops": FLOPS_PER_PAIR[p] * pairs / t / 1e12,
-                    "frac_fp64": FLOPS_PER_PAIR[p] * pairs / t / 1e12 / FP64_PEAK_TFLOPS}
+        other[p] = {"flops_per_pair": FLOPS_PER_PAIR[p], "tflops": FLOPS_PER_PAIR[p] * pairs / t / 1e12,
+                    "frac_fp64": FLOPS_PER_PAIR[p] * pairs / t / 1e12 / FP64_PEAK_TFLOPS,
+                    "counted": counted(kname, t)}
 
     # --- e2e: same metric through the C ABI with host buffers ---
     e2e = None
@@ -575,20 +660,27 @@ def main():
                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                "path": "sph_set_particles(pinned host) + sph_step + sph_get_field x11 (host)"}
 
-    p_idle = idle_power(sim) if args.energy_steps > 0 else None
-    energy = measure_energy(sim, sph, n, args, local) if args.energy_steps > 0 else None
+    p_idle = idle_power(sim) if args.energy_seconds > 0 else None
+    energy = measure_energy(sim, sph, n, args, local, ms_max / args.steps) if args.energy_seconds > 0 else None
     if energy is not None and p_idle is not None:
         energy["idle_W"] = p_idle
-    accounting = (in_situ_accounting(sim, sph, max(args.energy_steps // 2, 5), ms_max / args.steps)
-                  if args.energy_steps > 0 else None)
+    accounting = None
+    if energy and energy.get("available"):
+        ws = energy["step"]["windows"]
+        accounting = {"mode": "phase (in situ, no phase-edge syncs; sampled instant power per device-tagged phase)",
+                      "overhead_pct": statistics.median(w["overhead_pct_vs_off"] for w in ws),
+                      "counter_over_sampled": [w["counter_over_sampled"] for w in ws],
+                      "phase_J_sum_over_step": [w["phase_J_sum_over_step"] for w in ws]}
     trace = dvfs_trace(sim, sph, args.trace_seconds) if args.trace_seconds > 0 else None
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         k = args.cpu_sample or 240  # ~10 s of oracle work on the host cores
         v, sec, threads = cpu_baseline(w, k)
+        phys = cpu_physics_only(w)
         cpu = {"value": v, "unit": UNIT, "cores": threads, "kind": "oracle",
-               "sample": f"{k} random targets of {args.workload}, one step (oracle sampled mode), {sec:.1f} s"}
+               "sample": f"{k} random targets of {args.workload}, one step (oracle sampled mode), {sec:.1f} s",
+               "physics_only": phys}
 
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -609,7 +701,7 @@ def main():
                            "search_passes_per_warp": infos[-1]["search_passes"] / (n / 32)},
                 "phase_ms": phase_ms, "fp64_other": other, "roofline": roofline, "e2e": e2e,
                 "phases": phase_table(phase_ms, pairs, n, energy, p_idle),
-                "energy": energy, "accounting": accounting, "dvfs_trace": trace, "cpu_baseline": cpu, "clocks": clk.summary(),
+                "repeats": repeats, "energy": energy, "accounting": accounting, "dvfs_trace": trace, "cpu_baseline": cpu, "clocks": clk.summary(),
                 "gpu_launches": launches}
         s = json.dumps(line)
         print(s, flush=True)

@@ -70,9 +70,16 @@ typedef enum sph_eos_kind { SPH_EOS_IDEAL = 0, SPH_EOS_ISOTHERMAL = 1 } sph_eos_
 typedef enum sph_mem_kind { SPH_MEM_HOST = 0, SPH_MEM_DEVICE = 1 } sph_mem_kind;
 typedef enum sph_accounting_mode {
   SPH_ACCOUNTING_OFF = 0,   /* CUDA-event phase times only, no phase-edge syncs  */
-  SPH_ACCOUNTING_PHASE = 1  /* + stream sync and NVML energy read at every phase
-                               edge ("from the start of each function call
-                               until its completion")                             */
+  SPH_ACCOUNTING_PHASE = 1  /* + in-situ energy per phase ("from the start of
+                               each function call until its completion"): a host
+                               thread samples the phase the device runs (written
+                               by a 1-thread kernel at every phase edge) and the
+                               NVML instant power every ~0.25 ms and integrates
+                               P dt per phase.  No phase-edge syncs.  The B200
+                               refreshes that power value every ~100 ms, so a
+                               phase's joules are its device time at the power
+                               around it; isolated per-phase power needs
+                               sph_repeat_phase (REPEAT analog)          */
 } sph_accounting_mode;
 
 /* Phases = the functions whose energy the paper measures (Fig. 5).
@@ -191,8 +198,8 @@ typedef struct sph_energy_row {
   char name[32];
   int64_t calls;
   double seconds;           /* accumulated CUDA-event time                         */
-  double joules;            /* accumulated NVML energy delta (PHASE accounting)    */
-  double mean_sm_mhz;       /* mean SM clock read at the phase's end edges         */
+  double joules;            /* sampled energy while the device ran the phase (PHASE) */
+  double mean_sm_mhz;       /* mean SM clock sampled while it ran (PHASE)          */
   uint32_t locked_mhz;      /* clock requested by the policy, 0 = default          */
   int32_t available;        /* 1 if joules are valid                               */
 } sph_energy_row;
@@ -330,6 +337,63 @@ int sph_select_ghosts(sph_ctx* ctx, const double* boxes, int R, int self, double
 int sph_gather_field(sph_ctx* ctx, int field, const int64_t* idx, int64_t m, double* dst);
 int sph_scatter_field(sph_ctx* ctx, int field, const int64_t* idx, int64_t m, const double* src);
 
+/* --- SFC decomposition on the device ----------
+ * decomp.py issues the collectives (all-reduce, all-to-all over NCCL) between
+ * these calls; every selection, count, split, pack and map runs here.  All
+ * pointers are DEVICE pointers owned by the caller; all calls are asynchronous
+ * on the context's stream.  Ranks <= 64.
+ *
+ * sph_decomp_reduce: red[0..6] = (-min x, -min y, -min z, max x, max y, max z,
+ *   max h) over the held particles that are not ghosts (-inf when none).  An
+ *   element-wise MAX all-reduce of red over the ranks gives the global bounding
+ *   box and h_max exactly.
+ * sph_set_key_box: from now on the KEYS phase uses [-red[a], red[3 + a]] as the
+ *   box of every OPEN axis a (periodic axes keep the configured box) and red[6]
+ *   as h_max for sph_decomp_ghosts -- the all-reduced red makes every rank's
+ *   keys those of the single-GPU run.  red == NULL: each step's own box again.
+ * sph_key_histogram: hist[b] (int64, 2^bits) = held non-ghost particles whose
+ *   key has top bits b (after sph_compute_keys; bits a multiple of 3).
+ * sph_decomp_owners: from the histogram summed over ranks, the split bins
+ *   s_0 = 0 <= s_1 <= .. <= s_world = 2^bits with s_r = the first bin whose
+ *   inclusive prefix count exceeds floor(total r / world); rank r owns the keys
+ *   of bins [s_r, s_r+1).  mig_mask[i] = 1 << owner(i) if owner(i) != rank
+ *   else 0; counts[r] (int64, world) = held particles owned by r.  The splits
+ *   are kept for sph_decomp_ghosts.
+ * sph_decomp_ghosts: L = the finest level whose cells have side >= 2 h_max
+ *   (sph_set_key_box) on every axis; mask[i] = the ranks (except `rank`) owning
+ *   a key of one of the 27 level-L cells around particle i's (periodic wrap,
+ *   clipped at open faces); counts[r] = particles with bit r.  Every particle
+ *   within 2 h_max of a particle owned by r has bit r: the halo is conservative.
+ * sph_decomp_pack: one row per (particle i, rank r in mask[i]), grouped by r in
+ *   rank order and in particle order within r (id OR-ed with or_id);
+ *   pos[e] = i of row e.  rows/pos hold sum_i popcount(mask[i]) entries.
+ * sph_decomp_drop: stable compaction keeping the particles with
+ *   drop_mask[i] == 0 (drop_mask == NULL: the non-ghosts); the new count is the caller's n_expected (from the
+ *   counts, no synchronisation); a different device count is reported as
+ *   SPH_ERR_STATE at the next synchronising call.
+ * sph_decomp_map: after sph_build_tree, the positions after its sort of the
+ *   positions pre[k] before it (pre == NULL: first + k), for the halo lists.
+ * sph_halo_gather / sph_halo_scatter: rows [m][nf] of the fields at idx; the
+ *   scatter takes the same fields and refreshes what depends on them, as
+ *   sph_scatter_field does.
+ * sph_min_hc_dev / sph_set_min_hc_dev: the local min h/c (or h/v_sig) of the
+ *   last MOMENTUM_ENERGY into / the global minimum from a device double (the
+ *   P:220 collective without a host round trip). */
+int sph_decomp_reduce(sph_ctx* ctx, double* red);
+int sph_set_key_box(sph_ctx* ctx, const double* red);
+int sph_key_histogram(sph_ctx* ctx, int bits, int64_t* hist);
+int sph_decomp_owners(sph_ctx* ctx, const int64_t* hist, int bits, int rank, int world, uint64_t* mig_mask,
+                      int64_t* counts);
+int sph_decomp_ghosts(sph_ctx* ctx, int bits, int rank, int world, uint64_t* mask, int64_t* counts);
+int sph_decomp_pack(sph_ctx* ctx, const uint64_t* mask, int world, uint64_t or_id, double* rows, int64_t* pos);
+int sph_decomp_drop(sph_ctx* ctx, const uint64_t* drop_mask, int64_t n_expected);
+int sph_decomp_map(sph_ctx* ctx, const int64_t* pre, int64_t first, int64_t m, int64_t* post);
+int sph_halo_gather(sph_ctx* ctx, const int32_t* fields, int nf, const int64_t* idx, int64_t m, double* dst);
+int sph_halo_scatter(sph_ctx* ctx, const int32_t* fields, int nf, const int64_t* idx, int64_t m,
+                     const double* src);
+int sph_min_hc_dev(sph_ctx* ctx, double* dst);
+int sph_set_min_hc_dev(sph_ctx* ctx, const double* src);
+
 /* --- the hot path (each call = one accounted phase group) ------------------- */
 
 /* Items 1-3: box (open axes: exact min/max), 63-bit Morton keys, stable LSD
@@ -410,7 +474,25 @@ int sph_supported_clocks(sph_ctx* ctx, uint32_t* mhz, int cap, int* n);
 /* One row per phase (cap >= SPH_NPHASES).  Time is always filled; joules only
  * with PHASE accounting and a working NVML energy counter. */
 int sph_energy_report(sph_ctx* ctx, sph_energy_row* rows, int cap, int* n_rows);
+/* Zeroes the rows and the PHASE accumulators and reads the energy counter as
+ * the start of the accounting window. */
 int sph_energy_reset(sph_ctx* ctx);
+
+/* The accounting window since sph_energy_reset (synchronises): the sampled
+ * energy (sum over phases + between phases), the NVML total-energy counter
+ * delta over the same window (-1 when unreadable; the counter advances in
+ * ~100 ms / ~99 J steps on a B200, so windows of >= 10 s keep it within 1%),
+ * wall and sampled seconds.  sampled_joules vs counter_joules is the
+ * accounting's self-check (SURVEY 8(c) "Energy accounting"). */
+typedef struct sph_energy_window {
+  double wall_seconds;
+  double sampled_seconds;
+  double sampled_joules;
+  double between_joules;    /* sampled while no phase was running (host gaps)  */
+  double counter_joules;
+  int64_t samples;
+} sph_energy_window;
+int sph_energy_totals(sph_ctx* ctx, sph_energy_window* totals);
 
 /* Total-energy counter of the device in mJ (NVML), for whole-run deltas. */
 int sph_energy_counter_mj(sph_ctx* ctx, uint64_t* mj);

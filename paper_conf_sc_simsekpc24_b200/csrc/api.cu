@@ -9,6 +9,7 @@
 #include <algorithm>
 #include <atomic>
 #include <chrono>
+#include <mutex>
 #include <thread>
 #include <vector>
 
@@ -88,14 +89,23 @@ struct sph_ctx {
   bool pending[SPH_NPHASES];
   double last_ms[SPH_NPHASES];
   PhaseRow rows[SPH_NPHASES];
-  unsigned long long e0 = 0;
-  bool e0_ok = false;
-  // PHASE accounting: the counter read at a phase's end serves as the next
-  // phase's start read when that phase begins right after it (back-to-back
-  // phases inside sph_step); each NVML read costs milliseconds on this host.
-  unsigned long long e_last = 0;
-  bool e_last_ok = false;
-  std::chrono::steady_clock::time_point t_last_end{};
+  // PHASE accounting (in situ, no phase-edge syncs): a host thread samples the
+  // device-written phase tag and the NVML instant power and integrates
+  // E_p = sum P dt over the intervals the device spent in phase p.
+  struct Acct {
+    std::thread th;
+    std::atomic<bool> run{false};
+    bool active = false;
+    std::mutex mu;
+    double J[SPH_NPHASES + 1] = {};         // [SPH_NPHASES] = between phases
+    double mhz_sum[SPH_NPHASES + 1] = {};
+    int64_t mhz_n[SPH_NPHASES + 1] = {};
+    int64_t samples = 0;
+    double seconds = 0;                     // sampled wall time since reset
+    unsigned long long e_start = 0;         // energy counter at reset
+    std::chrono::steady_clock::time_point t_start{};
+    bool e_start_ok = false;
+  } acct;
   Nvml nvml;
   int clock_mode = SPH_CLOCK_DEFAULT;
   unsigned clock_mhz[SPH_NPHASES];
@@ -103,8 +113,11 @@ struct sph_ctx {
   bool locked_any = false;
   bool rec_m_dirty = false;
   uint32_t* last_perm = nullptr;  // the last sort's permutation (SPH_F_ORDER)
-  uint32_t* perm_saved = nullptr; // its copy while sph_repeat_phase(SORT) reuses the buffers
-  int64_t* compact_scratch = nullptr;  // per-block counts of sph_compact (+ total)
+  uint32_t* perm_saved = nullptr; // its copy while sph_repeat_phase(SORT) reuses the buffers;
+                                  // also the inverse permutation of sph_decomp_map
+  bool inv_valid = false;         // perm_saved holds the inverse of last_perm
+  int64_t* compact_scratch = nullptr;  // per-block counts of sph_compact / sph_decomp_pack (+ totals)
+  int64_t compact_scratch_len = 0;
   Stir stir{};          // turbulence driving (k_stir.cu)
   bool stir_on = false;
   // DVFS trace (sph_trace_start / sph_trace_stop)
@@ -213,9 +226,97 @@ __global__ void trace_mark_kernel(int* word, int phase) {
 
 // Tags the DVFS trace with the phase the stream reaches next (trace active only).
 void trace_mark(sph_ctx* c, int phase) {
-  if (!c->trace.active) return;
+  if (!c->trace.active && !c->acct.active) return;
   trace_mark_kernel<<<1, 1, 0, c->st>>>(c->trace.word_dev, phase);
   note_launch();
+}
+
+// The pinned, device-mapped word the trace_mark kernels write: the phase the
+// stream is executing (shared by the DVFS trace and PHASE accounting).
+int ensure_phase_word(sph_ctx* c) {
+  if (c->trace.word) return SPH_OK;
+  void* h = nullptr;
+  int rc = cuda_check(c, cudaHostAlloc(&h, sizeof(int), cudaHostAllocMapped), "cudaHostAlloc");
+  if (rc) return rc;
+  void* d = nullptr;
+  if ((rc = cuda_check(c, cudaHostGetDevicePointer(&d, h, 0), "cudaHostGetDevicePointer"))) return rc;
+  c->trace.word = (volatile int*)h;
+  c->trace.word_dev = (int*)d;
+  *c->trace.word = -1;
+  return SPH_OK;
+}
+
+void acct_reset(sph_ctx* c) {
+  sph_ctx::Acct& A = c->acct;
+  std::lock_guard<std::mutex> g(A.mu);
+  for (int p = 0; p <= SPH_NPHASES; ++p) A.J[p] = A.mhz_sum[p] = 0.0, A.mhz_n[p] = 0;
+  A.samples = 0;
+  A.seconds = 0.0;
+  A.e_start_ok = c->nvml.energy_mj(&A.e_start);
+  A.t_start = std::chrono::steady_clock::now();
+}
+
+// PHASE accounting sampler: every ~0.25 ms the phase tag and the instant power;
+// the interval since the previous sample is charged to the phase seen then at
+// the power read then (left Riemann sum).  NVML's instant power refreshes about
+// every 100 ms on a B200 (profiles/r02_probe_nvml_instant.json), so the joules
+// of a phase shorter than that are its time at the surrounding average power.
+int acct_start(sph_ctx* c) {
+  if (c->acct.active) return SPH_OK;
+  if (!c->nvml.ok) return fail(c, SPH_ERR_NVML, "NVML unavailable: %s", c->nvml.err);
+  unsigned probe = 0;
+  if (!c->nvml.power_instant_mw(&probe) && !c->nvml.power_mw(&probe))
+    return fail(c, SPH_ERR_NVML, "NVML power unreadable: %s", c->nvml.error_string(c->nvml.last_rc));
+  int rc = ensure_phase_word(c);
+  if (rc) return rc;
+  acct_reset(c);
+  c->acct.run.store(true);
+  c->acct.active = true;
+  sph_ctx::Acct* A = &c->acct;
+  Nvml* nv = &c->nvml;
+  volatile int* word = c->trace.word;
+  c->acct.th = std::thread([A, nv, word]() {
+    using clk = std::chrono::steady_clock;
+    const bool instant = [&] { unsigned v; return nv->power_instant_mw(&v); }();
+    auto power = [&](unsigned* v) { return instant ? nv->power_instant_mw(v) : nv->power_mw(v); };
+    auto prev = clk::now();
+    int ph_prev = *word;
+    unsigned p_prev = 0;
+    power(&p_prev);
+    int64_t k = 0;
+    while (A->run.load(std::memory_order_relaxed)) {
+      std::this_thread::sleep_for(std::chrono::microseconds(250));
+      const auto now = clk::now();
+      const int ph = *word;
+      unsigned pw = p_prev;
+      power(&pw);
+      unsigned mhz = 0;
+      const bool got_mhz = (++k & 15) == 0 && nv->sm_clock_mhz(&mhz);
+      const double dt = std::chrono::duration<double>(now - prev).count();
+      const int b = (ph_prev >= 0 && ph_prev < SPH_NPHASES) ? ph_prev : SPH_NPHASES;
+      {
+        std::lock_guard<std::mutex> g(A->mu);
+        A->J[b] += 1e-3 * p_prev * dt;
+        A->seconds += dt;
+        ++A->samples;
+        if (got_mhz) {
+          A->mhz_sum[b] += mhz;
+          ++A->mhz_n[b];
+        }
+      }
+      prev = now;
+      ph_prev = ph;
+      p_prev = pw;
+    }
+  });
+  return SPH_OK;
+}
+
+void acct_stop(sph_ctx* c) {
+  if (!c->acct.active) return;
+  c->acct.run.store(false);
+  if (c->acct.th.joinable()) c->acct.th.join();
+  c->acct.active = false;
 }
 
 int phase_begin(sph_ctx* c, int p) {
@@ -226,17 +327,6 @@ int phase_begin(sph_ctx* c, int p) {
   }
   apply_clock(c, p);
   c->rows[p].locked = c->current_lock;
-  if (c->cfg.accounting == SPH_ACCOUNTING_PHASE) {
-    int rc = cuda_check(c, cudaStreamSynchronize(c->st), "phase sync");
-    if (rc) return rc;
-    const auto now = std::chrono::steady_clock::now();
-    if (c->e_last_ok && now - c->t_last_end < std::chrono::microseconds(200)) {
-      c->e0 = c->e_last;  // nothing ran since the previous phase's end read
-      c->e0_ok = true;
-    } else {
-      c->e0_ok = c->nvml.energy_mj(&c->e0);
-    }
-  }
   return cuda_check(c, cudaEventRecord(c->ev[p][0], c->st), "cudaEventRecord");
 }
 
@@ -246,24 +336,6 @@ int phase_end(sph_ctx* c, int p) {
   trace_mark(c, -1);
   c->pending[p] = true;
   c->rows[p].calls++;
-  if (c->cfg.accounting == SPH_ACCOUNTING_PHASE) {
-    rc = cuda_check(c, cudaStreamSynchronize(c->st), "phase sync");
-    if (rc) return rc;
-    unsigned long long e1;
-    c->e_last_ok = false;
-    if (c->e0_ok && c->nvml.energy_mj(&e1)) {
-      c->rows[p].joules += (double)(e1 - c->e0) * 1e-3;
-      c->rows[p].avail = true;
-      c->e_last = e1;
-      c->e_last_ok = true;
-    }
-    unsigned mhz;  // SM clock sampled at every 8th end of each phase (NVML is slow)
-    if ((c->rows[p].calls & 7) == 1 && c->nvml.sm_clock_mhz(&mhz)) {
-      c->rows[p].mhz_sum += mhz;
-      c->rows[p].mhz_n++;
-    }
-    c->t_last_end = std::chrono::steady_clock::now();
-  }
   return SPH_OK;
 }
 
@@ -279,6 +351,7 @@ int sync_scalars(sph_ctx* c) {
   if (s & ST_CAPACITY)
     return fail(c, SPH_ERR_CAPACITY, "neighbour count %d exceeds ngmax %d", c->h_ds.max_nc, c->cfg.ngmax);
   if (s & ST_SINGULAR) return fail(c, SPH_ERR_SINGULAR, "singular IAD matrix (det <= 0 or non-finite)");
+  if (s & ST_DECOMP) return fail(c, SPH_ERR_STATE, "decomposition: a kept/received count differs from the caller's");
   if (s & ST_STIR_NOISE) return fail(c, SPH_ERR_CAPACITY, "driving noise table exhausted (%lld steps)", (long long)c->stir.nsteps);
   return SPH_OK;
 }
@@ -332,6 +405,7 @@ int body_tree(sph_ctx* c) {
                               c->status_bytes, &perm, &ksorted, c->st);
   if ((rc = cuda_check(c, e, "sort"))) return rc;
   c->last_perm = perm;
+  c->inv_valid = false;
   const int prv = c->cur;
   c->cur ^= 1;
   c->key_sorted = ksorted;
@@ -539,8 +613,13 @@ static size_t layout(const sph_config* cfg, char* base, sph_ctx* c) {
   char* hp = take(hb);
   char* sp = take(sb);
   char* dsp = take(sizeof(DevScalars));
-  char* csc = take(sizeof(int64_t) * ((cap + 1023) / 1024 + 2));
-  if (c) c->compact_scratch = (int64_t*)csc;
+  // compaction (blocks + total) and the grouped pack (64 ranks x blocks + total)
+  const size_t csl = (size_t)kMaxGhostRanks * ((cap + 1023) / 1024) + 2;
+  char* csc = take(sizeof(int64_t) * csl);
+  if (c) {
+    c->compact_scratch = (int64_t*)csc;
+    c->compact_scratch_len = (int64_t)csl;
+  }
   const size_t sst = (size_t)cfg->stir_steps;
   char* sA = sst ? take(sizeof(double) * kStirModes * 6) : nullptr;
   char* sB = sst ? take(sizeof(double) * kStirModes * 6) : nullptr;
@@ -605,6 +684,7 @@ int sph_init(const sph_config* cfg, void* arena, size_t arena_bytes, void* strea
   c->P.gradh = cfg->gradh ? 1 : 0;
   c->P.ve = cfg->ve ? 1 : 0;
   c->P.dt_vsig = cfg->dt_vsig ? 1 : 0;
+  c->P.key_box_set = 0;
   layout(cfg, (char*)arena, c);
   for (int p = 0; p < SPH_NPHASES; ++p) {
     c->pending[p] = false;
@@ -630,6 +710,9 @@ int sph_init(const sph_config* cfg, void* arena, size_t arena_bytes, void* strea
   }
   c->nvml.init(cfg->device);  // failure only disables energy/clock features
   c->stage = S_INIT;
+  // PHASE accounting from the start: without NVML the energy rows stay
+  // unavailable (NVML errors never fail or poison)
+  if (cfg->accounting == SPH_ACCOUNTING_PHASE && acct_start(c) != SPH_OK) c->err[0] = 0;
   *out = c;
   return SPH_OK;
 }
@@ -637,6 +720,7 @@ int sph_init(const sph_config* cfg, void* arena, size_t arena_bytes, void* strea
 void sph_finalize(sph_ctx* c) {
   if (!c) return;
   if (c->trace.active) sph_trace_stop(c, nullptr, 0, nullptr);
+  acct_stop(c);
   if (c->trace.word) cudaFreeHost((void*)c->trace.word);
   if (c->locked_any) c->nvml.reset_sm_clock();
   c->nvml.shutdown();
@@ -968,6 +1052,175 @@ int sph_scatter_field(sph_ctx* c, int field, const int64_t* idx, int64_t m, cons
   return cuda_check(c, cudaGetLastError(), "prho2");
 }
 
+// ---------------------------------------------------------------- SFC decomposition (device)
+int sph_decomp_reduce(sph_ctx* c, double* red) {
+  int rc = check_ready(c, S_PART, "sph_decomp_reduce");
+  if (rc) return rc;
+  if (!red) return fail(c, SPH_ERR_ARG, "null red");
+  return cuda_check(c, launch_decomp_reduce(c->n, c->state[c->cur], c->ids[c->cur], c->ds->red_ord, red, c->st),
+                    "decomp reduce");
+}
+
+int sph_set_key_box(sph_ctx* c, const double* red) {
+  int rc = check_ready(c, S_INIT, "sph_set_key_box");
+  if (rc) return rc;
+  if (!red) {
+    c->P.key_box_set = 0;
+    return SPH_OK;
+  }
+  rc = cuda_check(c, cudaMemcpyAsync(c->ds->key_box, red, sizeof(double) * 7, cudaMemcpyDeviceToDevice, c->st),
+                  "key box");
+  if (!rc) c->P.key_box_set = 1;
+  return rc;
+}
+
+int sph_key_histogram(sph_ctx* c, int bits, int64_t* hist) {
+  int rc = check_ready(c, S_PART, "sph_key_histogram");
+  if (rc) return rc;
+  if (bits < 3 || bits > 21 || bits % 3 || !hist) return fail(c, SPH_ERR_ARG, "bits must be a multiple of 3 in [3, 21]");
+  if (c->key_sorted != c->keyA) return fail(c, SPH_ERR_STATE, "sph_key_histogram needs sph_compute_keys");
+  return cuda_check(c, launch_key_histogram(c->n, c->keyA, c->ids[c->cur], bits, hist, c->st), "key histogram");
+}
+
+int sph_decomp_owners(sph_ctx* c, const int64_t* hist, int bits, int rank, int world, uint64_t* mig_mask,
+                      int64_t* counts) {
+  int rc = check_ready(c, S_PART, "sph_decomp_owners");
+  if (rc) return rc;
+  if (bits < 3 || bits > 21 || bits % 3 || !hist || !counts || (c->n > 0 && !mig_mask))
+    return fail(c, SPH_ERR_ARG, "bad bits / buffers");
+  if (world < 1 || world > kMaxGhostRanks || rank < 0 || rank >= world) return fail(c, SPH_ERR_ARG, "bad rank/world");
+  if (c->key_sorted != c->keyA) return fail(c, SPH_ERR_STATE, "sph_decomp_owners needs sph_compute_keys");
+  return cuda_check(c, launch_decomp_owners(c->n, c->keyA, hist, bits, rank, world, c->ds->splits, mig_mask, counts,
+                                            c->st), "decomp owners");
+}
+
+int sph_decomp_ghosts(sph_ctx* c, int bits, int rank, int world, uint64_t* mask, int64_t* counts) {
+  int rc = check_ready(c, S_PART, "sph_decomp_ghosts");
+  if (rc) return rc;
+  if (bits < 3 || bits > 21 || bits % 3 || !counts || (c->n > 0 && !mask)) return fail(c, SPH_ERR_ARG, "bad bits / buffers");
+  if (world < 1 || world > kMaxGhostRanks || rank < 0 || rank >= world) return fail(c, SPH_ERR_ARG, "bad rank/world");
+  if (!c->P.key_box_set) return fail(c, SPH_ERR_STATE, "sph_decomp_ghosts needs sph_set_key_box (global h_max)");
+  if (c->key_sorted != c->keyA) return fail(c, SPH_ERR_STATE, "sph_decomp_ghosts needs sph_compute_keys");
+  return cuda_check(c, launch_decomp_ghosts(c->n, c->keyA, bits, rank, world, c->ds->splits, c->ds, c->P, mask,
+                                            counts, c->st), "decomp ghosts");
+}
+
+int sph_decomp_pack(sph_ctx* c, const uint64_t* mask, int world, uint64_t or_id, double* rows, int64_t* pos) {
+  int rc = check_ready(c, S_PART, "sph_decomp_pack");
+  if (rc) return rc;
+  if (world < 1 || world > kMaxGhostRanks || (c->n > 0 && (!mask || !rows || !pos))) return fail(c, SPH_ERR_ARG, "bad buffers");
+  int64_t* total = c->compact_scratch + c->compact_scratch_len - 1;
+  const int64_t nb = div_up(c->n, 1024);
+  if (nb * world + 1 > c->compact_scratch_len) return fail(c, SPH_ERR_CAPACITY, "pack scratch too small");
+  return cuda_check(c, launch_route_pack(c->n, mask, world, c->state[c->cur], c->ids[c->cur], or_id, rows, pos,
+                                         c->compact_scratch, total, c->st), "decomp pack");
+}
+
+__global__ void check_count_kernel(const int64_t* total, int64_t expected, DevScalars* ds) {
+  if (*total != expected) ds->status |= ST_DECOMP;
+}
+
+int sph_decomp_drop(sph_ctx* c, const uint64_t* drop_mask, int64_t n_expected) {
+  int rc = check_ready(c, S_PART, "sph_decomp_drop");
+  if (rc) return rc;
+  if (n_expected < 0 || n_expected > c->n) return fail(c, SPH_ERR_ARG, "n_expected out of range");
+  const int nxt = c->cur ^ 1;
+  int64_t* total = c->compact_scratch + (c->cfg.n_capacity + 1023) / 1024 + 1;
+  // drop_mask == NULL: drop the ghosts (SPH_GHOST_BIT) instead
+  rc = cuda_check(c, launch_compact(c->n, nullptr, drop_mask ? 0 : 1, c->state[c->cur], c->ids[c->cur], c->state[nxt],
+                                    c->ids[nxt], c->compact_scratch, total, c->st, drop_mask), "decomp drop");
+  if (rc) return rc;
+  check_count_kernel<<<1, 1, 0, c->st>>>(total, n_expected, c->ds);
+  note_launch();
+  c->cur = nxt;
+  c->n = n_expected;  // the caller's count (known from the routed counts): no sync
+  c->stage = S_PART;
+  return cuda_check(c, cudaGetLastError(), "check count");
+}
+
+int sph_decomp_map(sph_ctx* c, const int64_t* pre, int64_t first, int64_t m, int64_t* post) {
+  int rc = check_ready(c, S_TREE, "sph_decomp_map");
+  if (rc) return rc;
+  if (m < 0 || (m > 0 && !post) || (!pre && (first < 0 || first + m > c->n))) return fail(c, SPH_ERR_ARG, "bad map arguments");
+  if (!c->inv_valid) {
+    if ((rc = cuda_check(c, launch_inverse_perm(c->n, c->last_perm, c->perm_saved, c->st), "inverse perm"))) return rc;
+    c->inv_valid = true;
+  }
+  return cuda_check(c, launch_map_positions(m, pre, first, c->perm_saved, post, c->st), "map positions");
+}
+
+static int halo_fields(sph_ctx* c, const int32_t* flds, int nf, double** f, bool for_scatter, bool* dirty_rec,
+                       bool* prho2, bool* eos) {
+  if (nf < 1 || nf > 16 || !flds) return fail(c, SPH_ERR_ARG, "1..16 fields");
+  for (int q = 0; q < nf; ++q) {
+    const int fd = flds[q];
+    f[q] = double_field(c, fd);
+    if (!f[q]) return fail(c, SPH_ERR_ARG, "field %d is not a double field of this configuration", fd);
+    if (!for_scatter) continue;
+    if (fd == SPH_F_RHO) {
+      if (c->stage < S_DENS) return fail(c, SPH_ERR_STATE, "halo(RHO) before sph_density");
+      *eos = *eos || (c->P.ve && c->gradh_done && c->stage == S_EOS);
+    } else if ((fd >= SPH_F_C11 && fd <= SPH_F_C33) || (fd == SPH_F_BAL && c->P.av_switch)) {
+      if (c->stage < S_IAD) return fail(c, SPH_ERR_STATE, "halo(C/BAL) before sph_iad");
+      *dirty_rec = true;
+    } else if (fd == SPH_F_OMEGA && c->omega) {
+      if (!c->gradh_done || c->stage != S_EOS) return fail(c, SPH_ERR_STATE, "halo(OMEGA) must follow sph_gradh, before sph_iad");
+      *prho2 = true;
+    } else {
+      return fail(c, SPH_ERR_ARG, "field %d is not settable", fd);
+    }
+  }
+  return SPH_OK;
+}
+
+int sph_halo_gather(sph_ctx* c, const int32_t* flds, int nf, const int64_t* idx, int64_t m, double* dst) {
+  int rc = check_ready(c, S_INIT, "sph_halo_gather");
+  if (rc) return rc;
+  if (m < 0 || (m > 0 && (!idx || !dst))) return fail(c, SPH_ERR_ARG, "bad idx/dst");
+  double* f[16];
+  bool a = false, b = false, e = false;
+  if ((rc = halo_fields(c, flds, nf, f, false, &a, &b, &e))) return rc;
+  return cuda_check(c, launch_halo(m, idx, f, nf, dst, true, c->st), "halo gather");
+}
+
+int sph_halo_scatter(sph_ctx* c, const int32_t* flds, int nf, const int64_t* idx, int64_t m, const double* src) {
+  int rc = check_ready(c, S_INIT, "sph_halo_scatter");
+  if (rc) return rc;
+  if (m < 0 || (m > 0 && (!idx || !src))) return fail(c, SPH_ERR_ARG, "bad idx/src");
+  double* f[16];
+  bool dirty = false, prho2 = false, eos = false;
+  if ((rc = halo_fields(c, flds, nf, f, true, &dirty, &prho2, &eos))) return rc;
+  if ((rc = cuda_check(c, launch_halo(m, idx, f, nf, const_cast<double*>(src), false, c->st), "halo scatter"))) return rc;
+  if (dirty) c->rec_m_dirty = true;
+  if (eos) launch_eos(fields(c), c->P, c->st, c->P.gradh != 0);  // owners' normalised rho (reading 23)
+  if (prho2) launch_prho2(fields(c), c->st);
+  return cuda_check(c, cudaGetLastError(), "halo refresh");
+}
+
+__global__ void min_hc_get_kernel(const DevScalars* ds, double* out) {
+  const unsigned long long o = ds->minhc_ord;
+  *out = o == ~0ull ? INFINITY : unord(o);
+}
+__global__ void min_hc_set_kernel(DevScalars* ds, const double* in) { ds->minhc_ord = ord_of(*in); }
+
+int sph_min_hc_dev(sph_ctx* c, double* dst) {
+  int rc = check_ready(c, S_MOM, "sph_min_hc_dev");
+  if (rc) return rc;
+  if (!dst) return fail(c, SPH_ERR_ARG, "null dst");
+  min_hc_get_kernel<<<1, 1, 0, c->st>>>(c->ds, dst);
+  note_launch();
+  return cuda_check(c, cudaGetLastError(), "min hc");
+}
+
+int sph_set_min_hc_dev(sph_ctx* c, const double* src) {
+  int rc = check_ready(c, S_MOM, "sph_set_min_hc_dev");
+  if (rc) return rc;
+  if (!src) return fail(c, SPH_ERR_ARG, "null src");
+  min_hc_set_kernel<<<1, 1, 0, c->st>>>(c->ds, src);
+  note_launch();
+  return cuda_check(c, cudaGetLastError(), "set min hc");
+}
+
 int sph_build_tree(sph_ctx* c) {
   int rc = check_ready(c, S_PART, "sph_build_tree");
   if (rc) return rc;
@@ -1173,10 +1426,13 @@ int sph_energy_report(sph_ctx* c, sph_energy_row* rows, int cap, int* n_rows) {
     snprintf(r.name, sizeof(r.name), "%s", kPhaseNames[p]);
     r.calls = c->rows[p].calls;
     r.seconds = c->rows[p].seconds;
-    r.joules = c->rows[p].joules;
-    r.mean_sm_mhz = c->rows[p].mhz_n ? c->rows[p].mhz_sum / c->rows[p].mhz_n : 0.0;
+    {
+      std::lock_guard<std::mutex> g(c->acct.mu);
+      r.joules = c->acct.J[p];
+      r.mean_sm_mhz = c->acct.mhz_n[p] ? c->acct.mhz_sum[p] / c->acct.mhz_n[p] : 0.0;
+      r.available = c->acct.samples > 0 ? 1 : 0;
+    }
     r.locked_mhz = c->rows[p].locked;
-    r.available = c->rows[p].avail ? 1 : 0;
   }
   if (n_rows) *n_rows = SPH_NPHASES;
   return SPH_OK;
@@ -1188,6 +1444,25 @@ int sph_energy_reset(sph_ctx* c) {
   cudaStreamSynchronize(c->st);
   collect_all(c);
   for (int p = 0; p < SPH_NPHASES; ++p) c->rows[p] = PhaseRow();
+  acct_reset(c);
+  return SPH_OK;
+}
+
+int sph_energy_totals(sph_ctx* c, sph_energy_window* t) {
+  int rc = check_ready(c, S_INIT, "sph_energy_totals");
+  if (rc) return rc;
+  if (!t) return fail(c, SPH_ERR_ARG, "null totals");
+  if (!c->poisoned && (rc = cuda_check(c, cudaStreamSynchronize(c->st), "sync"))) return rc;
+  memset(t, 0, sizeof(*t));
+  unsigned long long e1 = 0;
+  const bool eok = c->nvml.energy_mj(&e1);
+  std::lock_guard<std::mutex> g(c->acct.mu);
+  t->wall_seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - c->acct.t_start).count();
+  t->sampled_seconds = c->acct.seconds;
+  for (int p = 0; p <= SPH_NPHASES; ++p) t->sampled_joules += c->acct.J[p];
+  t->between_joules = c->acct.J[SPH_NPHASES];
+  t->counter_joules = (eok && c->acct.e_start_ok) ? (double)(e1 - c->acct.e_start) * 1e-3 : -1.0;
+  t->samples = c->acct.samples;
   return SPH_OK;
 }
 
@@ -1203,6 +1478,11 @@ int sph_set_accounting(sph_ctx* c, int mode) {
   int rc = check_ready(c, S_INIT, "sph_set_accounting");
   if (rc) return rc;
   if (mode != SPH_ACCOUNTING_OFF && mode != SPH_ACCOUNTING_PHASE) return fail(c, SPH_ERR_ARG, "unknown accounting mode %d", mode);
+  if (mode == SPH_ACCOUNTING_PHASE) {
+    if ((rc = acct_start(c))) return rc;
+  } else {
+    acct_stop(c);
+  }
   c->cfg.accounting = mode;
   return SPH_OK;
 }
@@ -1259,8 +1539,10 @@ int sph_repeat_phase(sph_ctx* c, int phase, int reps, double* ms_per_call, doubl
   Fk.key = spare_keys;
   const int prv = c->cur;
   const size_t perm_bytes = sizeof(uint32_t) * (size_t)c->n;
-  if (phase == SPH_PHASE_SORT && c->last_perm && c->n > 0)  // the repeats reuse its buffer
+  if (phase == SPH_PHASE_SORT && c->last_perm && c->n > 0) {  // the repeats reuse its buffer
     cudaMemcpyAsync(c->perm_saved, c->last_perm, perm_bytes, cudaMemcpyDeviceToDevice, c->st);
+    c->inv_valid = false;
+  }
   // EOS after GRADH: p/(Omega rho^2), as the pipeline left it (reading 21)
   const bool eos_omega = c->gradh_done && c->cfg.gradh;
   for (int r = 0; r < reps; ++r) {
@@ -1312,15 +1594,8 @@ int sph_trace_start(sph_ctx* c, double period_ms, int64_t capacity) {
   if (!(period_ms >= 0.1) || capacity < 1) return fail(c, SPH_ERR_ARG, "period_ms >= 0.1 and capacity >= 1 required");
   if (c->trace.active) return fail(c, SPH_ERR_STATE, "a trace is already running");
   if (!c->nvml.ok) return fail(c, SPH_ERR_NVML, "NVML unavailable: %s", c->nvml.err);
-  if (!c->trace.word) {
-    void* h = nullptr;
-    if ((rc = cuda_check(c, cudaHostAlloc(&h, sizeof(int), cudaHostAllocMapped), "cudaHostAlloc"))) return rc;
-    void* d = nullptr;
-    if ((rc = cuda_check(c, cudaHostGetDevicePointer(&d, h, 0), "cudaHostGetDevicePointer"))) return rc;
-    c->trace.word = (volatile int*)h;
-    c->trace.word_dev = (int*)d;
-  }
-  *c->trace.word = -1;
+  if ((rc = ensure_phase_word(c))) return rc;
+  if (!c->acct.active) *c->trace.word = -1;
   c->trace.buf.assign((size_t)capacity, sph_trace_sample{});
   c->trace.taken = 0;
   c->trace.run.store(true);

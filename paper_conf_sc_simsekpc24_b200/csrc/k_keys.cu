@@ -79,6 +79,11 @@ __global__ void box_finalize_kernel(DevScalars* ds, Params P, int64_t n) {
     if (P.periodic[a]) {
       ds->box_min[a] = P.box_min[a];
       ds->box_max[a] = P.box_max[a];
+    } else if (P.key_box_set) {  // the global box of a decomposed run (sph_set_key_box)
+      const double lo = -ds->key_box[a], hi = ds->key_box[3 + a];
+      ds->box_min[a] = lo;
+      ds->box_max[a] = hi;
+      if (!(hi > lo)) ds->status |= ST_BOX;
     } else {
       double lo = unord(ds->box_min_ord[a]), hi = unord(ds->box_max_ord[a]);
       ds->box_min[a] = lo;

@@ -23,6 +23,16 @@ typedef int (*fn_sup_gr)(void*, unsigned, unsigned*, unsigned*);
 typedef int (*fn_lock)(void*, unsigned, unsigned);
 typedef int (*fn_reset)(void*);
 typedef const char* (*fn_errstr)(int);
+// nvmlFieldValue_t (nvml.h:2677): fieldId, scopeId, timestamp, latencyUsec,
+// valueType, nvmlReturn, value (8-byte union)
+struct FieldValue {
+  unsigned fieldId, scopeId;
+  long long timestamp, latencyUsec;
+  int valueType, nvmlReturn;
+  unsigned long long value;
+};
+typedef int (*fn_fields)(void*, int, FieldValue*);
+constexpr unsigned kFiPowerInstant = 186;  // NVML_FI_DEV_POWER_INSTANT (nvml.h:2496)
 
 struct Syms {
   fn_init init;
@@ -36,6 +46,7 @@ struct Syms {
   fn_lock lock;
   fn_reset reset;
   fn_errstr errstr;
+  fn_fields fields;
 };
 Syms g_syms;
 constexpr int kNvmlClockSM = 1;  // NVML_CLOCK_SM
@@ -58,6 +69,7 @@ bool Nvml::init(int cuda_device) {
   g_syms.lock = (fn_lock)dlsym(lib, "nvmlDeviceSetGpuLockedClocks");
   g_syms.reset = (fn_reset)dlsym(lib, "nvmlDeviceResetGpuLockedClocks");
   g_syms.errstr = (fn_errstr)dlsym(lib, "nvmlErrorString");
+  g_syms.fields = (fn_fields)dlsym(lib, "nvmlDeviceGetFieldValues");
   if (!g_syms.init || !g_syms.by_pci) {
     snprintf(err, sizeof(err), "NVML symbols missing");
     return false;
@@ -103,6 +115,19 @@ bool Nvml::sm_clock_mhz(unsigned* mhz) {
 bool Nvml::power_mw(unsigned* mw) {
   if (!ok || !g_syms.power) return false;
   return (last_rc = g_syms.power(dev, mw)) == 0;
+}
+
+bool Nvml::power_instant_mw(unsigned* mw) {
+  if (!ok || !g_syms.fields) return false;
+  FieldValue v{};
+  v.fieldId = kFiPowerInstant;
+  if ((last_rc = g_syms.fields(dev, 1, &v)) != 0) return false;
+  if (v.nvmlReturn != 0) {
+    last_rc = v.nvmlReturn;
+    return false;
+  }
+  *mw = (unsigned)v.value;  // unsigned int member of the union (little endian)
+  return true;
 }
 
 int Nvml::supported_sm_clocks(unsigned* out, unsigned cap) {

@@ -20,7 +20,8 @@ struct Nvml {
   void shutdown();
   bool energy_mj(unsigned long long* mj);
   bool sm_clock_mhz(unsigned* mhz);
-  bool power_mw(unsigned* mw);
+  bool power_mw(unsigned* mw);          // nvmlDeviceGetPowerUsage (~1 s average)
+  bool power_instant_mw(unsigned* mw);  // field NVML_FI_DEV_POWER_INSTANT (fast read; B200 updates it ~every 100 ms)
   int supported_sm_clocks(unsigned* out, unsigned cap);  // returns count (<= cap)
   int lock_sm_clock(unsigned mhz);  // 0 ok, else NVML return code
   int reset_sm_clock();

@@ -28,7 +28,7 @@ constexpr int kRadix = 256;
 constexpr int kSortPasses = 8;  // 8 x 8 bits >= 63-bit keys
 
 // Device status bits (reported at the next synchronising call).
-enum DevStatus : int { ST_BOX = 1, ST_CAPACITY = 2, ST_SINGULAR = 4, ST_STIR_NOISE = 8 };
+enum DevStatus : int { ST_BOX = 1, ST_CAPACITY = 2, ST_SINGULAR = 4, ST_STIR_NOISE = 8, ST_DECOMP = 16 };
 
 // Small block of device scalars: reductions, the integrator clock and status.
 struct DevScalars {
@@ -50,6 +50,11 @@ struct DevScalars {
   unsigned long long stir_step;   // STIR phases run since sph_stir_init
   unsigned long long grav_mp, grav_pp, grav_pops;  // gravity walk diagnostics (per warp sums)
   unsigned long long grav_next;   // gravity walk: next 32-target tile (dynamic schedule)
+  // SFC decomposition (k_decomp.cu): the caller's all-reduced box / h_max
+  // (sph_set_key_box), the reduction scratch and the split bins
+  double key_box[7];              // -min x, -min y, -min z, max x, max y, max z, max h
+  unsigned long long red_ord[7];
+  int32_t splits[65];
 };
 
 // Self-gravity (k_gravity.cu).
@@ -136,6 +141,7 @@ struct Params {
   int max_cell_level;
   int divcurl, av_switch;
   int gradh, dt_vsig, ve;
+  int key_box_set;  // open axes take DevScalars::key_box (multi-rank: the global box)
 };
 
 // Process-wide count of libsph kernel launches (sph_kernel_launches).
@@ -287,7 +293,25 @@ constexpr int kRowDoubles = 11;     // SPH_ROW_DOUBLES
 constexpr int kMaxGhostRanks = 64;
 cudaError_t launch_compact(int64_t n, const uint8_t* keep, int drop, double* const* src, const int64_t* id_src,
                            double* const* dst, int64_t* id_dst, int64_t* scratch, int64_t* total,
-                           cudaStream_t st);
+                           cudaStream_t st, const uint64_t* drop_mask = nullptr);
+cudaError_t launch_decomp_reduce(int64_t n, double* const* f, const int64_t* id, unsigned long long* ord7,
+                                 double* red, cudaStream_t st);
+cudaError_t launch_key_histogram(int64_t n, const uint64_t* key, const int64_t* id, int bits, int64_t* hist,
+                                 cudaStream_t st);
+cudaError_t launch_decomp_owners(int64_t n, const uint64_t* key, const int64_t* hist, int bits, int rank,
+                                 int world, int32_t* splits, uint64_t* mig_mask, int64_t* counts,
+                                 cudaStream_t st);
+cudaError_t launch_decomp_ghosts(int64_t n, const uint64_t* key, int bits, int rank, int world,
+                                 const int32_t* splits, const DevScalars* ds, const Params& P, uint64_t* mask,
+                                 int64_t* counts, cudaStream_t st);
+cudaError_t launch_route_pack(int64_t n, const uint64_t* mask, int world, double* const* src, const int64_t* id,
+                              uint64_t or_id, double* rows, int64_t* pos, int64_t* scratch, int64_t* total,
+                              cudaStream_t st);
+cudaError_t launch_inverse_perm(int64_t n, const uint32_t* perm, uint32_t* inv, cudaStream_t st);
+cudaError_t launch_map_positions(int64_t m, const int64_t* pre, int64_t first, const uint32_t* inv, int64_t* post,
+                                 cudaStream_t st);
+cudaError_t launch_halo(int64_t m, const int64_t* idx, double* const* f, int nf, double* buf, bool gather,
+                        cudaStream_t st);
 cudaError_t launch_pack_rows(int64_t m, const int64_t* idx, double* const* src, const int64_t* id,
                              uint64_t or_id, double* dst, cudaStream_t st);
 cudaError_t launch_append_rows(int64_t m, int64_t n0, const double* rows, double* const* dst, int64_t* id,

@@ -3,28 +3,36 @@ exchange ("domain decomposition, halo exchanges",
 P:216 DomainDecompAndSync, P:220 the end-of-step collective for dt).
 
 One process per GPU.  Every rank owns a contiguous range of the 63-bit Morton
-curve; the split points come from a global histogram of the top key bits
-(all-reduce).  Each step:
+curve.  Each step (every selection, count, split, pack and map is a libsph
+device call, include/sph.h "SFC decomposition on the device"; this module only
+issues the collectives between them):
 
-  1. keys of the local particles (libsph sph_build_tree), migration of the
-     particles whose key left the rank's range (all-to-all);
-  2. ghosts: every local particle within 2 h_max (minimum image) of another
-     rank's domain box is sent to it (all-to-all) with SPH_GHOST_BIT in its id;
-  3. the full hot path in libsph on locals + ghosts, with two halo refreshes of
-     the owners' values over the ghosts: rho after DENSITY (then EOS derives
-     p, c, V) and C after IAD (H2, H3 of SURVEY 8(e));
-  4. dt = global min over ranks (all-reduce), update; the ghosts are dropped
-     (sph_compact) at the start of the next step.
-The particles stay in libsph; only emigrants, ghosts and halo values move.
+  1. drop last step's ghosts (the local count is known: no sync);
+  2. global box and h_max: MAX all-reduce of 7 doubles (exact), set as the key
+     box of the open axes -- every rank's keys are the single-GPU run's;
+  3. SFC partition: key histogram (2^15 bins of the top key bits), SUM
+     all-reduce, split bins and owners on the device; the per-rank counts go
+     through one all-to-all and ONE host read (host sync 1); the migrants move as
+     rows in one all-to-all;
+  4. ghosts by cells: every particle in a cell (side >= 2 h_max) adjacent to a
+     cell of rank r is sent to r with SPH_GHOST_BIT in its id -- counts (host
+     sync 2) and rows as in 3;
+  5. one tree build (sort) of locals + ghosts; the sort's inverse permutation
+     maps the sent and received ghosts to their new positions; the libsph hot
+     path with the owners' values scattered over the ghosts after DENSITY (rho;
+     EOS then derives p, c, V), GRADH (rho with volume elements, Omega) and IAD
+     (C, the Balsara factor) -- H2/H3 of SURVEY 8(e), all-to-alls with known
+     counts;
+  6. dt: MIN all-reduce of the local min h/c on the device (P:220), update;
+     sph_timestep's dt read is host sync 3.
+The particles stay in libsph; only migrants, ghosts and halo values move.
 
 The held set is sorted in the global Morton order and every target's
-neighbours are the same particles as in a single-GPU run, so for a periodic box
-the result is bit-identical to the one-GPU step (tests/test_gpu_decomp.py).
-
-The data-path collectives are torch.distributed calls on device tensors (NCCL
-over NVLink on GPUs; gloo on host tensors in the CPU tests).  All arithmetic of
-the method stays in libsph; this module moves particles and values between
-ranks and selects which to move (plumbing).
+neighbours are the same particles as in a single-GPU run, so the result is
+bit-identical to the one-GPU step, for periodic and open boxes alike
+(tests/test_gpu_decomp.py).  Collectives are torch.distributed calls on device
+tensors (NCCL over NVLink on GPUs; gloo, via host copies, in the tests that run
+several ranks on one GPU or on the CPU).
 """
 from __future__ import annotations
 
@@ -34,7 +42,8 @@ import torch.distributed as dist
 
 GHOST_BIT = 1 << 62
 STATE = ("x", "y", "z", "vx", "vy", "vz", "h", "m", "u", "du_m1")
-HIST_BITS = 15  # SFC partition granularity: 2^15 bins of the top key bits
+HIST_BITS = 15  # SFC partition granularity: 2^15 bins of the top key bits (level-5 cells)
+ROW = 11        # SPH_ROW_DOUBLES
 
 
 # ----------------------------------------------------------------------------- comm
@@ -55,6 +64,35 @@ class Comm:
         x = self._to(t.clone())
         dist.all_reduce(x, op=op)
         return x.to(t.device)
+
+    def all_reduce_(self, t, op):
+        """In-place all-reduce of a device tensor (gloo: through a host copy)."""
+        if self.world == 1:
+            return t
+        if self.host:
+            x = t.cpu()
+            dist.all_reduce(x, op=op)
+            t.copy_(x)
+        else:
+            dist.all_reduce(t, op=op)
+        return t
+
+    def all_to_all(self, recv, send, recv_counts, send_counts):
+        """Rows send[sum send_counts, ...] -> recv[sum recv_counts, ...] (dim-0
+        splits known on the host: no count exchange here)."""
+        if self.world == 1:
+            if recv.numel():
+                recv.copy_(send)
+            return recv
+        if self.host:
+            r = torch.empty(recv.shape, dtype=recv.dtype)
+            dist.all_to_all_single(r, send.cpu().contiguous(), [int(c) for c in recv_counts],
+                                   [int(c) for c in send_counts])
+            recv.copy_(r)
+        else:
+            dist.all_to_all_single(recv, send.contiguous(), [int(c) for c in recv_counts],
+                                   [int(c) for c in send_counts])
+        return recv
 
     def all_gather(self, t):
         if self.world == 1:
@@ -84,65 +122,6 @@ class Comm:
         return list(torch.split(recv, [int(c) for c in rc], 0))
 
 
-# ----------------------------------------------------------------------------- partition
-def sfc_splits(keys, comm: Comm, bits: int = HIST_BITS):
-    """Split bins of the global key histogram: rank r owns bins [s[r], s[r+1])."""
-    nb = 1 << bits
-    b = (keys >> (63 - bits)).to(torch.int64)
-    hist = torch.bincount(b, minlength=nb).to(torch.int64)
-    hist = comm.all_reduce(hist, dist.ReduceOp.SUM if comm.world > 1 else None)
-    cum = torch.cumsum(hist, 0)
-    total = int(cum[-1])
-    targets = torch.tensor([total * r // comm.world for r in range(1, comm.world)], dtype=torch.int64,
-                           device=cum.device)
-    inner = torch.searchsorted(cum, targets, right=True)  # first bin past each quota
-    s = torch.cat([torch.zeros(1, dtype=torch.int64, device=cum.device), inner,
-                   torch.full((1,), nb, dtype=torch.int64, device=cum.device)])
-    return s
-
-
-def owners(keys, splits, bits: int = HIST_BITS):
-    b = (keys >> (63 - bits)).to(torch.int64)
-    return torch.searchsorted(splits, b, right=True) - 1
-
-
-def domain_boxes(x, comm: Comm):
-    """[world, 2, 3] bounding boxes (min, max) of every rank's particles."""
-    if x.shape[0]:
-        lo, hi = x.min(0).values, x.max(0).values
-    else:
-        lo = torch.full((3,), float("inf"), dtype=x.dtype, device=x.device)
-        hi = torch.full((3,), -float("inf"), dtype=x.dtype, device=x.device)
-    return torch.stack(comm.all_gather(torch.stack([lo, hi])))
-
-
-def box_distance(x, lo, hi, box_len, periodic):
-    """Minimum-image distance of points x [n,3] to the axis-aligned box [lo, hi]."""
-    d2 = torch.zeros(x.shape[0], dtype=x.dtype, device=x.device)
-    for a in range(3):
-        if periodic[a]:
-            best = None
-            for k in (-1.0, 0.0, 1.0):
-                xa = x[:, a] + k * box_len[a]
-                da = torch.clamp(torch.maximum(lo[a] - xa, xa - hi[a]), min=0.0)
-                best = da if best is None else torch.minimum(best, da)
-        else:
-            best = torch.clamp(torch.maximum(lo[a] - x[:, a], x[:, a] - hi[a]), min=0.0)
-        d2 = d2 + best * best
-    return torch.sqrt(d2)
-
-
-def ghost_masks(x, boxes, rank, radius, box_len, periodic):
-    """masks[r]: local particles within `radius` of rank r's domain box (r != rank)."""
-    out = []
-    for r in range(boxes.shape[0]):
-        if r == rank or not torch.isfinite(boxes[r]).all():
-            out.append(torch.zeros(x.shape[0], dtype=torch.bool, device=x.device))
-            continue
-        out.append(box_distance(x, boxes[r, 0], boxes[r, 1], box_len, periodic) < radius)
-    return out
-
-
 # ----------------------------------------------------------------------------- rows
 def pack(state, idx=None):
     """Particles as rows [n, 11] of float64 (id bit-cast into the last column)."""
@@ -155,15 +134,6 @@ def unpack(rows):
     st = {k: rows[:, c].contiguous() for c, k in enumerate(STATE)}
     st["id"] = rows[:, len(STATE)].contiguous().view(torch.int64)
     return st
-
-
-def positions_of(ids_current, query):
-    """Positions in the current order of the particles with ids `query`."""
-    order = torch.argsort(ids_current)
-    srt = ids_current[order]
-    p = torch.searchsorted(srt, query)
-    assert bool((srt[p.clamp(max=srt.numel() - 1)] == query).all()), "halo id not found"
-    return order[p]
 
 
 # ----------------------------------------------------------------------------- stepping
@@ -212,6 +182,7 @@ class DistributedSim:
             self.sim.set_particles({k: st[k].to(self.dev).contiguous() for k in STATE + ("id",)})
         self.sim.set_time(self.t, self.dt_prev, self.first)
         self.has_ghosts = False
+        self.n_local = self.sim.n
 
     def _mark(self, name):
         if self.profile is None:
@@ -241,70 +212,62 @@ class DistributedSim:
         caller.wait_stream(self.sim.stream)  # the caller's later work (events, copies) follows the step
         return dt
 
-    def _exchange_rows(self, idx, dest, or_id=0):
-        """Rows of the particles idx (current order) to ranks dest; returns the
-        received rows (cat, in source-rank order) and the per-source counts."""
-        world = self.comm.world
-        order = torch.argsort(dest, stable=True)
-        idx = idx[order]
-        counts = torch.bincount(dest, minlength=world).cpu().tolist()
-        rows = self.sim.pack_rows(idx, or_id)
-        recv = self.comm.alltoallv(list(torch.split(rows, counts, 0)))
-        return torch.cat(recv, 0), [int(r.shape[0]) for r in recv], idx, counts
-
     def _step(self):
         comm, sim = self.comm, self.sim
         world, rank = comm.world, comm.rank
         xchg = world > 1 or self.xchg
+        dev = self.dev
         self._mark(None)
         if xchg:
-            # 1. drop last step's ghosts; keys in the current order; SFC partition
+            # 1. last step's ghosts out: the local count is known, no sync
             if self.has_ghosts:
-                sim.compact(drop_ghosts=True)
+                sim.decomp_drop(None, self.n_local)
+            # 2. global box and h_max (exact MAX), the key box of the open axes
+            red = sim.decomp_reduce()
+            comm.all_reduce_(red, dist.ReduceOp.MAX)
+            sim.set_key_box(red)
+            # 3. SFC partition and migration
             sim.compute_keys()
-            keys = self._field("key", torch.int64)
-            splits = sfc_splits(keys, comm)
-            own = owners(keys, splits)
-            self._mark("keys_partition")
-            # migration: particles whose key left this rank's range
-            emig = own != rank
-            eidx = torch.nonzero(emig).flatten()
-            rows, _, _, _ = self._exchange_rows(eidx, own[eidx])
-            sim.compact(keep=~emig)
-            sim.append_rows(rows)
-            self._mark("migrate")
-            # 2. ghosts within 2 h_max of every other rank's domain box
-            x = torch.stack([self._field("x"), self._field("y"), self._field("z")], 1)
-            hl = self._field("h")
-            hmax = comm.all_reduce(hl.max().reshape(1) if hl.numel() else
-                                   torch.zeros(1, dtype=torch.float64, device=self.dev),
-                                   dist.ReduceOp.MAX if world > 1 else None)
-            boxes = domain_boxes(x, comm)
-            radius = float(2.0 * hmax.item()) * (1.0 + 1e-9)
-            mask = sim.select_ghosts(boxes.reshape(world, 6).cpu().numpy(), rank, radius)
-            gidx, gdest = [], []
-            for r in range(world):
-                if r == rank:
-                    continue
-                ir = torch.nonzero((mask >> r) & 1).flatten()
-                gidx.append(ir)
-                gdest.append(torch.full_like(ir, r))
-            e = torch.zeros(0, dtype=torch.int64, device=self.dev)
-            gidx, gdest = torch.cat(gidx + [e]), torch.cat(gdest + [e])
-            grows, gcounts, sent_idx, scounts = self._exchange_rows(gidx, gdest, GHOST_BIT)
-            n_loc = sim.n
-            sim.append_rows(grows)
+            hist = sim.key_histogram(HIST_BITS)
+            comm.all_reduce_(hist, dist.ReduceOp.SUM)
+            mig, own = sim.decomp_owners(hist, HIST_BITS, rank, world)
+            send = own.clone()
+            send[rank] = 0
+            recv = torch.empty_like(send)
+            comm.all_to_all(recv, send, [1] * world, [1] * world)
+            host = torch.cat([own, recv]).tolist()                         # host sync 1
+            keep = int(host[rank])
+            send_c = [0 if r == rank else int(host[r]) for r in range(world)]
+            recv_c = [int(v) for v in host[world:]]
+            rows, _ = sim.decomp_pack(mig, world, sum(send_c))
+            rrows = torch.empty((sum(recv_c), ROW), dtype=torch.float64, device=dev)
+            comm.all_to_all(rrows, rows, recv_c, send_c)
+            sim.decomp_drop(mig, keep)
+            if rrows.shape[0]:
+                sim.append_rows(rrows)
+            self.n_local = keep + sum(recv_c)
+            self._mark("partition_migrate")
+            # 4. ghosts by cells
+            sim.compute_keys()
+            gmask, gcnt = sim.decomp_ghosts(HIST_BITS, rank, world)
+            grecv = torch.empty_like(gcnt)
+            comm.all_to_all(grecv, gcnt, [1] * world, [1] * world)
+            gh = torch.cat([gcnt, grecv]).tolist()                         # host sync 2
+            self.g_send = [int(v) for v in gh[:world]]
+            self.g_recv = [int(v) for v in gh[world:]]
+            grows, gpos = sim.decomp_pack(gmask, world, sum(self.g_send), GHOST_BIT)
+            grr = torch.empty((sum(self.g_recv), ROW), dtype=torch.float64, device=dev)
+            comm.all_to_all(grr, grows, self.g_recv, self.g_send)
+            if grr.shape[0]:
+                sim.append_rows(grr)
             self.has_ghosts = True
-            self.stats = {"n_local": n_loc, "n_ghost": int(sum(gcounts))}
+            self.stats = {"n_local": self.n_local, "n_ghost": sum(self.g_recv), "n_migrated_in": sum(recv_c)}
             self._mark("ghosts")
-        # 3. the hot path with the halo refreshes
+        # 5. one tree build of locals + ghosts, the halo maps, the hot path
         sim.build_tree()
         if xchg:
-            order = self._field("order", torch.int32).to(torch.int64)
-            inv = torch.empty_like(order)
-            inv[order] = torch.arange(order.numel(), device=self.dev)
-            self._src = torch.split(inv[sent_idx], scounts, 0)              # mine others hold
-            self._dst = inv[n_loc:n_loc + sum(gcounts)]                      # theirs I hold
+            self._src = sim.decomp_map(gpos)                                   # mine that others hold
+            self._dst = sim.decomp_map(None, first=self.n_local, m=sum(self.g_recv))  # theirs I hold
             self._mark("tree_maps")
         sim.find_neighbors(stats=False)
         sim.density()
@@ -324,12 +287,12 @@ class DistributedSim:
         if sim.stir_enabled:  # driving: every rank holds the same OU state and noise
             sim.stir()
         self._mark("physics_halos")
-        # 4. global dt, update (ghosts are dropped at the next step)
+        # 6. global dt on the device, update
         if xchg:
-            mhc = torch.tensor([sim.get_local_min_hc()], dtype=torch.float64, device=self.dev)
-            mhc = comm.all_reduce(mhc, dist.ReduceOp.MIN if world > 1 else None)
-            sim.set_global_min_hc(float(mhc.item()))
-        dt = sim.timestep()
+            mhc = sim.min_hc_dev()
+            comm.all_reduce_(mhc, dist.ReduceOp.MIN)
+            sim.set_min_hc_dev(mhc)
+        dt = sim.timestep()                                                # host sync 3
         sim.update()
         self.t, self.dt_prev, self.first = self.t + dt, dt, False
         self._mark("dt_update")
@@ -339,10 +302,11 @@ class DistributedSim:
         if not (self.comm.world > 1 or self.xchg):
             return
         sim = self.sim
-        parts = [torch.stack([sim.gather_field(k, p) for k in names], 1) for p in self._src]
-        recv = torch.cat(self.comm.alltoallv(parts), 0)
-        for c, k in enumerate(names):
-            sim.scatter_field(k, self._dst, recv[:, c].contiguous())
+        send = sim.halo_gather(names, self._src)
+        recv = torch.empty((sum(self.g_recv), len(names)), dtype=torch.float64, device=self.dev)
+        self.comm.all_to_all(recv, send, self.g_recv, self.g_send)
+        if recv.shape[0]:
+            sim.halo_scatter(names, self._dst, recv)
 
     def gather_state(self):
         """All particles on every rank, sorted by id (host numpy) -- for tests."""

@@ -76,6 +76,12 @@ class EnergyRow(C.Structure):
                 ("locked_mhz", C.c_uint32), ("available", C.c_int32)]
 
 
+class EnergyWindow(C.Structure):
+    _fields_ = [("wall_seconds", C.c_double), ("sampled_seconds", C.c_double),
+                ("sampled_joules", C.c_double), ("between_joules", C.c_double),
+                ("counter_joules", C.c_double), ("samples", C.c_int64)]
+
+
 class StirParams(C.Structure):
     _fields_ = [("sigma", C.c_double), ("t_decay", C.c_double), ("sol_weight", C.c_double)]
 
@@ -91,13 +97,16 @@ EXPORTS = ("sph_config_default", "sph_workspace_size", "sph_init", "sph_finalize
            "sph_get_time", "sph_get_n", "sph_get_field", "sph_build_tree", "sph_find_neighbors",
            "sph_get_neighbors", "sph_density", "sph_eos", "sph_iad", "sph_momentum_energy",
            "sph_timestep", "sph_update", "sph_step", "sph_set_clock_policy",
-           "sph_energy_report", "sph_energy_reset", "sph_energy_counter_mj", "sph_repeat_phase",
+           "sph_energy_report", "sph_energy_reset", "sph_energy_counter_mj", "sph_energy_totals", "sph_repeat_phase",
            "sph_set_accounting", "sph_kernel_launches", "sph_set_field",
            "sph_get_local_min_hc", "sph_set_global_min_hc", "sph_get_neighbor_rows",
            "sph_trace_start", "sph_trace_stop", "sph_stir_modes", "sph_stir_init", "sph_stir",
            "sph_stir_get_state", "sph_supported_clocks", "sph_gravity", "sph_gradh",
            "sph_compute_keys", "sph_compact", "sph_pack_rows", "sph_append_rows",
-           "sph_select_ghosts", "sph_gather_field", "sph_scatter_field")
+           "sph_select_ghosts", "sph_gather_field", "sph_scatter_field",
+           "sph_decomp_reduce", "sph_set_key_box", "sph_key_histogram", "sph_decomp_owners",
+           "sph_decomp_ghosts", "sph_decomp_pack", "sph_decomp_drop", "sph_decomp_map",
+           "sph_halo_gather", "sph_halo_scatter", "sph_min_hc_dev", "sph_set_min_hc_dev")
 GHOST_BIT = 1 << 62
 
 _lib = None
@@ -140,6 +149,7 @@ def load(build_if_missing: bool = True):
     L.sph_set_clock_policy.argtypes = [P, I, C.POINTER(C.c_uint32)]
     L.sph_energy_report.argtypes = [P, C.POINTER(EnergyRow), I, C.POINTER(I)]
     L.sph_energy_counter_mj.argtypes = [P, C.POINTER(C.c_uint64)]
+    L.sph_energy_totals.argtypes = [P, C.POINTER(EnergyWindow)]
     L.sph_repeat_phase.argtypes = [P, I, I, C.POINTER(D), C.POINTER(D)]
     L.sph_set_accounting.argtypes = [P, I]
     L.sph_set_field.argtypes = [P, I, V, I]
@@ -160,6 +170,18 @@ def load(build_if_missing: bool = True):
     L.sph_gather_field.argtypes = [P, I, V, I64, V]
     L.sph_scatter_field.argtypes = [P, I, V, I64, V]
     L.sph_stir_get_state.argtypes = [P, V, C.POINTER(I64)]
+    L.sph_decomp_reduce.argtypes = [P, V]
+    L.sph_set_key_box.argtypes = [P, V]
+    L.sph_key_histogram.argtypes = [P, I, V]
+    L.sph_decomp_owners.argtypes = [P, V, I, I, I, V, V]
+    L.sph_decomp_ghosts.argtypes = [P, I, I, I, V, V]
+    L.sph_decomp_pack.argtypes = [P, V, I, C.c_uint64, V, V]
+    L.sph_decomp_drop.argtypes = [P, V, I64]
+    L.sph_decomp_map.argtypes = [P, V, I64, I64, V]
+    L.sph_halo_gather.argtypes = [P, V, I, V, I64, V]
+    L.sph_halo_scatter.argtypes = [P, V, I, V, I64, V]
+    L.sph_min_hc_dev.argtypes = [P, V]
+    L.sph_set_min_hc_dev.argtypes = [P, V]
     L.sph_supported_clocks.argtypes = [P, V, I, C.POINTER(I)]
     L.sph_trace_start.argtypes = [P, D, I64]
     L.sph_trace_stop.argtypes = [P, V, I64, C.POINTER(I64)]
@@ -381,6 +403,94 @@ class Simulation:
         self._ok(self.L.sph_scatter_field(self.ctx, FIELD_ID[name], C.c_void_p(idx.data_ptr()), idx.numel(),
                                           C.c_void_p(src.data_ptr())))
 
+    # ------------------------------------------ SFC decomposition on the device (8(e))
+    # All tensors are cuda tensors on self.device; callers run under
+    # torch.cuda.stream(self.stream).  Nothing here synchronises.
+    def _t(self, a):
+        self._keep_field = a
+        return C.c_void_p(a.data_ptr()) if a is not None else None
+
+    def decomp_reduce(self):
+        """float64 [7]: (-min x, -min y, -min z, max x, max y, max z, max h) of the non-ghosts."""
+        red = self.torch.empty(7, dtype=self.torch.float64, device=self.device)
+        self._ok(self.L.sph_decomp_reduce(self.ctx, self._t(red)))
+        return red
+
+    def set_key_box(self, red):
+        self._keep_box = red
+        self._ok(self.L.sph_set_key_box(self.ctx, None if red is None else C.c_void_p(red.data_ptr())))
+
+    def key_histogram(self, bits: int):
+        hist = self.torch.empty(1 << bits, dtype=self.torch.int64, device=self.device)
+        self._ok(self.L.sph_key_histogram(self.ctx, int(bits), self._t(hist)))
+        return hist
+
+    def decomp_owners(self, hist, bits: int, rank: int, world: int):
+        """(migration mask int64 [n] = 1 << owner or 0, counts int64 [world])."""
+        mask = self.torch.empty(max(self.n, 1), dtype=self.torch.int64, device=self.device)
+        counts = self.torch.empty(world, dtype=self.torch.int64, device=self.device)
+        self._keep_hist = hist
+        self._ok(self.L.sph_decomp_owners(self.ctx, C.c_void_p(hist.data_ptr()), int(bits), int(rank), int(world),
+                                          C.c_void_p(mask.data_ptr()), C.c_void_p(counts.data_ptr())))
+        return mask[:self.n], counts
+
+    def decomp_ghosts(self, bits: int, rank: int, world: int):
+        """(ghost mask int64 [n], counts int64 [world])."""
+        mask = self.torch.empty(max(self.n, 1), dtype=self.torch.int64, device=self.device)
+        counts = self.torch.empty(world, dtype=self.torch.int64, device=self.device)
+        self._ok(self.L.sph_decomp_ghosts(self.ctx, int(bits), int(rank), int(world), C.c_void_p(mask.data_ptr()),
+                                          C.c_void_p(counts.data_ptr())))
+        return mask[:self.n], counts
+
+    def decomp_pack(self, mask, world: int, total: int, or_id: int = 0):
+        """(rows [total, ROW_DOUBLES], pos int64 [total]) grouped by destination rank."""
+        rows = self.torch.empty((max(total, 1), ROW_DOUBLES), dtype=self.torch.float64, device=self.device)
+        pos = self.torch.empty(max(total, 1), dtype=self.torch.int64, device=self.device)
+        self._keep_mask = mask
+        self._ok(self.L.sph_decomp_pack(self.ctx, C.c_void_p(mask.data_ptr()), int(world), C.c_uint64(or_id),
+                                        C.c_void_p(rows.data_ptr()), C.c_void_p(pos.data_ptr())))
+        return rows[:total], pos[:total]
+
+    def decomp_drop(self, mask, n_expected: int):
+        """Keep mask == 0 (mask None: drop the ghosts); the new n is n_expected (no sync)."""
+        self._keep_mask = mask
+        self._ok(self.L.sph_decomp_drop(self.ctx, None if mask is None else C.c_void_p(mask.data_ptr()),
+                                        int(n_expected)))
+        self.n = int(n_expected)
+
+    def decomp_map(self, pre=None, first: int = 0, m: int | None = None):
+        """Post-sort positions of pre-sort positions (pre, or first + arange(m))."""
+        m = int(pre.numel()) if pre is not None else int(m)
+        post = self.torch.empty(max(m, 1), dtype=self.torch.int64, device=self.device)
+        self._keep_pre = pre
+        self._ok(self.L.sph_decomp_map(self.ctx, None if pre is None else C.c_void_p(pre.data_ptr()), int(first), m,
+                                       C.c_void_p(post.data_ptr())))
+        return post[:m]
+
+    def halo_gather(self, names, idx):
+        f = (C.c_int32 * len(names))(*[FIELD_ID[k] for k in names])
+        out = self.torch.empty((max(idx.numel(), 1), len(names)), dtype=self.torch.float64, device=self.device)
+        self._keep_idx = idx
+        self._ok(self.L.sph_halo_gather(self.ctx, f, len(names), C.c_void_p(idx.data_ptr()), idx.numel(),
+                                        C.c_void_p(out.data_ptr())))
+        return out[:idx.numel()]
+
+    def halo_scatter(self, names, idx, src):
+        f = (C.c_int32 * len(names))(*[FIELD_ID[k] for k in names])
+        src = src.contiguous()
+        self._keep_src = (idx, src)
+        self._ok(self.L.sph_halo_scatter(self.ctx, f, len(names), C.c_void_p(idx.data_ptr()), idx.numel(),
+                                         C.c_void_p(src.data_ptr())))
+
+    def min_hc_dev(self):
+        out = self.torch.empty(1, dtype=self.torch.float64, device=self.device)
+        self._ok(self.L.sph_min_hc_dev(self.ctx, C.c_void_p(out.data_ptr())))
+        return out
+
+    def set_min_hc_dev(self, v):
+        self._keep_mhc = v
+        self._ok(self.L.sph_set_min_hc_dev(self.ctx, C.c_void_p(v.data_ptr())))
+
     def get_local_min_hc(self) -> float:
         v = C.c_double()
         self._ok(self.L.sph_get_local_min_hc(self.ctx, C.byref(v)))
@@ -473,6 +583,16 @@ class Simulation:
 
     def energy_reset(self):
         self._ok(self.L.sph_energy_reset(self.ctx))
+
+    def energy_totals(self):
+        """sph_energy_totals: the accounting window since energy_reset -- sampled
+        joules (PHASE accounting) vs the NVML counter delta (None if unreadable)."""
+        t = EnergyWindow()
+        self._ok(self.L.sph_energy_totals(self.ctx, C.byref(t)))
+        return {"wall_seconds": t.wall_seconds, "sampled_seconds": t.sampled_seconds,
+                "sampled_joules": t.sampled_joules, "between_joules": t.between_joules,
+                "counter_joules": t.counter_joules if t.counter_joules >= 0 else None,
+                "samples": int(t.samples)}
 
     def energy_counter_mj(self):
         v = C.c_uint64()

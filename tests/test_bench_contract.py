@@ -32,7 +32,7 @@ def test_reference_arm_line():
 @pytest.mark.gpu
 def test_libsph_arm_line():
     d = _run(["--workload", "turbulence40", "--steps", "3", "--warmup", "3", "--e2e-steps", "1",
-              "--energy-steps", "10", "--trace-seconds", "0", "--cpu-sample", "4"])
+              "--energy-seconds", "1.5", "--energy-repeats", "1", "--trace-seconds", "0", "--cpu-sample", "4"])
     for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better",
               "scaling", "dtype", "data", "config", "roofline", "e2e", "cpu_baseline", "clocks",
               "gpu_launches", "phases"):
@@ -44,3 +44,8 @@ def test_libsph_arm_line():
     assert 0 < d["e2e"]["value"] <= d["value"] * 1.05
     assert d["gpu_launches"] > 0 and d["cpu_baseline"]["kind"] == "oracle"
     assert d["phases"]["momentum_energy"]["bound"] == "fp64" and d["phases"]["update"]["GBps"] > 0
+    assert d["repeats"]["blocks"] >= 4 and d["repeats"]["cv"] >= 0
+    e = d["energy"]
+    assert e["available"] and e["step"]["J_median"] > 0 and e["phases"]["momentum_energy"]["J"] > 0
+    assert d["cpu_baseline"]["physics_only"]["s_per_particle"] > 0
+    assert d["roofline"]["flops_per_pair"] == 171

@@ -1,6 +1,8 @@
-"""Host logic of the multi-GPU decomposition (paper_conf_sc_simsekpc24_b200.decomp)
-on CPU with the gloo backend, world size 2 -- partition, migration, ghost
-selection and the halo all-to-all -- checked against brute force."""
+"""Host side of the multi-GPU decomposition on CPU with the gloo backend at world
+sizes 2, 4 and 8: decomp.Comm's collectives (MAX/SUM all-reduce, all-to-all with
+host counts) driving the selection logic of tests/decomp_reference.py (global
+box, SFC split points, owners, cell-stencil ghosts) -- checked against the
+one-rank box and brute-force neighbours, periodic and open boxes."""
 import os
 import socket
 
@@ -10,6 +12,7 @@ import torch
 import torch.distributed as dist
 import torch.multiprocessing as mp
 
+import decomp_reference as ref
 import oracle
 from paper_conf_sc_simsekpc24_b200 import decomp, ics
 
@@ -50,82 +53,99 @@ def run_world(fn, world=2):
     return [res[r] for r in range(world)]
 
 
-def _workload():
-    return ics.random_box(4000, seed=31, periodic=True)
+def _workload(case="periodic"):
+    if case == "periodic":
+        return ics.random_box(4000, seed=31, periodic=True)
+    w = ics.noh(16)  # open box (bounding box per step)
+    return w
 
 
-def _keys(w):
+def _route_fn(rank, world, case):
+    """One rank of the decomposition's selection logic (tests/decomp_reference.py)
+    driven through decomp.Comm's real collectives: global box (MAX), key
+    histogram (SUM), migration and ghost rows (all-to-all with host counts)."""
+    w = _workload(case)
     s = w.state
-    bmin, bmax = oracle.box(s["x"], s["y"], s["z"], w.params)
-    return oracle.keys(s["x"], s["y"], s["z"], bmin, bmax)
-
-
-def _partition_fn(rank, world):
-    w = _workload()
-    k = _keys(w)
+    comm = decomp.Comm()
     mine = np.arange(w.n)[rank::world]          # arbitrary initial distribution
-    comm = decomp.Comm()
-    kt = torch.from_numpy(k[mine].astype(np.int64))
-    splits = decomp.sfc_splits(kt, comm)
-    own = decomp.owners(kt, splits)
-    st = {f: torch.from_numpy(np.ascontiguousarray(w.state[f][mine])) for f in decomp.STATE + ("id",)}
+    red = torch.from_numpy(ref.red7(s["x"][mine], s["y"][mine], s["z"][mine], s["h"][mine]))
+    comm.all_reduce_(red, dist.ReduceOp.MAX)
+    lo, hi = ref.key_box(red.numpy(), w.params)
+    keys_all = oracle.keys(s["x"], s["y"], s["z"], lo, hi)
+    k = keys_all[mine]
+    hist = torch.from_numpy(np.bincount((k >> np.uint64(63 - ref.HIST_BITS)).astype(np.int64),
+                                        minlength=1 << ref.HIST_BITS).astype(np.int64))
+    comm.all_reduce_(hist, dist.ReduceOp.SUM)
+    splits = ref.splits_from_hist(hist.numpy(), world)
+    own = ref.owners(k, splits)
+    st = {f: torch.from_numpy(np.ascontiguousarray(s[f][mine])) for f in decomp.STATE + ("id",)}
     rows = decomp.pack(st)
-    got = decomp.unpack(torch.cat(comm.alltoallv([rows[own == r] for r in range(world)]), 0))
-    return splits.numpy(), got["id"].numpy()
+
+    def exchange(sel_rows, dest_lists):
+        send_c = [len(d) for d in dest_lists]
+        sc = torch.tensor(send_c, dtype=torch.int64)
+        rc = torch.empty_like(sc)
+        comm.all_to_all(rc, sc, [1] * world, [1] * world)
+        send = torch.cat([sel_rows[d] for d in dest_lists], 0) if sum(send_c) else torch.zeros((0, decomp.ROW), dtype=torch.float64)
+        recv = torch.empty((int(rc.sum()), decomp.ROW), dtype=torch.float64)
+        comm.all_to_all(recv, send, rc.tolist(), send_c)
+        return decomp.unpack(recv)
+
+    mig = exchange(rows, [torch.from_numpy(np.nonzero((own == r) & (r != rank))[0]) for r in range(world)])
+    keep = own == rank
+    loc = {f: torch.cat([st[f][torch.from_numpy(keep)], mig[f]]) for f in st}
+    ids = loc["id"].numpy()
+    # ghosts by cells of the new locals (keys from the same global box)
+    kl = keys_all[ids]
+    gm = ref.ghost_masks_cells(kl, lo, hi, float(red[6]), w.params.periodic, splits, rank, world)
+    lrows = decomp.pack(loc)
+    g = exchange(lrows, [torch.from_numpy(np.nonzero((gm >> np.uint64(r)) & np.uint64(1))[0]) for r in range(world)])
+    return splits, red.numpy(), ids, g["id"].numpy()
 
 
-def test_partition_and_migration():
-    (s0, ids0), (s1, ids1) = run_world(_partition_fn)
-    assert np.array_equal(s0, s1), "every rank computes the same split points"
-    w = _workload()
-    k = _keys(w)
-    # ownership is a contiguous key range, complete and disjoint
-    assert len(set(ids0) & set(ids1)) == 0 and len(ids0) + len(ids1) == w.n
-    b = (k >> np.uint64(63 - decomp.HIST_BITS)).astype(np.int64)
-    assert np.all(b[ids0] < s0[1]) and np.all(b[ids1] >= s0[1])
-    # balanced to within one histogram bin's worth of particles
-    assert abs(len(ids0) - len(ids1)) < 0.05 * w.n
-
-
-def _ghost_fn(rank, world):
-    w = _workload()
-    k = _keys(w)
-    comm = decomp.Comm()
-    kt = torch.from_numpy(k.astype(np.int64))
-    splits = decomp.sfc_splits(kt[rank::world], comm)
-    own = decomp.owners(kt, splits).numpy()
-    mine = np.nonzero(own == rank)[0]
-    x = torch.from_numpy(np.stack([w.state[a][mine] for a in ("x", "y", "z")], 1))
-    boxes = decomp.domain_boxes(x, comm)
-    radius = 2.0 * float(w.state["h"].max()) * (1 + 1e-9)
-    box_len = [b - a for a, b in zip(w.params.box_min, w.params.box_max)]
-    masks = decomp.ghost_masks(x, boxes, rank, radius, box_len, w.params.periodic)
-    st = {f: torch.from_numpy(np.ascontiguousarray(w.state[f][mine])) for f in decomp.STATE + ("id",)}
-    rows = decomp.pack(st)
-    recv = comm.alltoallv([rows[m] for m in masks])
-    ghosts = np.concatenate([decomp.unpack(r)["id"].numpy() for r in recv])
-    return mine, ghosts
-
-
-def test_ghosts_cover_every_neighbour():
-    """Locals + ghosts of each rank contain every brute-force neighbour of its
-    locals (the halo is conservative), and no rank receives its own particles."""
-    res = run_world(_ghost_fn)
-    w = _workload()
+@pytest.mark.parametrize("case,world", [("periodic", 2), ("periodic", 4), ("open", 4), ("periodic", 8)])
+def test_route_partition_and_halo_coverage(case, world):
+    """Every rank computes the same global box and split points; ownership is
+    complete, disjoint and a contiguous key range per rank, balanced to within a
+    histogram bin; locals + ghosts of each rank hold every brute-force neighbour
+    of its locals (the cell-stencil halo is conservative), and no rank receives
+    its own particles as ghosts."""
+    import functools
+    res = run_world(functools.partial(_route_fn, case=case), world=world)
+    w = _workload(case)
     s = w.state
+    for r in range(1, world):
+        assert np.array_equal(res[r][0], res[0][0]) and np.array_equal(res[r][1], res[0][1])
     bmin, bmax = oracle.box(s["x"], s["y"], s["z"], w.params)
+    lo, hi = ref.key_box(res[0][1], w.params)
+    assert np.array_equal(lo, bmin) and np.array_equal(hi, bmax), "the global box is the one-rank box"
+    keys = oracle.keys(s["x"], s["y"], s["z"], bmin, bmax)
+    bins = (keys >> np.uint64(63 - ref.HIST_BITS)).astype(np.int64)
+    splits = res[0][0]
+    all_ids = np.concatenate([r[2] for r in res])
+    assert np.array_equal(np.sort(all_ids), np.arange(w.n)), "ownership complete and disjoint"
+    for r, (_, _, ids, _) in enumerate(res):
+        assert np.all((bins[ids] >= splits[r]) & (bins[ids] < splits[r + 1]))
+        assert abs(len(ids) - w.n / world) < 0.05 * w.n
     nb = oracle.neighbors(s["x"], s["y"], s["z"], s["h"], bmin, bmax, w.params.periodic)
-    for mine, ghosts in res:
-        held = set(mine.tolist()) | set(ghosts.tolist())
-        assert not set(ghosts.tolist()) & set(mine.tolist())
-        need = set(nb.idx[np.concatenate([np.arange(nb.offsets[i], nb.offsets[i + 1]) for i in mine])].tolist())
-        assert need <= held
+    for r, (_, _, ids, ghosts) in enumerate(res):
+        held = set(ids.tolist()) | set(ghosts.tolist())
+        assert not set(ghosts.tolist()) & set(ids.tolist())
+        need = set(nb.idx[np.concatenate([np.arange(nb.offsets[i], nb.offsets[i + 1]) for i in ids])].tolist())
+        assert need <= held, f"rank {r} misses {len(need - held)} neighbours"
+        assert len(ghosts) < 0.9 * w.n  # not everything
 
 
-def test_positions_of_and_pack_roundtrip():
+def test_splits_reference_edge_cases():
+    assert ref.splits_from_hist(np.zeros(8, np.int64), 3).tolist() == [0, 8, 8, 8]
+    h = np.zeros(8, np.int64)
+    h[5] = 10
+    assert ref.splits_from_hist(h, 2).tolist() == [0, 5, 8]
+    assert ref.splits_from_hist(np.ones(8, np.int64), 4).tolist() == [0, 2, 4, 6, 8]
+
+
+def test_pack_roundtrip():
     ids = torch.tensor([7, 3, 11, 5, 1 | decomp.GHOST_BIT], dtype=torch.int64)
-    q = torch.tensor([11, 1 | decomp.GHOST_BIT, 7], dtype=torch.int64)
-    assert decomp.positions_of(ids, q).tolist() == [2, 4, 0]
     st = {f: torch.arange(5, dtype=torch.float64) * (c + 1) for c, f in enumerate(decomp.STATE)}
     st["id"] = ids
     back = decomp.unpack(decomp.pack(st))
@@ -137,8 +157,8 @@ def test_box_distance_minimum_image():
     x = torch.tensor([[0.49, 0.0, 0.0], [-0.3, 0.0, 0.0]], dtype=torch.float64)
     lo = torch.tensor([-0.5, -0.1, -0.1], dtype=torch.float64)
     hi = torch.tensor([-0.45, 0.1, 0.1], dtype=torch.float64)
-    d = decomp.box_distance(x, lo, hi, [1.0, 1.0, 1.0], (1, 1, 1))
+    d = ref.box_distance(x, lo, hi, [1.0, 1.0, 1.0], (1, 1, 1))
     assert d[0].item() == pytest.approx(0.01, abs=1e-12)   # through the periodic face
     assert d[1].item() == pytest.approx(0.15, abs=1e-12)
-    d = decomp.box_distance(x, lo, hi, [1.0, 1.0, 1.0], (0, 1, 1))
+    d = ref.box_distance(x, lo, hi, [1.0, 1.0, 1.0], (0, 1, 1))
     assert d[0].item() == pytest.approx(0.94, abs=1e-12)

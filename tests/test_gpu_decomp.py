@@ -47,8 +47,16 @@ def _random_ve():
     return w
 
 
+def _noh():
+    import dataclasses
+    w = ics.noh(14)  # open box: the global key box of sph_set_key_box
+    w.params = dataclasses.replace(w.params, dt_vsig=1, ngmax=400)
+    return w
+
+
 def _make(name):
     return {"turbulence16": lambda: ics.turbulence(16), "random": lambda: ics.random_box(6000, seed=5),
+            "noh14_open": _noh,
             "sedov14": lambda: ics.sedov(14), "sedov14_balsara": _sedov_balsara,
             "random_gradh_vsig": _random_gradh_vsig, "random_ve": _random_ve}[name]()
 
@@ -85,7 +93,7 @@ def _single(name):
 
 
 @pytest.mark.parametrize("name", ["turbulence16", "random", "sedov14", "sedov14_balsara",
-                                  "random_gradh_vsig", "random_ve"])
+                                  "random_gradh_vsig", "random_ve", "noh14_open"])
 def test_two_ranks_bit_identical_to_one(name):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
@@ -137,7 +145,8 @@ def test_one_rank_forced_plumbing_equals_plain():
 def test_device_plumbing_matches_host_logic():
     """sph_select_ghosts == decomp.ghost_masks; compact / pack / append /
     gather / scatter move exactly the selected particles."""
-    from paper_conf_sc_simsekpc24_b200 import decomp, sph
+    import decomp_reference as ref
+    from paper_conf_sc_simsekpc24_b200 import sph
     w = ics.random_box(5000, seed=11)
     sim = sph.Simulation(w.params, n_capacity=2 * w.n)
     sim.set_particles({k: np.ascontiguousarray(v) for k, v in w.state.items()})
@@ -148,7 +157,7 @@ def test_device_plumbing_matches_host_logic():
                               [[0.1, 0.1, 0.1], [0.2, 0.2, 0.3]],
                               [[float("inf")] * 3, [-float("inf")] * 3]], dtype=torch.float64, device=dev)
         box_len = [1.0, 1.0, 1.0]
-        want = decomp.ghost_masks(x, boxes, 0, 0.07, box_len, w.params.periodic)
+        want = ref.ghost_masks_boxes(x, boxes, 0, 0.07, box_len, w.params.periodic)
         got = sim.select_ghosts(boxes.reshape(4, 6).cpu().numpy(), 0, 0.07)
         for r in range(4):
             assert torch.equal(((got >> r) & 1).bool(), want[r]), r
@@ -198,4 +207,66 @@ def test_device_plumbing_edge_cases():
         sim.append_rows(rows[:10])
         st = sim.get_state()
         assert np.array_equal(st["x"], w.state["x"][:10])
+    sim.finalize()
+
+
+@pytest.mark.parametrize("case", ["periodic", "open"])
+def test_device_routing_matches_reference(case):
+    """libsph's device routing (sph_decomp_reduce / sph_key_histogram /
+    sph_decomp_owners / sph_decomp_ghosts / sph_decomp_pack / sph_decomp_drop /
+    sph_decomp_map) equals tests/decomp_reference.py element by element: one
+    context holding every particle plays rank 1 of 4."""
+    import decomp_reference as ref
+    import oracle
+    from paper_conf_sc_simsekpc24_b200 import sph
+    w = ics.random_box(7000, seed=13, periodic=True) if case == "periodic" else ics.noh(18)
+    s = w.state
+    sim = sph.Simulation(w.params, n_capacity=w.n)
+    sim.set_particles({k: np.ascontiguousarray(v) for k, v in w.state.items()})
+    sim.set_time(0.0, w.params.dt_first, True)
+    world, rank = 4, 1
+    with torch.cuda.stream(sim.stream):
+        red = sim.decomp_reduce()
+        want_red = ref.red7(s["x"], s["y"], s["z"], s["h"])
+        assert np.array_equal(red.cpu().numpy(), want_red)
+        sim.set_key_box(red)
+        sim.compute_keys()
+        keys = sim.get_field("key")
+        lo, hi = ref.key_box(want_red, w.params)
+        assert np.array_equal(keys, oracle.keys(s["x"], s["y"], s["z"], lo, hi))
+        hist = sim.key_histogram(ref.HIST_BITS)
+        want_hist = np.bincount((keys >> np.uint64(63 - ref.HIST_BITS)).astype(np.int64), minlength=1 << ref.HIST_BITS)
+        assert np.array_equal(hist.cpu().numpy(), want_hist)
+        mig, cnt = sim.decomp_owners(hist, ref.HIST_BITS, rank, world)
+        splits = ref.splits_from_hist(want_hist, world)
+        own = ref.owners(keys, splits)
+        want_mig = np.where(own == rank, 0, 1 << own).astype(np.int64)
+        assert np.array_equal(mig.cpu().numpy(), want_mig)
+        assert cnt.cpu().tolist() == [int((own == r).sum()) for r in range(world)]
+        # grouped pack: by destination rank, particle order within one
+        total = int((want_mig != 0).sum())
+        rows, pos = sim.decomp_pack(mig, world, total)
+        order = np.concatenate([np.nonzero(own == r)[0] for r in range(world) if r != rank])
+        assert np.array_equal(pos.cpu().numpy(), order)
+        assert np.array_equal(rows[:, 0].cpu().numpy(), s["x"][order])
+        # keep rank 1's particles; ghosts of them by cells
+        sim.decomp_drop(mig, int((own == rank).sum()))
+        kept = np.nonzero(own == rank)[0]
+        st = sim.get_state()
+        assert np.array_equal(st["id"], s["id"][kept])
+        sim.compute_keys()
+        gm, gc = sim.decomp_ghosts(ref.HIST_BITS, rank, world)
+        want_gm = ref.ghost_masks_cells(keys[kept], lo, hi, want_red[6], w.params.periodic, splits, rank, world)
+        assert np.array_equal(gm.cpu().numpy().view(np.uint64), want_gm)
+        assert gc.cpu().tolist() == [int(((want_gm >> np.uint64(r)) & np.uint64(1)).sum()) for r in range(world)]
+        assert gc.cpu().numpy().sum() > 0
+        # positions through the sort
+        sim.build_tree()
+        perm = sim.get_field("order").astype(np.int64)
+        pre = torch.tensor([0, 5, len(kept) - 1], dtype=torch.int64, device="cuda")
+        post = sim.decomp_map(pre).cpu().numpy()
+        inv = np.empty_like(perm)
+        inv[perm] = np.arange(perm.size)
+        assert np.array_equal(post, inv[[0, 5, len(kept) - 1]])
+        assert np.array_equal(sim.decomp_map(None, first=2, m=3).cpu().numpy(), inv[2:5])
     sim.finalize()

@@ -2,7 +2,7 @@
 # Quick GPU iteration: build, short bench (no e2e/energy/cpu legs), parity tests.
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || { echo build failed; tail gpurun_out/build.log; exit 1; }
-timeout 300 python bench.py --steps 5 --warmup 3 --e2e-steps 0 --energy-steps 0 --trace-seconds ${TRACE:-0} --no-cpu-baseline ${BENCH_ARGS} > gpurun_out/quick_bench.log 2>&1; echo "bench rc=$?"
+timeout 300 python bench.py --steps 5 --warmup 3 --e2e-steps 0 --energy-seconds 0 --timing-repeats 0 --trace-seconds ${TRACE:-0} --no-cpu-baseline ${BENCH_ARGS} > gpurun_out/quick_bench.log 2>&1; echo "bench rc=$?"
 python - <<'PY'
 import json
 for l in open('gpurun_out/quick_bench.log'):
