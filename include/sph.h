@@ -353,7 +353,8 @@ int sph_scatter_field(sph_ctx* ctx, int field, const int64_t* idx, int64_t m, co
  *   keys those of the single-GPU run.  red == NULL: each step's own box again.
  * sph_key_histogram: hist[b] (int64, 2^bits) = held non-ghost particles whose
  *   key has top bits b (after sph_compute_keys; bits a multiple of 3).
- * sph_decomp_owners: from the histogram summed over ranks, the split bins
+ * sph_decomp_owners: (ghosts held from the last step are skipped: mask 0,
+ *   not counted) from the histogram summed over ranks, the split bins
  *   s_0 = 0 <= s_1 <= .. <= s_world = 2^bits with s_r = the first bin whose
  *   inclusive prefix count exceeds floor(total r / world); rank r owns the keys
  *   of bins [s_r, s_r+1).  mig_mask[i] = 1 << owner(i) if owner(i) != rank
@@ -367,8 +368,9 @@ int sph_scatter_field(sph_ctx* ctx, int field, const int64_t* idx, int64_t m, co
  * sph_decomp_pack: one row per (particle i, rank r in mask[i]), grouped by r in
  *   rank order and in particle order within r (id OR-ed with or_id);
  *   pos[e] = i of row e.  rows/pos hold sum_i popcount(mask[i]) entries.
- * sph_decomp_drop: stable compaction keeping the particles with
- *   drop_mask[i] == 0 (drop_mask == NULL: the non-ghosts); the new count is the caller's n_expected (from the
+ * sph_decomp_drop: stable compaction keeping the non-ghosts with
+ *   drop_mask[i] == 0 (drop_mask may be NULL; n_expected == n: nothing to
+ *   do); the new count is the caller's n_expected (from the
  *   counts, no synchronisation); a different device count is reported as
  *   SPH_ERR_STATE at the next synchronising call.
  * sph_decomp_map: after sph_build_tree, the positions after its sort of the

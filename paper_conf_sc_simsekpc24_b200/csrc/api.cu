@@ -1090,8 +1090,8 @@ int sph_decomp_owners(sph_ctx* c, const int64_t* hist, int bits, int rank, int w
     return fail(c, SPH_ERR_ARG, "bad bits / buffers");
   if (world < 1 || world > kMaxGhostRanks || rank < 0 || rank >= world) return fail(c, SPH_ERR_ARG, "bad rank/world");
   if (c->key_sorted != c->keyA) return fail(c, SPH_ERR_STATE, "sph_decomp_owners needs sph_compute_keys");
-  return cuda_check(c, launch_decomp_owners(c->n, c->keyA, hist, bits, rank, world, c->ds->splits, mig_mask, counts,
-                                            c->st), "decomp owners");
+  return cuda_check(c, launch_decomp_owners(c->n, c->keyA, c->ids[c->cur], hist, bits, rank, world, c->ds->splits,
+                                            mig_mask, counts, c->st), "decomp owners");
 }
 
 int sph_decomp_ghosts(sph_ctx* c, int bits, int rank, int world, uint64_t* mask, int64_t* counts) {
@@ -1124,17 +1124,18 @@ int sph_decomp_drop(sph_ctx* c, const uint64_t* drop_mask, int64_t n_expected) {
   int rc = check_ready(c, S_PART, "sph_decomp_drop");
   if (rc) return rc;
   if (n_expected < 0 || n_expected > c->n) return fail(c, SPH_ERR_ARG, "n_expected out of range");
+  c->stage = S_PART;
+  if (n_expected == c->n) return SPH_OK;  // the caller's counts say nothing goes
   const int nxt = c->cur ^ 1;
   int64_t* total = c->compact_scratch + (c->cfg.n_capacity + 1023) / 1024 + 1;
-  // drop_mask == NULL: drop the ghosts (SPH_GHOST_BIT) instead
-  rc = cuda_check(c, launch_compact(c->n, nullptr, drop_mask ? 0 : 1, c->state[c->cur], c->ids[c->cur], c->state[nxt],
+  // the ghosts (SPH_GHOST_BIT) and the particles with drop_mask[i] != 0 go
+  rc = cuda_check(c, launch_compact(c->n, nullptr, 1, c->state[c->cur], c->ids[c->cur], c->state[nxt],
                                     c->ids[nxt], c->compact_scratch, total, c->st, drop_mask), "decomp drop");
   if (rc) return rc;
   check_count_kernel<<<1, 1, 0, c->st>>>(total, n_expected, c->ds);
   note_launch();
   c->cur = nxt;
   c->n = n_expected;  // the caller's count (known from the routed counts): no sync
-  c->stage = S_PART;
   return cuda_check(c, cudaGetLastError(), "check count");
 }
 

@@ -301,12 +301,16 @@ cudaError_t launch_decomp_reduce(int64_t n, double* const* f, const int64_t* id,
 }
 
 // ---- histogram of the top `bits` key bits
+// (the keys are nearly sorted, so a warp's particles share one or two bins:
+// one atomic per distinct bin per warp)
 __global__ void __launch_bounds__(256) key_hist_kernel(int64_t n, const uint64_t* __restrict__ key,
                                                        const int64_t* __restrict__ id, int bits,
                                                        unsigned long long* hist) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (i >= n || (id[i] & SPH_GHOST_BIT)) return;
-  atomicAdd(hist + (key[i] >> (63 - bits)), 1ull);
+  const bool live = i < n && !(id[i] & SPH_GHOST_BIT);
+  const unsigned long long b = live ? (key[i] >> (63 - bits)) : ~0ull;
+  const uint32_t peers = __match_any_sync(0xffffffffu, b);
+  if (live && (peers & ((1u << (threadIdx.x & 31)) - 1u)) == 0) atomicAdd(hist + b, (unsigned long long)__popc(peers));
 }
 
 cudaError_t launch_key_histogram(int64_t n, const uint64_t* key, const int64_t* id, int bits, int64_t* hist,
@@ -369,29 +373,38 @@ __device__ __forceinline__ int owner_of_bin(const int32_t* s, int world, int bin
   return lo;
 }
 
-__global__ void __launch_bounds__(256) owners_kernel(int64_t n, const uint64_t* __restrict__ key, int bits,
+__global__ void __launch_bounds__(256) owners_kernel(int64_t n, const uint64_t* __restrict__ key,
+                                                     const int64_t* __restrict__ id, int bits,
                                                      int rank, int world, const int32_t* __restrict__ splits,
                                                      uint64_t* __restrict__ mig_mask,
                                                      unsigned long long* __restrict__ counts) {
   __shared__ int32_t s[kMaxGhostRanks + 1];
+  __shared__ unsigned long long bc[kMaxGhostRanks];  // this block's count per owner
   if (threadIdx.x <= world) s[threadIdx.x] = splits[threadIdx.x];
+  if (threadIdx.x < world) bc[threadIdx.x] = 0ull;
   __syncthreads();
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (i >= n) return;
-  const int o = owner_of_bin(s, world, (int)(key[i] >> (63 - bits)));
-  mig_mask[i] = o == rank ? 0ull : (1ull << o);
-  atomicAdd(counts + o, 1ull);
+  // last step's ghosts are neither owned nor sent (sph_decomp_drop removes them)
+  const bool live = i < n && !(id[i] & SPH_GHOST_BIT);
+  const int o = live ? owner_of_bin(s, world, (int)(key[i] >> (63 - bits))) : -1;
+  if (i < n) mig_mask[i] = (!live || o == rank) ? 0ull : (1ull << o);
+  // one shared-memory add per distinct owner per warp, one global add per
+  // owner per block (an owner holds long runs of the sorted keys)
+  const uint32_t peers = __match_any_sync(0xffffffffu, o);
+  if (live && (peers & ((1u << (threadIdx.x & 31)) - 1u)) == 0) atomicAdd(bc + o, (unsigned long long)__popc(peers));
+  __syncthreads();
+  if (threadIdx.x < world && bc[threadIdx.x]) atomicAdd(counts + threadIdx.x, bc[threadIdx.x]);
 }
 
-cudaError_t launch_decomp_owners(int64_t n, const uint64_t* key, const int64_t* hist, int bits, int rank,
-                                 int world, int32_t* splits, uint64_t* mig_mask, int64_t* counts,
+cudaError_t launch_decomp_owners(int64_t n, const uint64_t* key, const int64_t* id, const int64_t* hist, int bits,
+                                 int rank, int world, int32_t* splits, uint64_t* mig_mask, int64_t* counts,
                                  cudaStream_t st) {
   splits_kernel<<<1, 1024, 0, st>>>(hist, bits, world, splits);
   note_launch();
   cudaError_t e = cudaMemsetAsync(counts, 0, sizeof(int64_t) * world, st);
   if (e != cudaSuccess) return e;
   if (n > 0) {
-    owners_kernel<<<(unsigned)div_up(n, 256), 256, 0, st>>>(n, key, bits, rank, world, splits, mig_mask,
+    owners_kernel<<<(unsigned)div_up(n, 256), 256, 0, st>>>(n, key, id, bits, rank, world, splits, mig_mask,
                                                             (unsigned long long*)counts);
     note_launch();
   }
@@ -403,6 +416,9 @@ cudaError_t launch_decomp_owners(int64_t n, const uint64_t* key, const int64_t* 
 // 27 level-L cells around its own (periodic wrap, clipped at open faces).  A
 // particle within 2 h_max of a particle j lies in a cell adjacent to j's cell,
 // so j's owner receives it: the halo is conservative.
+__device__ uint64_t stencil_owners(uint64_t cell, int o, int bits, int world, const int32_t* s, int L,
+                                   const Params& P);
+
 __global__ void __launch_bounds__(256) ghost_route_kernel(int64_t n, const uint64_t* __restrict__ key, int bits,
                                                           int rank, int world, const int32_t* __restrict__ splits,
                                                           const DevScalars* __restrict__ ds, Params P,
@@ -410,6 +426,8 @@ __global__ void __launch_bounds__(256) ghost_route_kernel(int64_t n, const uint6
                                                           unsigned long long* __restrict__ counts) {
   __shared__ int32_t s[kMaxGhostRanks + 1];
   __shared__ int sL;
+  __shared__ unsigned long long bc[kMaxGhostRanks];
+  if (threadIdx.x < world) bc[threadIdx.x] = 0ull;
   if (threadIdx.x <= world) s[threadIdx.x] = splits[threadIdx.x];
   if (threadIdx.x == 0) {
     const double hmax = ds->key_box[6];
@@ -427,39 +445,59 @@ __global__ void __launch_bounds__(256) ghost_route_kernel(int64_t n, const uint6
   }
   __syncthreads();
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (i >= n) return;
+  const int lane = threadIdx.x & 31;
   const int L = sL;
+  // every particle of a level-L cell has the cell's mask: the warp computes it
+  // once per distinct cell (the held keys are nearly sorted: 1-2 cells per
+  // warp), one stencil cell per lane, OR-reduced
+  const uint64_t cell = i < n ? (key[i] >> (3 * (21 - L))) : ~0ull;
+  uint32_t todo = __ballot_sync(0xffffffffu, i < n);
+  uint64_t m = 0;
+  while (todo) {
+    const int lead = __ffs(todo) - 1;
+    const uint64_t c = __shfl_sync(0xffffffffu, cell, lead);
+    const uint64_t part = lane < 27 ? stencil_owners(c, lane, bits, world, s, L, P) : 0ull;
+    const uint32_t lo = __reduce_or_sync(0xffffffffu, (uint32_t)part);
+    const uint32_t hi = __reduce_or_sync(0xffffffffu, (uint32_t)(part >> 32));
+    const uint32_t mine = __ballot_sync(0xffffffffu, cell == c);
+    if (cell == c) m = (((uint64_t)hi << 32) | lo) & ~(1ull << rank);
+    todo &= ~mine;
+  }
+  if (i < n) mask[i] = m;
+  for (int r = 0; r < world; ++r) {  // one shared add per rank per warp, one global add per block
+    const uint32_t b = __ballot_sync(0xffffffffu, (m >> r) & 1ull);
+    if ((threadIdx.x & 31) == 0 && b) atomicAdd(bc + r, (unsigned long long)__popc(b));
+  }
+  __syncthreads();
+  if (threadIdx.x < world && bc[threadIdx.x]) atomicAdd(counts + threadIdx.x, bc[threadIdx.x]);
+}
+
+__device__ uint64_t stencil_owners(uint64_t cell, int o, int bits, int world, const int32_t* s, int L,
+                                   const Params& P) {
+  // the ranks owning a key of stencil cell o (0..26) around level-L cell `cell`
   const int lb = bits / 3;  // histogram bins are the level-lb cells
   const int nside = 1 << L;
-  const uint64_t k = key[i];
-  const int c[3] = {(int)(compact3(k >> 2) >> (21 - L)), (int)(compact3(k >> 1) >> (21 - L)),
-                    (int)(compact3(k) >> (21 - L))};
-  uint64_t m = 0;
-  for (int o = 0; o < 27; ++o) {
-    int u[3] = {c[0] + o / 9 - 1, c[1] + (o / 3) % 3 - 1, c[2] + o % 3 - 1};
-    bool ok = true;
+  const int c[3] = {(int)compact3(cell >> 2), (int)compact3(cell >> 1), (int)compact3(cell)};
+  int u[3] = {c[0] + o / 9 - 1, c[1] + (o / 3) % 3 - 1, c[2] + o % 3 - 1};
 #pragma unroll
-    for (int a = 0; a < 3; ++a) {
-      if (u[a] < 0 || u[a] >= nside) {
-        if (P.periodic[a]) u[a] = (u[a] + nside) & (nside - 1);
-        else ok = false;
-      }
+  for (int a = 0; a < 3; ++a) {
+    if (u[a] < 0 || u[a] >= nside) {
+      if (P.periodic[a]) u[a] = (u[a] + nside) & (nside - 1);
+      else return 0ull;  // clipped at an open face
     }
-    if (!ok) continue;
-    const uint64_t ck = morton3((uint32_t)u[0], (uint32_t)u[1], (uint32_t)u[2]);  // level-L cell key
-    int b0, b1;  // bins [b0, b1] covered by the cell
-    if (L >= lb) {
-      b0 = b1 = (int)(ck >> (3 * (L - lb)));
-    } else {
-      b0 = (int)(ck << (3 * (lb - L)));
-      b1 = (int)(((ck + 1) << (3 * (lb - L))) - 1);
-    }
-    const int r0 = owner_of_bin(s, world, b0), r1 = owner_of_bin(s, world, b1);
-    for (int r = r0; r <= r1; ++r) m |= 1ull << r;
   }
-  m &= ~(1ull << rank);
-  mask[i] = m;
-  for (uint64_t q = m; q; q &= q - 1) atomicAdd(counts + (__ffsll((long long)q) - 1), 1ull);
+  const uint64_t ck = morton3((uint32_t)u[0], (uint32_t)u[1], (uint32_t)u[2]);  // level-L cell key
+  int b0, b1;  // bins [b0, b1] covered by the cell
+  if (L >= lb) {
+    b0 = b1 = (int)(ck >> (3 * (L - lb)));
+  } else {
+    b0 = (int)(ck << (3 * (lb - L)));
+    b1 = (int)(((ck + 1) << (3 * (lb - L))) - 1);
+  }
+  const int r0 = owner_of_bin(s, world, b0), r1 = owner_of_bin(s, world, b1);
+  uint64_t m = 0;
+  for (int r = r0; r <= r1; ++r) m |= 1ull << r;
+  return m;
 }
 
 cudaError_t launch_decomp_ghosts(int64_t n, const uint64_t* key, int bits, int rank, int world,

@@ -298,8 +298,8 @@ cudaError_t launch_decomp_reduce(int64_t n, double* const* f, const int64_t* id,
                                  double* red, cudaStream_t st);
 cudaError_t launch_key_histogram(int64_t n, const uint64_t* key, const int64_t* id, int bits, int64_t* hist,
                                  cudaStream_t st);
-cudaError_t launch_decomp_owners(int64_t n, const uint64_t* key, const int64_t* hist, int bits, int rank,
-                                 int world, int32_t* splits, uint64_t* mig_mask, int64_t* counts,
+cudaError_t launch_decomp_owners(int64_t n, const uint64_t* key, const int64_t* id, const int64_t* hist, int bits,
+                                 int rank, int world, int32_t* splits, uint64_t* mig_mask, int64_t* counts,
                                  cudaStream_t st);
 cudaError_t launch_decomp_ghosts(int64_t n, const uint64_t* key, int bits, int rank, int world,
                                  const int32_t* splits, const DevScalars* ds, const Params& P, uint64_t* mask,

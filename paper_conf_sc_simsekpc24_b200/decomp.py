@@ -7,7 +7,8 @@ curve.  Each step (every selection, count, split, pack and map is a libsph
 device call, include/sph.h "SFC decomposition on the device"; this module only
 issues the collectives between them):
 
-  1. drop last step's ghosts (the local count is known: no sync);
+  1. last step's ghosts stay until the migration's compaction (skipped by
+     every reduction);
   2. global box and h_max: MAX all-reduce of 7 doubles (exact), set as the key
      box of the open axes -- every rank's keys are the single-GPU run's;
   3. SFC partition: key histogram (2^15 bins of the top key bits), SUM
@@ -219,10 +220,9 @@ class DistributedSim:
         dev = self.dev
         self._mark(None)
         if xchg:
-            # 1. last step's ghosts out: the local count is known, no sync
-            if self.has_ghosts:
-                sim.decomp_drop(None, self.n_local)
-            # 2. global box and h_max (exact MAX), the key box of the open axes
+            # 1.-2. (last step's ghosts are skipped by the reduction, the histogram
+            # and the owners, and dropped with the emigrants in one compaction)
+            # global box and h_max (exact MAX), the key box of the open axes
             red = sim.decomp_reduce()
             comm.all_reduce_(red, dist.ReduceOp.MAX)
             sim.set_key_box(red)

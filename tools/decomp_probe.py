@@ -1,6 +1,8 @@
 """Probe: cost of the decomposed step (decomp.py) at world = 1 against the plain
 sph_step on the same workload, with a synchronising section timer."""
+import os
 import sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import time
 
 import numpy as np
