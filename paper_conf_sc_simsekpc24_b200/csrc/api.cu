@@ -41,6 +41,9 @@ int level_cap_for(const sph_config* c) {
   return std::max(L, 0);
 }
 
+constexpr int kSortSkipDefault = 4;  // LSD passes over digits 4..7 (the top 31 key bits)
+constexpr unsigned long long kSortMaxRun = 64;
+
 struct PhaseRow {
   int64_t calls = 0;
   double seconds = 0, joules = 0, mhz_sum = 0;
@@ -116,6 +119,10 @@ struct sph_ctx {
   uint32_t* perm_saved = nullptr; // its copy while sph_repeat_phase(SORT) reuses the buffers;
                                   // also the inverse permutation of sph_decomp_map
   bool inv_valid = false;         // perm_saved holds the inverse of last_perm
+  // SORT: radix passes over digits sort_skip..7 + the run fixup (k_sort.cu);
+  // all 8 passes (skip 0) after a step whose fixup met a long run
+  int sort_skip = kSortSkipDefault;
+  int sort_full_steps = 0;
   int64_t* compact_scratch = nullptr;  // per-block counts of sph_compact / sph_decomp_pack (+ totals)
   int64_t compact_scratch_len = 0;
   Stir stir{};          // turbulence driving (k_stir.cu)
@@ -346,6 +353,14 @@ int sync_scalars(sph_ctx* c) {
   rc = cuda_check(c, cudaStreamSynchronize(c->st), "stream sync");
   if (rc) return rc;
   collect_all(c);
+  // sort policy for the next steps: long fixup runs (particles closer than a
+  // level-(21 - 8 skip / 3) cell) -> all 8 passes for a while
+  if (c->h_ds.sort_maxrun > kSortMaxRun) {
+    c->sort_skip = 0;
+    c->sort_full_steps = 16;
+  } else if (c->sort_full_steps > 0 && --c->sort_full_steps == 0) {
+    c->sort_skip = kSortSkipDefault;
+  }
   int s = c->h_ds.status;
   if (s & ST_BOX) return fail(c, SPH_ERR_BOX, "degenerate open-axis box (max == min)");
   if (s & ST_CAPACITY)
@@ -402,7 +417,7 @@ int body_tree(sph_ctx* c) {
   uint32_t* perm = nullptr;
   uint64_t* ksorted = nullptr;
   cudaError_t e = launch_sort(F, c->keyA, c->keyB, c->valA, c->valB, c->sort_hist, c->sort_status,
-                              c->status_bytes, &perm, &ksorted, c->st);
+                              c->status_bytes, &perm, &ksorted, c->st, c->sort_skip);
   if ((rc = cuda_check(c, e, "sort"))) return rc;
   c->last_perm = perm;
   c->inv_valid = false;
@@ -1553,7 +1568,7 @@ int sph_repeat_phase(sph_ctx* c, int phase, int reps, double* ms_per_call, doubl
         uint32_t* perm = nullptr;
         uint64_t* ks = nullptr;
         launch_sort(F, c->key_sorted, spare_keys, c->valA, c->valB, c->sort_hist, c->sort_status,
-                    c->status_bytes, &perm, &ks, c->st);
+                    c->status_bytes, &perm, &ks, c->st, c->sort_skip);
         c->cur = prv ^ 1;
         Fields Fd = fields(c);
         c->cur = prv;

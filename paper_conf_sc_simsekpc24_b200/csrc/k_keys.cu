@@ -16,6 +16,7 @@ __global__ void reset_scalars_kernel(DevScalars* ds) {
   }
   ds->hmax_ord = 0ull;
   ds->minhc_ord = ~0ull;
+  ds->sort_maxrun = 0ull;
   ds->status = 0;
   ds->max_nc = 0;
   ds->min_nc = 0x7fffffff;

@@ -91,6 +91,38 @@ void launch_cells(const Fields& F, const Params& P, int level_cap, cudaStream_t 
   }
 }
 
+// L2 residency of the scratch rows (SPH_NBR_EVICT): the column-major list
+// stores stream 3.2 GB through L2 with evict_first priority, the rows are
+// written and read back with evict_last, so the rows are not evicted (and
+// written to DRAM and read back) between the appends and the copy-out.
+#ifndef SPH_NBR_EVICT
+#define SPH_NBR_EVICT 1
+#endif
+struct L2Pol {
+  uint64_t first, last;
+};
+__device__ __forceinline__ L2Pol make_l2pol() {
+  L2Pol p{0, 0};
+  if (SPH_NBR_EVICT) {
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p.first));
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p.last));
+  }
+  return p;
+}
+__device__ __forceinline__ void st_hint(int32_t* a, int32_t v, uint64_t pol) {
+  if (SPH_NBR_EVICT) asm volatile("st.global.L2::cache_hint.b32 [%0], %1, %2;" ::"l"(a), "r"(v), "l"(pol) : "memory");
+  else *a = v;
+}
+__device__ __forceinline__ void ld8i_hint(const int32_t* p, int (&v)[8], uint64_t pol) {
+  if (SPH_NBR_EVICT)
+    asm volatile("ld.global.L2::cache_hint.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+                 : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+                 : "l"(p), "l"(pol)
+                 : "memory");
+  else
+    ld8i(p, v);
+}
+
 constexpr int kNbrThreads = 128;
 constexpr int kNbrWarps = kNbrThreads / 32;
 constexpr int kMaxWarpCells = 128;
@@ -339,7 +371,7 @@ __device__ __forceinline__ GroupBox build_cells(const Box& B, const int (&cc)[3]
 template <bool kFull>
 __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const Target& t, int64_t i,
                                           const GroupBox& G, WarpSmem& S, int lane, int& cnt,
-                                          int32_t* __restrict__ rows) {
+                                          int32_t* __restrict__ rows, const L2Pol& pol) {
   const int n = B.nside;
   const int T = G.T;
   const int ngmax = F.ngmax;
@@ -549,8 +581,8 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
         const int32_t v0 = (int32_t)S.cj[b0], v1 = (int32_t)S.cj[b1];
         // branch-free: past the capacity (or for a missing second hit) the
         // store goes to the row's spare word ngmax (nrows_ld > ngmax), never read
-        myrow[min(slot, ngmax)] = v0;
-        myrow[two ? min(slot + 1, ngmax) : ngmax] = v1;
+        st_hint(myrow + min(slot, ngmax), v0, pol.last);
+        st_hint(myrow + (two ? min(slot + 1, ngmax) : ngmax), v1, pol.last);
         slot += two ? 2 : 1;
       }
     }
@@ -575,6 +607,7 @@ __global__ void __launch_bounds__(kNbrThreads, 6) neighbors_kernel(Fields F, Par
     B.side[a] = (float)(B.L[a] / B.nside);
     B.per[a] = P.periodic[a] != 0;
   }
+  const L2Pol pol = make_l2pol();
   // this warp's 32 scratch rows (row of lane l: rows + l * nrows_ld)
   int32_t* const rows = F.nrows + ((int64_t)blockIdx.x * kNbrThreads + warp * 32) * F.nrows_ld;
   // warps take 32-target tiles dynamically, in order (Morton-adjacent tiles run
@@ -624,9 +657,9 @@ __global__ void __launch_bounds__(kNbrThreads, 6) neighbors_kernel(Fields F, Par
       Target tg = t;
       if (lane / g != gid) tg.r_out2 = tg.r_in2 = tg.rc = -1.f;  // not in this pass
       if (G.full[0] || G.full[1] || G.full[2])
-        warp_walk<true>(F, B, tg, i, G, s_w[warp], lane, cnt, rows);
+        warp_walk<true>(F, B, tg, i, G, s_w[warp], lane, cnt, rows, pol);
       else
-        warp_walk<false>(F, B, tg, i, G, s_w[warp], lane, cnt, rows);
+        warp_walk<false>(F, B, tg, i, G, s_w[warp], lane, cnt, rows, pol);
       __syncwarp();
     }
     if (active) F.nc[i] = cnt;
@@ -639,10 +672,10 @@ __global__ void __launch_bounds__(kNbrThreads, 6) neighbors_kernel(Fields F, Par
     int32_t* col = F.nbr + i;
     for (int k0 = 0; k0 < wlen; k0 += 8) {
       int v[8];
-      if (k0 < len) ld8i(myrow + k0, v);
+      if (k0 < len) ld8i_hint(myrow + k0, v, pol.last);
 #pragma unroll
       for (int u = 0; u < 8; ++u)
-        if (k0 + u < len) col[(int64_t)(k0 + u) * F.cap] = v[u];
+        if (k0 + u < len) st_hint(col + (int64_t)(k0 + u) * F.cap, v[u], pol.first);
     }
     __syncwarp();  // the rows are reused by the next tile
 

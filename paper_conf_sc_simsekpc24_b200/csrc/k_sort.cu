@@ -235,9 +235,43 @@ void sort_workspace(int64_t cap, size_t* hist_bytes, size_t* status_bytes) {
 // Sorts F.n keys from key_in.  Returns the sorted keys and the permutation
 // (perm[k] = input index of the k-th smallest) in *key_out / *perm_out, which
 // point into the ping-pong buffers.
+// Runs of keys equal in the sorted digits: after LSD passes over the digits
+// skip..7 only, the order is sorted by key >> 8 skip, and equal prefixes keep
+// the input order (stable passes).  Sorting every such run by the full key with
+// a stable insertion sort then gives exactly the stable sort by the full key
+// (ties keep the input order).  The keys arrive from last step's order with
+// particles far apart compared with a level-10 cell, so the runs are almost all
+// of length 1: the fixup is one read of the keys.  The longest run is recorded
+// (DevScalars::sort_maxrun) and the host falls back to all 8 passes when runs
+// grow long (launch_sort's `skip`, api.cu).
+__global__ void __launch_bounds__(256) sort_fixup_kernel(uint64_t* __restrict__ key, uint32_t* __restrict__ val,
+                                                         int64_t n, int shift, DevScalars* ds) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const uint64_t h = key[i] >> shift;
+  if (i > 0 && (key[i - 1] >> shift) == h) return;           // not the first of its run
+  if (i + 1 >= n || (key[i + 1] >> shift) != h) return;      // run of one: nothing to do
+  int64_t e = i + 2;
+  while (e < n && (key[e] >> shift) == h) ++e;
+  for (int64_t a = i + 1; a < e; ++a) {  // stable insertion sort of [i, e) by the full key
+    const uint64_t k = key[a];
+    const uint32_t v = val[a];
+    int64_t b = a - 1;
+    while (b >= i && key[b] > k) {
+      key[b + 1] = key[b];
+      val[b + 1] = val[b];
+      --b;
+    }
+    key[b + 1] = k;
+    val[b + 1] = v;
+  }
+  const unsigned long long len = (unsigned long long)(e - i);
+  atomicMax(&ds->sort_maxrun, len);
+}
+
 cudaError_t launch_sort(const Fields& F, uint64_t* key_in, uint64_t* key_tmp, uint32_t* val_a,
                         uint32_t* val_b, uint32_t* hist, uint32_t* status, size_t status_bytes,
-                        uint32_t** perm_out, uint64_t** key_out, cudaStream_t st) {
+                        uint32_t** perm_out, uint64_t** key_out, cudaStream_t st, int skip) {
   const int64_t n = F.n;
   *perm_out = val_a;
   *key_out = key_in;
@@ -265,9 +299,10 @@ cudaError_t launch_sort(const Fields& F, uint64_t* key_in, uint64_t* key_tmp, ui
   uint64_t* ks[2] = {key_in, key_tmp};
   uint32_t* vs[2] = {val_a, val_b};
   int cur = 0;
-  for (int p = 0; p < kSortPasses; ++p) {
+  skip = std::max(0, std::min(skip, kSortPasses - 1));
+  for (int p = skip; p < kSortPasses; ++p) {
     uint32_t* stp = status + (size_t)p * tiles * kRadix;
-    if (p == 0)
+    if (p == skip)
       onesweep_kernel<true><<<(unsigned)tiles, kSortThreads, smem, st>>>(
           ks[cur], nullptr, ks[cur ^ 1], vs[cur ^ 1], n, p * kRadixBits, hist + p * kRadix, stp,
           tile_ctr + p);
@@ -280,6 +315,10 @@ cudaError_t launch_sort(const Fields& F, uint64_t* key_in, uint64_t* key_tmp, ui
   }
   *key_out = ks[cur];
   *perm_out = vs[cur];
+  if (skip > 0) {
+    sort_fixup_kernel<<<(unsigned)div_up(n, 256), 256, 0, st>>>(ks[cur], vs[cur], n, skip * kRadixBits, F.ds);
+    note_launch();
+  }
   return cudaGetLastError();
 }
 

@@ -55,6 +55,7 @@ struct DevScalars {
   double key_box[7];              // -min x, -min y, -min z, max x, max y, max z, max h
   unsigned long long red_ord[7];
   int32_t splits[65];
+  unsigned long long sort_maxrun;  // longest run of the sort's fixup (k_sort.cu)
 };
 
 // Self-gravity (k_gravity.cu).
@@ -277,7 +278,7 @@ void launch_box_keys(const Fields& F, const Params& P, cudaStream_t st);
 void sort_workspace(int64_t cap, size_t* hist_bytes, size_t* status_bytes);
 cudaError_t launch_sort(const Fields& F, uint64_t* key_in, uint64_t* key_tmp, uint32_t* val_a,
                         uint32_t* val_b, uint32_t* hist, uint32_t* status, size_t status_bytes,
-                        uint32_t** perm_out, uint64_t** key_out, cudaStream_t st);
+                        uint32_t** perm_out, uint64_t** key_out, cudaStream_t st, int skip = 0);
 void launch_permute(const Fields& Fdst, const uint32_t* perm, double* const* src,
                     const int64_t* id_src, cudaStream_t st);
 void launch_cells(const Fields& F, const Params& P, int level_cap, cudaStream_t st);

@@ -186,3 +186,34 @@ def test_host_and_device_inputs_agree():
     b.step()
     for k in ("x", "vx", "u", "h"):
         assert np.array_equal(a.get_field(k), b.get_field(k))
+
+
+@pytest.mark.parametrize("spread", [1e-4, 3e-3])
+def test_sort_fixup_and_fallback_bit_exact(spread):
+    """The production sort runs the LSD passes over the top key digits only and
+    then stable-sorts the runs of equal top digits by the full key (k_sort.cu).
+    Clustered particles (all within `spread` of a point, with exact duplicate
+    positions: ties keep the input order) make long runs: the fixup's result,
+    and the all-8-pass fallback the next build takes after a long run, both equal
+    the oracle's stable sort bit for bit."""
+    from paper_conf_sc_simsekpc24_b200 import sph
+    w = ics.random_box(6000, seed=17, periodic=True)
+    rng = np.random.default_rng(5)
+    for k in ("x", "y", "z"):
+        w.state[k] = 0.1 + rng.uniform(0, spread, w.n)
+    dup = np.arange(0, w.n - 1, 7)
+    for k in ("x", "y", "z"):
+        w.state[k][dup] = w.state[k][dup + 1]   # exact duplicate positions: equal keys
+    w.state["h"][:] = 1e-5
+    sim = sph.Simulation(w.params, n_capacity=w.n)
+    s = {k: np.ascontiguousarray(v) for k, v in w.state.items()}
+    sim.set_particles(s)
+    sim.set_time(0.0, w.params.dt_first, True)
+    bmin, bmax = oracle.box(s["x"], s["y"], s["z"], w.params)
+    want = s["id"][oracle.sort_order(oracle.keys(s["x"], s["y"], s["z"], bmin, bmax))]
+    for rep in range(3):   # fixup, then (after the long runs) the full-pass fallback
+        sim.build_tree()
+        assert np.array_equal(sim.get_field("id"), want), rep
+        sim.find_neighbors()  # its scalar sync updates the sort policy
+        sim.set_particles(s)  # same input again
+    sim.finalize()
