@@ -57,7 +57,7 @@ MOM_BYTES_PER_PARTICLE = 19 * 8 + 4 + 4 * 8   # + 4 * nc
 # entry), FP64 flops per pair, and the roofline that binds the phase.
 PHASE_COST = {
     "keys": (40, 0, 0, "hbm"),
-    "sort": (196 + 224, 0, 0, "hbm"),          # 8 radix passes + the permutation
+    "sort": (8 + 92 + 8 + 224, 0, 0, "hbm"),   # histogram, 4 radix passes (top digits), run fixup, permutation
     "cells": (8, 0, 0, "hbm"),
     "neighbors": (52, 4, 0, "issue"),          # pos4/x/y/z/h in, nc out, list out
     "density": (48, 4, FLOPS_PER_PAIR["density"], "fp64"),
