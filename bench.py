@@ -170,55 +170,85 @@ def make_workload(name: str, rank: int):
 
 
 class ClockSampler:
-    """nvidia-smi clocks/throttle reasons sampled every 100 ms during the timed region."""
+    """SM clock, power and clock-event (throttle) reasons sampled every ~10 ms by
+    an NVML thread during the timed region (nvidia-smi -lms 100 as fallback)."""
 
-    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
-         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-         "clocks_event_reasons.sw_power_cap")
+    REASONS = {0x4: "sw_power_cap", 0x8: "hw_slowdown", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown"}
 
-    def __init__(self, gpu_index: int):
+    def __init__(self, gpu_index: int, period_s: float = 0.01):
         self.gpu = gpu_index
+        self.period = period_s
+        self.samples = []
         self.p = None
+        self.th = None
+
+    def _nvml_loop(self, N, h):
+        import time as _t
+        while not self.stop:
+            try:
+                sm = N.nvmlDeviceGetClockInfo(h, N.NVML_CLOCK_SM)
+                mx = N.nvmlDeviceGetMaxClockInfo(h, N.NVML_CLOCK_SM)
+                pw = N.nvmlDeviceGetPowerUsage(h) / 1e3
+                try:
+                    rs = N.nvmlDeviceGetCurrentClocksEventReasons(h)
+                except AttributeError:
+                    rs = N.nvmlDeviceGetCurrentClocksThrottleReasons(h)
+                self.samples.append((sm, mx, pw, rs))
+            except Exception:
+                pass
+            _t.sleep(self.period)
 
     def __enter__(self):
+        self.stop = False
         try:
-            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
-                                       "--format=csv,noheader,nounits", "-lms", "100"],
-                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-        except OSError:
-            self.p = None
-        time.sleep(0.3)
+            import threading
+            import pynvml as N
+            N.nvmlInit()
+            h = N.nvmlDeviceGetHandleByIndex(self.gpu)
+            self.th = threading.Thread(target=self._nvml_loop, args=(N, h), daemon=True)
+            self.th.start()
+        except Exception:
+            self.th = None
+            try:
+                self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), "--query-gpu=clocks.sm,clocks.max.sm,"
+                                           "power.draw,clocks_event_reasons.active", "--format=csv,noheader,nounits",
+                                           "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            except OSError:
+                self.p = None
+        time.sleep(0.05)
         return self
 
     def __exit__(self, *a):
-        self.lines = []
+        self.stop = True
+        if self.th:
+            self.th.join(timeout=2)
         if self.p:
             time.sleep(0.25)
             self.p.terminate()
             out, _ = self.p.communicate(timeout=10)
-            self.lines = [l for l in out.splitlines() if l.strip()]
+            for l in out.splitlines():
+                f = [x.strip() for x in l.split(",")]
+                try:
+                    self.samples.append((float(f[0]), float(f[1]), float(f[2]), int(f[3], 16)))
+                except (ValueError, IndexError):
+                    pass
 
     def summary(self):
-        sm, mx, pw = [], [], []
-        reasons = set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for l in getattr(self, "lines", []):
-            f = [x.strip() for x in l.split(",")]
-            if len(f) < 7:
-                continue
-            try:
-                sm.append(float(f[0]))
-                mx.append(float(f[1]))
-                pw.append(float(f[2]))
-            except ValueError:
-                continue
-            for k, v in zip(names, f[3:7]):
-                if v.lower().startswith("active"):
-                    reasons.add(k)
-        if not sm:
+        if not self.samples:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
-        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx), "reasons": sorted(reasons),
-                "power_w_median": statistics.median(pw), "samples": len(sm)}
+        reasons = set()
+        counts = {}
+        for _, _, _, rs in self.samples:
+            for bit, name in self.REASONS.items():
+                if rs & bit:
+                    reasons.add(name)
+                    counts[name] = counts.get(name, 0) + 1
+        return {"sm_mhz": statistics.median(x[0] for x in self.samples),
+                "sm_max_mhz": max(x[1] for x in self.samples), "reasons": sorted(reasons),
+                "reason_samples": counts,
+                "power_w_median": statistics.median(x[2] for x in self.samples), "samples": len(self.samples),
+                "source": "NVML thread, ~10 ms period" if self.th else "nvidia-smi -lms 100"}
 
 
 def cpu_baseline(w, n_targets: int, seed: int = 3):

@@ -8,6 +8,6 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
   --log-file gpurun_out/${TAG}_launches.csv python bench.py $ARGS > gpurun_out/${TAG}_ncu_launch_bench.log 2>&1
 echo "launch list rc=$?"
 timeout 1500 ncu --set full --clock-control none --import-source on \
-  -k regex:"neighbors_kernel|momentum_energy_kernel|density_kernel|iad_kernel|onesweep|permute" -s 12 -c 12 \
+  -k regex:"neighbors_kernel|momentum_energy_kernel|density_kernel|iad_kernel|onesweep|permute|sort_fixup|update_kernel|eos_kernel" -s 12 -c 12 \
   -o gpurun_out/${TAG}_full python bench.py $ARGS > gpurun_out/${TAG}_ncu_full.log 2>&1
 echo "full rc=$?"

@@ -17,7 +17,9 @@ METRICS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.
            "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum",
            "sm__sass_thread_inst_executed_op_dfma_pred_on.sum",
            "sm__sass_thread_inst_executed_op_dmul_pred_on.sum",
-           "sm__sass_thread_inst_executed_op_dadd_pred_on.sum"]
+           "sm__sass_thread_inst_executed_op_dadd_pred_on.sum",
+           "l1tex__data_pipe_lsu_wavefronts.avg.pct_of_peak_sustained_elapsed",
+           "smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio"]
 
 
 def full(rep):
