@@ -67,7 +67,13 @@ typedef enum sph_status {
 } sph_status;
 
 typedef enum sph_eos_kind { SPH_EOS_IDEAL = 0, SPH_EOS_ISOTHERMAL = 1 } sph_eos_kind;
-typedef enum sph_mem_kind { SPH_MEM_HOST = 0, SPH_MEM_DEVICE = 1 } sph_mem_kind;
+typedef enum sph_mem_kind {
+  SPH_MEM_HOST = 0,       /* host memory; the call synchronises                      */
+  SPH_MEM_DEVICE = 1,     /* device memory; asynchronous on the context's stream     */
+  SPH_MEM_HOST_ASYNC = 2  /* sph_get_field only: asynchronous copy into (pinned) host
+                             memory, valid after sph_sync -- lets a caller overlap a
+                             step's read-back with other work                        */
+} sph_mem_kind;
 typedef enum sph_accounting_mode {
   SPH_ACCOUNTING_OFF = 0,   /* CUDA-event phase times only, no phase-edge syncs  */
   SPH_ACCOUNTING_PHASE = 1  /* + in-situ energy per phase ("from the start of
@@ -279,8 +285,12 @@ int sph_get_time(sph_ctx* ctx, double* t, double* dt_prev, int* first_step);
 int sph_get_n(const sph_ctx* ctx, int64_t* n);
 
 /* Copies field f (n values; int64 for SPH_F_ID, uint64 for SPH_F_KEY, int32 for
- * SPH_F_NC, double otherwise) to dst (host or device).  Synchronises. */
+ * SPH_F_NC, double otherwise) to dst (host or device).  Synchronises, except
+ * with SPH_MEM_HOST_ASYNC (valid after sph_sync). */
 int sph_get_field(sph_ctx* ctx, int field, void* dst, int mem);
+
+/* Waits for everything enqueued on the context's stream. */
+int sph_sync(sph_ctx* ctx);
 
 /* Multi-GPU halo support (SFC domain decomposition).  A particle
  * whose id has bit SPH_GHOST_BIT set is a ghost: a copy of a particle owned by

@@ -813,7 +813,8 @@ int sph_get_field(sph_ctx* c, int field, void* dst, int mem) {
   int rc = check_ready(c, S_INIT, "sph_get_field");
   if (rc) return rc;
   if (!dst && c->n > 0) return fail(c, SPH_ERR_ARG, "null dst");
-  if (mem != SPH_MEM_HOST && mem != SPH_MEM_DEVICE) return fail(c, SPH_ERR_ARG, "mem must be HOST or DEVICE");
+  if (mem != SPH_MEM_HOST && mem != SPH_MEM_DEVICE && mem != SPH_MEM_HOST_ASYNC)
+    return fail(c, SPH_ERR_ARG, "mem must be HOST, DEVICE or HOST_ASYNC");
   const void* src = nullptr;
   size_t esz = sizeof(double);
   if (field >= SPH_F_X && field <= SPH_F_DU_M1) src = c->state[c->cur][field - SPH_F_X];
@@ -850,8 +851,16 @@ int sph_get_field(sph_ctx* c, int field, void* dst, int mem) {
   }
   else return fail(c, SPH_ERR_ARG, "unknown field %d", field);
   if (c->n == 0) return SPH_OK;
-  const cudaMemcpyKind kind = mem == SPH_MEM_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
+  const cudaMemcpyKind kind = mem == SPH_MEM_DEVICE ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost;
   rc = cuda_check(c, cudaMemcpyAsync(dst, src, esz * c->n, kind, c->st), "field copy");
+  if (rc || mem == SPH_MEM_HOST_ASYNC) return rc;  // valid after sph_sync (pinned dst: overlaps)
+  rc = cuda_check(c, cudaStreamSynchronize(c->st), "sync");
+  if (!rc) collect_all(c);
+  return rc;
+}
+
+int sph_sync(sph_ctx* c) {
+  int rc = check_ready(c, S_INIT, "sph_sync");
   if (rc) return rc;
   rc = cuda_check(c, cudaStreamSynchronize(c->st), "sync");
   if (!rc) collect_all(c);

@@ -30,7 +30,7 @@ FIELDS = ("x", "y", "z", "vx", "vy", "vz", "h", "m", "u", "du_m1", "id", "key", 
 FIELD_ID = {name: k for k, name in enumerate(FIELDS)}
 FIELD_DTYPE = {"id": np.int64, "key": np.uint64, "nc": np.int32, "order": np.int32}
 ROW_DOUBLES = 11  # SPH_ROW_DOUBLES: x y z vx vy vz h m u du_m1 id(bits)
-MEM_HOST, MEM_DEVICE = 0, 1
+MEM_HOST, MEM_DEVICE, MEM_HOST_ASYNC = 0, 1, 2
 ACCOUNTING_OFF, ACCOUNTING_PHASE = 0, 1
 CLOCK_DEFAULT, CLOCK_STATIC, CLOCK_PER_PHASE = 0, 1, 2
 
@@ -106,7 +106,7 @@ EXPORTS = ("sph_config_default", "sph_workspace_size", "sph_init", "sph_finalize
            "sph_select_ghosts", "sph_gather_field", "sph_scatter_field",
            "sph_decomp_reduce", "sph_set_key_box", "sph_key_histogram", "sph_decomp_owners",
            "sph_decomp_ghosts", "sph_decomp_pack", "sph_decomp_drop", "sph_decomp_map",
-           "sph_halo_gather", "sph_halo_scatter", "sph_min_hc_dev", "sph_set_min_hc_dev")
+           "sph_halo_gather", "sph_halo_scatter", "sph_min_hc_dev", "sph_set_min_hc_dev", "sph_sync")
 GHOST_BIT = 1 << 62
 
 _lib = None
@@ -182,6 +182,7 @@ def load(build_if_missing: bool = True):
     L.sph_halo_scatter.argtypes = [P, V, I, V, I64, V]
     L.sph_min_hc_dev.argtypes = [P, V]
     L.sph_set_min_hc_dev.argtypes = [P, V]
+    L.sph_sync.argtypes = [P]
     L.sph_supported_clocks.argtypes = [P, V, I, C.POINTER(I)]
     L.sph_trace_start.argtypes = [P, D, I64]
     L.sph_trace_stop.argtypes = [P, V, I64, C.POINTER(I64)]
@@ -332,15 +333,22 @@ class Simulation:
         self._ok(self.L.sph_get_time(self.ctx, C.byref(t), C.byref(d), C.byref(f)))
         return t.value, d.value, bool(f.value)
 
-    def get_field(self, name: str, out=None):
+    def get_field(self, name: str, out=None, async_: bool = False):
+        """Field `name` (current order) into `out` (numpy / torch host or cuda).
+        async_: a pinned host `out` is filled asynchronously (valid after sync())."""
         dt = FIELD_DTYPE.get(name, np.float64)
         if out is None:
             out = np.empty(self.n, dtype=dt)
         p, mem = _ptr(out)
         if mem == MEM_DEVICE:  # the destination may be memory torch's stream still uses
             self.stream.wait_stream(self.torch.cuda.current_stream(self.device))
+        elif async_:
+            mem = MEM_HOST_ASYNC
         self._ok(self.L.sph_get_field(self.ctx, FIELD_ID[name], C.c_void_p(p), mem))
         return out
+
+    def sync(self):
+        self._ok(self.L.sph_sync(self.ctx))
 
     def set_field(self, name: str, src):
         """Overwrite RHO or C11..C33 (n values, current order) -- multi-GPU halo."""
