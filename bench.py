@@ -251,7 +251,7 @@ class ClockSampler:
                 "source": "NVML thread, ~10 ms period" if self.th else "nvidia-smi -lms 100"}
 
 
-def cpu_baseline(w, n_targets: int, seed: int = 3):
+def cpu_baseline(w, n_targets: int, seed: int = 3, keep: dict | None = None, dt_override=None):
     """The oracle as it stands on a bounded sample: one step at n_targets random
     particles of the same workload (sampled mode: exact global sort/dt, each
     target's dependency ball brute-forced).  Returns (targets/s, seconds, threads)."""
@@ -260,10 +260,71 @@ def cpu_baseline(w, n_targets: int, seed: int = 3):
     rng = np.random.default_rng(seed)
     tg = np.sort(rng.choice(w.n, size=n_targets, replace=False))
     t0 = time.perf_counter()
-    oracle.sample_step({k: v for k, v in w.state.items()}, w.params, w.params.dt_first, True, tg)
+    res = oracle.sample_step({k: v for k, v in w.state.items()}, w.params, w.params.dt_first, True, tg,
+                             dt=dt_override) if dt_override is not None else \
+        oracle.sample_step({k: v for k, v in w.state.items()}, w.params, w.params.dt_first, True, tg)
     dt = time.perf_counter() - t0
     threads = int(os.environ.get("OMP_NUM_THREADS", os.cpu_count() or 1))
+    if keep is not None:
+        keep.update({"targets": tg, "order": res[0], "out": res[1]})
     return n_targets / dt, dt, threads
+
+
+def gpu_first_step(sim, w):
+    """The staged first step of the workload's initial state on `sim` (for the
+    per-run parity block); returns the GPU fields in the step's sorted order."""
+    import numpy as np
+    sim.set_particles({k: np.ascontiguousarray(v) for k, v in w.state.items()})
+    sim.set_time(0.0, w.params.dt_first, True)
+    sim.build_tree()
+    sim.find_neighbors(stats=False)
+    sim.density()
+    sim.eos()
+    if sim.cfg.gradh or sim.cfg.ve:
+        sim.gradh()
+    sim.iad()
+    sim.momentum_energy()
+    g = {k: sim.get_field(k) for k in ("id", "rho", "p", "c", "ax", "ay", "az", "du")}
+    g["C"] = np.stack([sim.get_field(k) for k in ("c11", "c12", "c13", "c22", "c23", "c33")], 1)
+    g["sim"] = sim
+    g["dt"] = sim.timestep()
+    return g
+
+
+def parity_block(sim, g, ref):
+    """SURVEY 8(d)'s per-run parity record: the bench workload's first step on
+    the GPU against the oracle's sampled mode at the cpu_baseline targets (the
+    same oracle run): Morton order of all particles, neighbour lists, dt, and
+    the largest error of each field in the DESIGN.md section 3 metric."""
+    import numpy as np
+    tg, o = ref["targets"], ref["out"]
+    off, idx = sim.get_neighbor_rows(tg)
+    nbr_exact = all(np.array_equal(idx[off[q]:off[q + 1]].astype(np.int64), o["nbrs"][q]) for q in range(len(tg)))
+    sim.update()
+    after = {k: sim.get_field(k) for k in ("x", "y", "z", "vx", "vy", "vz", "u", "h")}
+    err = {}
+
+    def rel(a, b, scale):
+        return float(np.max(np.abs(a - b) / np.maximum(scale, 1e-300)))
+    err["rho"] = rel(g["rho"][tg], o["rho"], np.abs(o["rho"]))
+    err["p"] = rel(g["p"][tg], o["p"], np.abs(o["p"]))
+    err["c"] = rel(g["c"][tg], o["c"], np.abs(o["c"]))
+    Cn = np.linalg.norm(o["C"], axis=1)
+    err["C"] = max(rel(g["C"][tg, e], o["C"][:, e], Cn) for e in range(6))
+    for a, k in enumerate(("ax", "ay", "az")):
+        err[k] = rel(g[k][tg], o[k], o["a_abs"][:, a])
+    err["du"] = rel(g["du"][tg], o["du"], o["du_abs"])
+    L = float(np.max(np.asarray(o["bmax"]) - np.asarray(o["bmin"])))
+    err["x"] = max(rel(after[k][tg], o[k], np.full(len(tg), L)) for k in ("x", "y", "z"))
+    vs = max(np.abs(np.concatenate([o["vx"], o["vy"], o["vz"]])).max(), 1e-300)
+    err["v"] = max(rel(after[k][tg], o[k], np.maximum(np.abs(o[k]), vs)) for k in ("vx", "vy", "vz"))
+    err["u"] = rel(after["u"][tg], o["u"], np.abs(o["u"]))
+    err["h"] = rel(after["h"][tg], o["h"], np.abs(o["h"]))
+    return {"targets": int(len(tg)), "order_exact": bool(np.array_equal(g["id"], ref["order"])),
+            "nbr_exact": bool(nbr_exact), "dt_exact": bool(g["dt"] == o["dt"]),
+            "max_err_by_field": err, "tolerance": 1e-10,
+            "pass": bool(nbr_exact and np.array_equal(g["id"], ref["order"]) and max(err.values()) <= 1e-10),
+            "what": "first step of the bench workload, GPU vs oracle.sample_step at the cpu_baseline targets"}
 
 
 def _cv(xs):
@@ -745,13 +806,23 @@ def main():
     trace = dvfs_trace(sim, sph, args.trace_seconds) if args.trace_seconds > 0 else None
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    parity = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and w.params.gravity:
+        cpu = {"unavailable": "gravity is long-range: the sampled oracle has no finite dependency ball",
+               "physics_only": cpu_physics_only(w)}
+    elif rank == 0 and world == 1 and not args.no_cpu_baseline:
         k = args.cpu_sample or 240  # ~10 s of oracle work on the host cores
-        v, sec, threads = cpu_baseline(w, k)
+        ref = {}
+        gfirst = gpu_first_step(sim, w)
+        v, sec, threads = cpu_baseline(w, k, keep=ref, dt_override=gfirst["dt"] if w.params.dt_vsig else None)
         phys = cpu_physics_only(w)
         cpu = {"value": v, "unit": UNIT, "cores": threads, "kind": "oracle",
                "sample": f"{k} random targets of {args.workload}, one step (oracle sampled mode), {sec:.1f} s",
                "physics_only": phys}
+        try:
+            parity = parity_block(sim, gfirst, ref)
+        except Exception as e:  # reported, never hidden
+            parity = {"error": repr(e)}
 
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -772,7 +843,7 @@ def main():
                            "search_passes_per_warp": infos[-1]["search_passes"] / (n / 32)},
                 "phase_ms": phase_ms, "fp64_other": other, "roofline": roofline, "e2e": e2e,
                 "phases": phase_table(phase_ms, pairs, n, energy, p_idle),
-                "repeats": repeats, "energy": energy, "accounting": accounting, "dvfs_trace": trace, "cpu_baseline": cpu, "clocks": clk.summary(),
+                "repeats": repeats, "parity": parity, "energy": energy, "accounting": accounting, "dvfs_trace": trace, "cpu_baseline": cpu, "clocks": clk.summary(),
                 "gpu_launches": launches}
         s = json.dumps(line)
         print(s, flush=True)

@@ -49,3 +49,5 @@ def test_libsph_arm_line():
     assert e["available"] and e["step"]["J_median"] > 0 and e["phases"]["momentum_energy"]["J"] > 0
     assert d["cpu_baseline"]["physics_only"]["s_per_particle"] > 0
     assert d["roofline"]["flops_per_pair"] == 171
+    assert d["parity"]["order_exact"] and d["parity"]["nbr_exact"] and d["parity"]["pass"], d["parity"]
+    assert d["e2e"]["sequential"]["value"] > 0
