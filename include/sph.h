@@ -406,6 +406,18 @@ int sph_halo_scatter(sph_ctx* ctx, const int32_t* fields, int nf, const int64_t*
 int sph_min_hc_dev(sph_ctx* ctx, double* dst);
 int sph_set_min_hc_dev(sph_ctx* ctx, const double* src);
 
+/* Split IAD / MOMENTUM_ENERGY for overlapping the halo exchanges with compute
+ * (SURVEY 8(e)): the neighbour search flags every target that has a ghost among
+ * its neighbours.  With part INTERIOR, sph_iad / sph_momentum_energy process
+ * only the targets without one (they need no halo value) and leave the stage
+ * unchanged; BOUNDARY processes the rest (and the ghosts' momentum records in
+ * IAD) and advances the stage; ALL (default) is the plain call.  GHOSTS makes
+ * sph_eos recompute only the ghosts (after their rho arrived).  Each target is
+ * computed once with the same inputs, so the results equal the unsplit step
+ * bit for bit.  Not with grad-h / volume elements (SPH_ERR_NOT_SUPPORTED). */
+enum { SPH_PART_ALL = 0, SPH_PART_INTERIOR = 1, SPH_PART_BOUNDARY = 2, SPH_PART_GHOSTS = 3 };
+int sph_set_part(sph_ctx* ctx, int part);
+
 /* --- the hot path (each call = one accounted phase group) ------------------- */
 
 /* Items 1-3: box (open axes: exact min/max), 63-bit Morton keys, stable LSD

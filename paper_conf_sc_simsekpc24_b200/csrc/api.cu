@@ -116,6 +116,7 @@ struct sph_ctx {
   bool locked_any = false;
   bool rec_m_dirty = false;
   uint32_t* last_perm = nullptr;  // the last sort's permutation (SPH_F_ORDER)
+  uint8_t* bnd = nullptr;         // per target: a ghost among its neighbours (search)
   uint32_t* perm_saved = nullptr; // its copy while sph_repeat_phase(SORT) reuses the buffers;
                                   // also the inverse permutation of sph_decomp_map
   bool inv_valid = false;         // perm_saved holds the inverse of last_perm
@@ -185,7 +186,7 @@ Fields fields(sph_ctx* c) {
   F.phi = c->phi; F.gcell_start = c->gcell_start; F.gmom = c->gmom;
   F.omega = c->omega; F.vsig = c->vsig;
   for (int a = 0; a < 3; ++a) F.curl[a] = c->curl[a];
-  F.nc = c->nc; F.nbr = c->nbr; F.ngmax = c->cfg.ngmax;
+  F.nc = c->nc; F.nbr = c->nbr; F.ngmax = c->cfg.ngmax; F.bnd = c->bnd;
   F.nrows = c->nrows; F.nrows_ld = nrows_ld(&c->cfg);
   F.cell_start = c->cell_start;
   F.pos4 = c->pos4;
@@ -465,7 +466,9 @@ int body_simple(sph_ctx* c, int phase, int next_stage) {
         launch_refresh_rec_m(F, c->st);
         c->rec_m_dirty = false;
       }
-      cudaMemsetAsync(&c->ds->minhc_ord, 0xff, sizeof(unsigned long long), c->st);
+      // (the BOUNDARY half of a split step adds to the INTERIOR half's minimum)
+      if (c->P.part != SPH_PART_BOUNDARY)
+        cudaMemsetAsync(&c->ds->minhc_ord, 0xff, sizeof(unsigned long long), c->st);
       launch_momentum_energy(F, c->P, c->st);
       break;
     case SPH_PHASE_TIMESTEP: launch_timestep(F, c->P, c->st); break;
@@ -619,6 +622,8 @@ static size_t layout(const sph_config* cfg, char* base, sph_ctx* c) {
     c->rec_m = (Rec4*)rm;
   }
   char* ncp = take(sizeof(int32_t) * cap);
+  char* bndp = take(sizeof(uint8_t) * cap);
+  if (c) c->bnd = (uint8_t*)bndp;
   char* nbp = take(sizeof(int32_t) * cap * (size_t)cfg->ngmax);
   char* nrp = take(sizeof(int32_t) * (size_t)kNbrSlots * kNbrSlotRows * (size_t)nrows_ld(cfg));
   const int Lc = level_cap_for(cfg);
@@ -700,6 +705,7 @@ int sph_init(const sph_config* cfg, void* arena, size_t arena_bytes, void* strea
   c->P.ve = cfg->ve ? 1 : 0;
   c->P.dt_vsig = cfg->dt_vsig ? 1 : 0;
   c->P.key_box_set = 0;
+  c->P.part = SPH_PART_ALL;
   layout(cfg, (char*)arena, c);
   for (int p = 0; p < SPH_NPHASES; ++p) {
     c->pending[p] = false;
@@ -1325,7 +1331,26 @@ int sph_density(sph_ctx* c) {
 
 int sph_eos(sph_ctx* c) {
   int rc = check_ready(c, S_DENS, "sph_eos");
-  return rc ? rc : body_simple(c, SPH_PHASE_EOS, S_EOS);
+  if (rc) return rc;
+  if (c->P.part == SPH_PART_GHOSTS) {  // the ghosts' EOS after their rho arrived: stage unchanged
+    if (c->stage < S_EOS) return fail(c, SPH_ERR_STATE, "sph_eos(GHOSTS) needs a full sph_eos first");
+    const int stage = c->stage;
+    const bool gd = c->gradh_done;
+    rc = body_simple(c, SPH_PHASE_EOS, stage);
+    c->gradh_done = gd;
+    return rc;
+  }
+  return body_simple(c, SPH_PHASE_EOS, S_EOS);
+}
+
+int sph_set_part(sph_ctx* c, int part) {
+  int rc = check_ready(c, S_INIT, "sph_set_part");
+  if (rc) return rc;
+  if (part < SPH_PART_ALL || part > SPH_PART_GHOSTS) return fail(c, SPH_ERR_ARG, "unknown part %d", part);
+  if (part != SPH_PART_ALL && (c->cfg.gradh || c->cfg.ve))
+    return fail(c, SPH_ERR_NOT_SUPPORTED, "split IAD / momentum with grad-h or volume elements");
+  c->P.part = part;
+  return SPH_OK;
 }
 
 int sph_gradh(sph_ctx* c) {
@@ -1340,12 +1365,16 @@ int sph_iad(sph_ctx* c) {
   if (rc) return rc;
   if ((c->cfg.gradh || c->cfg.ve) && !c->gradh_done)
     return fail(c, SPH_ERR_STATE, "cfg.gradh / cfg.ve: sph_gradh must run before sph_iad");
-  return body_simple(c, SPH_PHASE_IAD, S_IAD);
+  if (c->P.part == SPH_PART_GHOSTS) return fail(c, SPH_ERR_ARG, "part GHOSTS is for sph_eos");
+  // the INTERIOR half of a split IAD leaves the stage: the BOUNDARY half follows
+  return body_simple(c, SPH_PHASE_IAD, c->P.part == SPH_PART_INTERIOR ? S_EOS : S_IAD);
 }
 
 int sph_momentum_energy(sph_ctx* c) {
   int rc = check_ready(c, S_IAD, "sph_momentum_energy");
-  return rc ? rc : body_simple(c, SPH_PHASE_MOMENTUM_ENERGY, S_MOM);
+  if (rc) return rc;
+  if (c->P.part == SPH_PART_GHOSTS) return fail(c, SPH_ERR_ARG, "part GHOSTS is for sph_eos");
+  return body_simple(c, SPH_PHASE_MOMENTUM_ENERGY, c->P.part == SPH_PART_INTERIOR ? S_IAD : S_MOM);
 }
 
 int sph_timestep(sph_ctx* c, double* dt) {
@@ -1362,7 +1391,17 @@ int sph_update(sph_ctx* c) {
   return rc ? rc : body_simple(c, SPH_PHASE_UPDATE, S_PART);
 }
 
+static int sph_step_all(sph_ctx* c, sph_step_info* info);
 int sph_step(sph_ctx* c, sph_step_info* info) {
+  if (!c) return fail(nullptr, SPH_ERR_ARG, "sph_step: null context");
+  const int part = c->P.part;  // a whole step is never split
+  c->P.part = SPH_PART_ALL;
+  const int rc_step = sph_step_all(c, info);
+  c->P.part = part;
+  return rc_step;
+}
+
+static int sph_step_all(sph_ctx* c, sph_step_info* info) {
   int rc = check_ready(c, S_PART, "sph_step");
   if (rc) return rc;
   if ((rc = body_tree(c))) return rc;
@@ -1556,6 +1595,8 @@ int sph_repeat_phase(sph_ctx* c, int phase, int reps, double* ms_per_call, doubl
   bool eok = c->nvml.energy_mj(&e0);
   cudaEventRecord(a, c->st);
   Fields F = fields(c);
+  Params Pr = c->P;  // whole phases (not a split half)
+  Pr.part = SPH_PART_ALL;
   // KEYS writes into the key buffer not holding the sorted keys; SORT re-sorts
   // the (already sorted) keys in place and permutes into the spare state buffer
   // without switching to it: both leave the pipeline state unchanged.
@@ -1572,7 +1613,7 @@ int sph_repeat_phase(sph_ctx* c, int phase, int reps, double* ms_per_call, doubl
   const bool eos_omega = c->gradh_done && c->cfg.gradh;
   for (int r = 0; r < reps; ++r) {
     switch (phase) {
-      case SPH_PHASE_KEYS: launch_box_keys(Fk, c->P, c->st); break;
+      case SPH_PHASE_KEYS: launch_box_keys(Fk, Pr, c->st); break;
       case SPH_PHASE_SORT: {
         uint32_t* perm = nullptr;
         uint64_t* ks = nullptr;
@@ -1584,14 +1625,14 @@ int sph_repeat_phase(sph_ctx* c, int phase, int reps, double* ms_per_call, doubl
         launch_permute(Fd, perm, c->state[prv], c->ids[prv], c->st);
         break;
       }
-      case SPH_PHASE_CELLS: launch_cells(F, c->P, c->level_cap, c->st); break;
-      case SPH_PHASE_TIMESTEP: launch_timestep(F, c->P, c->st); break;
-      case SPH_PHASE_NEIGHBORS: launch_neighbors(F, c->P, c->st); break;
-      case SPH_PHASE_DENSITY: launch_density(F, c->P, c->st); break;
-      case SPH_PHASE_EOS: launch_eos(F, c->P, c->st, eos_omega); break;
-      case SPH_PHASE_IAD: launch_iad(F, c->P, c->st); break;
-      case SPH_PHASE_GRADH: launch_gradh(F, c->P, c->st); break;
-      case SPH_PHASE_MOMENTUM_ENERGY: launch_momentum_energy(F, c->P, c->st); break;
+      case SPH_PHASE_CELLS: launch_cells(F, Pr, c->level_cap, c->st); break;
+      case SPH_PHASE_TIMESTEP: launch_timestep(F, Pr, c->st); break;
+      case SPH_PHASE_NEIGHBORS: launch_neighbors(F, Pr, c->st); break;
+      case SPH_PHASE_DENSITY: launch_density(F, Pr, c->st); break;
+      case SPH_PHASE_EOS: launch_eos(F, Pr, c->st, eos_omega); break;
+      case SPH_PHASE_IAD: launch_iad(F, Pr, c->st); break;
+      case SPH_PHASE_GRADH: launch_gradh(F, Pr, c->st); break;
+      case SPH_PHASE_MOMENTUM_ENERGY: launch_momentum_energy(F, Pr, c->st); break;
     }
   }
   cudaEventRecord(b, c->st);

@@ -371,7 +371,7 @@ __device__ __forceinline__ GroupBox build_cells(const Box& B, const int (&cc)[3]
 template <bool kFull>
 __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const Target& t, int64_t i,
                                           const GroupBox& G, WarpSmem& S, int lane, int& cnt,
-                                          int32_t* __restrict__ rows, const L2Pol& pol) {
+                                          bool& bnd, int32_t* __restrict__ rows, const L2Pol& pol) {
   const int n = B.nside;
   const int T = G.T;
   const int ngmax = F.ngmax;
@@ -505,6 +505,7 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
   const int sg = 4 * (lane & 7) + (lane >> 3);
   const unsigned long long rin2x2 = pack2(t.r_in2, t.r_in2), rout2x2 = pack2(t.r_out2, t.r_out2);
   for (uint32_t c = 0; c < nchunks; ++c) {
+    const uint32_t gmask = __ballot_sync(0xffffffffu, q.w != 0.f);  // candidates that are ghosts
     S.cx[sg] = q.x + sx;
     S.cy[sg] = q.y + sy;
     S.cz[sg] = q.z + sz;
@@ -560,6 +561,7 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
     }
     // the target itself (d = 0) is not its own neighbour
     hin &= ~S.selfm[lane];
+    bnd = bnd || (hin & gmask) != 0u;
     // append: every lane writes its own hits, in candidate (= ascending index)
     // order, to its L2-resident row.  The warp runs the busiest lane's
     // iterations (~8-12 per chunk), but each is 5 instructions; a cooperative
@@ -633,6 +635,7 @@ __global__ void __launch_bounds__(kNbrThreads, 6) neighbors_kernel(Fields F, Par
       ckey = (uint32_t)(key >> (3 * sh));
     }
     int cnt = 0;
+    bool bnd = false;
 
     // group size: the whole warp unless it spans more than kMaxGroupCells distinct
     // coarse cells (Morton jumps); then halves, quarters, ...
@@ -657,13 +660,18 @@ __global__ void __launch_bounds__(kNbrThreads, 6) neighbors_kernel(Fields F, Par
       Target tg = t;
       if (lane / g != gid) tg.r_out2 = tg.r_in2 = tg.rc = -1.f;  // not in this pass
       if (G.full[0] || G.full[1] || G.full[2])
-        warp_walk<true>(F, B, tg, i, G, s_w[warp], lane, cnt, rows, pol);
+        warp_walk<true>(F, B, tg, i, G, s_w[warp], lane, cnt, bnd, rows, pol);
       else
-        warp_walk<false>(F, B, tg, i, G, s_w[warp], lane, cnt, rows, pol);
+        warp_walk<false>(F, B, tg, i, G, s_w[warp], lane, cnt, bnd, rows, pol);
       __syncwarp();
     }
-    if (active) F.nc[i] = cnt;
-    else if (ghost) F.nc[i] = 0;
+    if (active) {
+      F.nc[i] = cnt;
+      F.bnd[i] = bnd ? 1 : 0;
+    } else if (ghost) {
+      F.nc[i] = 0;
+      F.bnd[i] = 0;
+    }
     // copy the rows to the column-major list: lane l holds row l; the store of
     // slot k by the 32 lanes is one 128-B line
     const int len = active ? min(cnt, F.ngmax) : 0;

@@ -131,6 +131,13 @@ __device__ __forceinline__ void density_body(const Fields& F, const Params& P, c
 // IAD).
 __device__ __forceinline__ bool is_ghost(const Fields& F, int64_t i) { return (F.id[i] & SPH_GHOST_BIT) != 0; }
 
+// Target classes of a split IAD / MOMENTUM_ENERGY (sph_set_part, multi-rank
+// overlap): INTERIOR = no ghost among the neighbours (can run before the halo
+// values arrive), BOUNDARY = the rest (+ the ghosts' momentum records in IAD).
+__device__ __forceinline__ bool in_part(const Fields& F, int part, int64_t i) {
+  return part == SPH_PART_ALL || (part == SPH_PART_INTERIOR ? F.bnd[i] == 0 : F.bnd[i] != 0);
+}
+
 // The momentum record of a ghost (its C comes from the owner: halo, then
 // refresh_rec_m rewrites the C chunks).
 __device__ __forceinline__ void ghost_rec_m(const Fields& F, int64_t i, const Rec4& me) {
@@ -166,6 +173,7 @@ __global__ void __launch_bounds__(kDensThreads, 1024 / kDensThreads) density_ker
 __global__ void __launch_bounds__(256) eos_kernel(Fields F, Params P, bool apply_omega) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= F.n) return;
+  if (P.part == SPH_PART_GHOSTS && !is_ghost(F, i)) return;  // the ghosts' EOS after the rho halo
   const double rho = F.rho[i], u = F.f[FU][i];
   double p, c;
   if (P.eos == SPH_EOS_IDEAL) {
@@ -453,9 +461,10 @@ __global__ void __launch_bounds__(kIadDcThreads, 1) iad_dc_kernel(Fields F, Para
   const Geom g = load_geom(F.ds, P);
   const Rec4 me = F.rec_i[i];
   if (is_ghost(F, i)) {
-    ghost_rec_m(F, i, me);
+    if (P.part != SPH_PART_INTERIOR) ghost_rec_m(F, i, me);
     return;
   }
+  if (!in_part(F, P.part, i)) return;
   if (__any_sync(__activemask(), needs_wrap(g, me.a, me.b, me.c, F.f[FH][i])))
     iad_dc_body<true>(F, P, g, i, me);
   else
@@ -468,9 +477,10 @@ __global__ void __launch_bounds__(kIadThreads, 768 / kIadThreads) iad_kernel(Fie
   const Geom g = load_geom(F.ds, P);
   const Rec4 me = F.rec_i[i];
   if (is_ghost(F, i)) {
-    ghost_rec_m(F, i, me);
+    if (P.part != SPH_PART_INTERIOR) ghost_rec_m(F, i, me);
     return;
   }
+  if (!in_part(F, P.part, i)) return;
   if (__any_sync(__activemask(), needs_wrap(g, me.a, me.b, me.c, F.f[FH][i])))
     iad_body<true>(F, g, i, me);
   else
@@ -584,7 +594,8 @@ __device__ __forceinline__ double momentum_body(const Fields& F, const Params& P
 
 __global__ void __launch_bounds__(kMomThreads, 512 / kMomThreads) momentum_energy_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  const bool active = i < F.n && !is_ghost(F, i);  // ghosts: no sums, not in the dt minimum
+  // ghosts: no sums, not in the dt minimum; a split launch takes its class only
+  const bool active = i < F.n && !is_ghost(F, i) && in_part(F, P.part, i);
   unsigned long long hc = ~0ull;
   if (active) {
     const Geom g = load_geom(F.ds, P);

@@ -344,8 +344,9 @@ __global__ void __launch_bounds__(256) permute_kernel(Fields F, const uint32_t* 
   }
   F.id[i] = __ldg(id_src + p);
   const DevScalars* ds = F.ds;
+  // w = 1 marks a ghost (the neighbour search flags the targets that touch one)
   F.pos4[i] = make_float4((float)(v[FX] - ds->box_min[0]), (float)(v[FY] - ds->box_min[1]),
-                          (float)(v[FZ] - ds->box_min[2]), 0.f);
+                          (float)(v[FZ] - ds->box_min[2]), (__ldg(id_src + p) & SPH_GHOST_BIT) ? 1.f : 0.f);
   st4(F.rec_d + i, v[FX], v[FY], v[FZ], v[FM]);
 }
 

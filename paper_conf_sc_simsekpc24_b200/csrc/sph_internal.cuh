@@ -121,6 +121,7 @@ struct Fields {
   uint32_t* gcell_start;  // gravity octree: leaf ranges at level grav_level
   Rec4* gmom;             // gravity octree moments, 3 records per cell, levels 0..Lt
   int32_t* nc;
+  uint8_t* bnd;           // 1: the target has a ghost among its neighbours (search; multi-rank overlap)
   int32_t* nbr;           // [ngmax][cap] column-major: neighbour k of target i at nbr[k * cap + i]
   int32_t* nrows;         // neighbour-search scratch: row-major rows of the resident warps
   int64_t nrows_ld;       // their row stride (ngmax + 1 rounded up to 8: 32-B aligned rows, a spare word)
@@ -143,6 +144,7 @@ struct Params {
   int divcurl, av_switch;
   int gradh, dt_vsig, ve;
   int key_box_set;  // open axes take DevScalars::key_box (multi-rank: the global box)
+  int part;         // SPH_PART_*: which targets IAD / MOMENTUM_ENERGY / EOS process (sph_set_part)
 };
 
 // Process-wide count of libsph kernel launches (sph_kernel_launches).

@@ -95,6 +95,21 @@ class Comm:
                                    [int(c) for c in send_counts])
         return recv
 
+    def all_to_all_start(self, recv, send, recv_counts, send_counts):
+        """all_to_all that overlaps the caller's next kernels (NCCL: async on its
+        own stream; all_to_all_finish makes the current stream wait).  gloo and
+        world 1: completes here."""
+        if self.world == 1 or self.host:
+            self.all_to_all(recv, send, recv_counts, send_counts)
+            return None
+        return dist.all_to_all_single(recv, send.contiguous(), [int(c) for c in recv_counts],
+                                      [int(c) for c in send_counts], async_op=True)
+
+    @staticmethod
+    def all_to_all_finish(work):
+        if work is not None:
+            work.wait()
+
     def all_gather(self, t):
         if self.world == 1:
             return [t]
@@ -157,6 +172,8 @@ class DistributedSim:
         # force_exchange: run the partition / migration / ghost / halo plumbing even
         # on one rank (it then moves nothing) -- measures its cost (tools/decomp_probe.py)
         self.xchg = force_exchange
+        # overlap the H2 / H3 halos with the interior targets (not with grad-h / VE)
+        self.overlap = kw.pop("overlap", True) and not (getattr(params, "gradh", 0) or getattr(params, "ve", 0))
         self.params = params
         self.comm = Comm()
         self.dev = torch.device("cuda", device)
@@ -271,19 +288,40 @@ class DistributedSim:
             self._mark("tree_maps")
         sim.find_neighbors(stats=False)
         sim.density()
-        self._halo(["rho"])
-        sim.eos()
-        if getattr(self.params, "gradh", 0) or getattr(self.params, "ve", 0):
-            sim.gradh()  # owners' normalised rho (volume elements) and Omega over the ghosts
-            self._halo((["rho"] if getattr(self.params, "ve", 0) else [])
-                       + (["omega"] if getattr(self.params, "gradh", 0) else []))
-        sim.iad()
-        # H3: the owners' C (and Balsara factors when the AV switch is on)
         h3 = ["c11", "c12", "c13", "c22", "c23", "c33"]
         if getattr(self.params, "av_switch", 0):
             h3.append("bal")
-        self._halo(h3)
-        sim.momentum_energy()
+        if xchg and self.overlap:
+            # H2 / H3 in flight while the targets without ghost neighbours are
+            # computed (sph_set_part); each target is computed once, so the
+            # result equals the unsplit step bit for bit
+            P = self.sph
+            w2 = self._halo_start(["rho"])
+            sim.eos()                                  # ghosts' values fixed below
+            sim.set_part(P.PART_INTERIOR)
+            sim.iad()
+            self._halo_finish(w2)
+            sim.set_part(P.PART_GHOSTS)
+            sim.eos()
+            sim.set_part(P.PART_BOUNDARY)
+            sim.iad()
+            w3 = self._halo_start(h3)
+            sim.set_part(P.PART_INTERIOR)
+            sim.momentum_energy()
+            self._halo_finish(w3)
+            sim.set_part(P.PART_BOUNDARY)
+            sim.momentum_energy()
+            sim.set_part(P.PART_ALL)
+        else:
+            self._halo(["rho"])
+            sim.eos()
+            if getattr(self.params, "gradh", 0) or getattr(self.params, "ve", 0):
+                sim.gradh()  # owners' normalised rho (volume elements) and Omega over the ghosts
+                self._halo((["rho"] if getattr(self.params, "ve", 0) else [])
+                           + (["omega"] if getattr(self.params, "gradh", 0) else []))
+            sim.iad()
+            self._halo(h3)  # H3: the owners' C (and Balsara factors with the AV switch)
+            sim.momentum_energy()
         if sim.stir_enabled:  # driving: every rank holds the same OU state and noise
             sim.stir()
         self._mark("physics_halos")
@@ -301,12 +339,20 @@ class DistributedSim:
     def _halo(self, names):
         if not (self.comm.world > 1 or self.xchg):
             return
+        self._halo_finish(self._halo_start(names))
+
+    def _halo_start(self, names):
         sim = self.sim
         send = sim.halo_gather(names, self._src)
         recv = torch.empty((sum(self.g_recv), len(names)), dtype=torch.float64, device=self.dev)
-        self.comm.all_to_all(recv, send, self.g_recv, self.g_send)
+        work = self.comm.all_to_all_start(recv, send, self.g_recv, self.g_send)
+        return names, send, recv, work
+
+    def _halo_finish(self, h):
+        names, send, recv, work = h
+        self.comm.all_to_all_finish(work)
         if recv.shape[0]:
-            sim.halo_scatter(names, self._dst, recv)
+            self.sim.halo_scatter(names, self._dst, recv)
 
     def gather_state(self):
         """All particles on every rank, sorted by id (host numpy) -- for tests."""

@@ -31,6 +31,7 @@ FIELD_ID = {name: k for k, name in enumerate(FIELDS)}
 FIELD_DTYPE = {"id": np.int64, "key": np.uint64, "nc": np.int32, "order": np.int32}
 ROW_DOUBLES = 11  # SPH_ROW_DOUBLES: x y z vx vy vz h m u du_m1 id(bits)
 MEM_HOST, MEM_DEVICE, MEM_HOST_ASYNC = 0, 1, 2
+PART_ALL, PART_INTERIOR, PART_BOUNDARY, PART_GHOSTS = 0, 1, 2, 3
 ACCOUNTING_OFF, ACCOUNTING_PHASE = 0, 1
 CLOCK_DEFAULT, CLOCK_STATIC, CLOCK_PER_PHASE = 0, 1, 2
 
@@ -106,7 +107,8 @@ EXPORTS = ("sph_config_default", "sph_workspace_size", "sph_init", "sph_finalize
            "sph_select_ghosts", "sph_gather_field", "sph_scatter_field",
            "sph_decomp_reduce", "sph_set_key_box", "sph_key_histogram", "sph_decomp_owners",
            "sph_decomp_ghosts", "sph_decomp_pack", "sph_decomp_drop", "sph_decomp_map",
-           "sph_halo_gather", "sph_halo_scatter", "sph_min_hc_dev", "sph_set_min_hc_dev", "sph_sync")
+           "sph_halo_gather", "sph_halo_scatter", "sph_min_hc_dev", "sph_set_min_hc_dev", "sph_sync",
+           "sph_set_part")
 GHOST_BIT = 1 << 62
 
 _lib = None
@@ -183,6 +185,7 @@ def load(build_if_missing: bool = True):
     L.sph_min_hc_dev.argtypes = [P, V]
     L.sph_set_min_hc_dev.argtypes = [P, V]
     L.sph_sync.argtypes = [P]
+    L.sph_set_part.argtypes = [P, I]
     L.sph_supported_clocks.argtypes = [P, V, I, C.POINTER(I)]
     L.sph_trace_start.argtypes = [P, D, I64]
     L.sph_trace_stop.argtypes = [P, V, I64, C.POINTER(I64)]
@@ -489,6 +492,10 @@ class Simulation:
         self._keep_src = (idx, src)
         self._ok(self.L.sph_halo_scatter(self.ctx, f, len(names), C.c_void_p(idx.data_ptr()), idx.numel(),
                                          C.c_void_p(src.data_ptr())))
+
+    def set_part(self, part: int):
+        """sph_set_part: PART_ALL / PART_INTERIOR / PART_BOUNDARY / PART_GHOSTS."""
+        self._ok(self.L.sph_set_part(self.ctx, int(part)))
 
     def min_hc_dev(self):
         out = self.torch.empty(1, dtype=self.torch.float64, device=self.device)

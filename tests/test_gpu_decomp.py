@@ -270,3 +270,45 @@ def test_device_routing_matches_reference(case):
         assert np.array_equal(post, inv[[0, 5, len(kept) - 1]])
         assert np.array_equal(sim.decomp_map(None, first=2, m=3).cpu().numpy(), inv[2:5])
     sim.finalize()
+
+
+def test_split_parts_state_machine_and_identity():
+    """sph_set_part on one rank: INTERIOR leaves the stage, BOUNDARY advances it;
+    the split calls give the unsplit fields bit for bit; GHOSTS is EOS-only;
+    split calls are refused with grad-h."""
+    from paper_conf_sc_simsekpc24_b200 import sph
+    from parity import gpu_pipeline, new_sim
+    w = ics.turbulence(16)
+    a = new_sim(w)
+    ga = gpu_pipeline(a)
+    b = new_sim(w)
+    b.build_tree()
+    b.find_neighbors()
+    b.density()
+    b.eos()
+    b.set_part(sph.PART_INTERIOR)
+    b.iad()
+    with pytest.raises(sph.SphError):
+        b.momentum_energy()                 # the boundary IAD half is pending
+    b.set_part(sph.PART_GHOSTS)
+    b.eos()
+    with pytest.raises(sph.SphError):
+        b.iad()                              # GHOSTS is for EOS only
+    b.set_part(sph.PART_BOUNDARY)
+    b.iad()
+    b.set_part(sph.PART_INTERIOR)
+    b.momentum_energy()
+    b.set_part(sph.PART_BOUNDARY)
+    b.momentum_energy()
+    b.set_part(sph.PART_ALL)
+    for k in ("rho", "c11", "c23", "ax", "ay", "az", "du"):
+        assert np.array_equal(b.get_field(k), a.get_field(k)), k
+    assert b.timestep() == a.timestep()
+    a.finalize()
+    b.finalize()
+    import dataclasses
+    w.params = dataclasses.replace(w.params, gradh=1)
+    c = new_sim(w)
+    with pytest.raises(sph.SphError):
+        c.set_part(sph.PART_INTERIOR)
+    c.finalize()
