@@ -19,6 +19,12 @@
 
 namespace sph {
 
+// diagnostic builds only (SPH_NVCC_EXTRA=-DSPH_MOM_DIAG=1 / 2): the
+// momentum-energy loop with its gathers alone / its arithmetic alone
+#ifndef SPH_MOM_DIAG
+#define SPH_MOM_DIAG 0
+#endif
+
 constexpr double kPi = 3.14159265358979323846;
 constexpr double kPi2Over4 = kPi * kPi / 4.0;
 constexpr double kPi2 = kPi * kPi;
@@ -525,10 +531,27 @@ __device__ __forceinline__ double momentum_body(const Fields& F, const Params& P
     p0 = p1;
     r0 = r1;
     if (k + 2 < nci) {
+#if SPH_MOM_DIAG == 2
+      r1 = rec + (int64_t)kRecM * ((i & ~31ll) + ((jn & 1) ? 1 : 0));  // diagnostic: broadcast records
+#else
       r1 = rec + (int64_t)kRecM * jn;
+#endif
       p1 = ldg4(r1);
     }
     if (k + 3 < nci) jn = __ldg(nb + (int64_t)(k + 3) * cap);
+#if SPH_MOM_DIAG == 1
+    // diagnostic: the gathers alone (every load, no pair arithmetic)
+    ax += j0.a + j1.a + j2.b + j3.c;
+    if (j0.d < 0.0) {  // never: keeps the AV-chunk load of ~half the pairs
+      const Rec4 j4d = ldg4(rcur + 4);
+      ay += j4d.a;
+    }
+    if ((k & 1) == 0) {
+      const Rec4 j4d = ldg4(rcur + 4);
+      az += j4d.b;
+    }
+    continue;
+#endif
     double dx, dy, dz;
     pair_d<kWrap>(g, xi, yi, zi, j0.a, j0.b, j0.c, dx, dy, dz);
     const double r2 = dx * dx + dy * dy + dz * dz;
