@@ -124,6 +124,9 @@ __device__ __forceinline__ void ld8i_hint(const int32_t* p, int (&v)[8], uint64_
 }
 
 constexpr int kNbrThreads = 128;
+#ifndef SPH_NBR_MINB
+#define SPH_NBR_MINB 6  // resident CTAs per SM (6 -> 80 registers)
+#endif
 constexpr int kNbrWarps = kNbrThreads / 32;
 constexpr int kMaxWarpCells = 128;
 
@@ -594,7 +597,7 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
   }
 }
 
-__global__ void __launch_bounds__(kNbrThreads, 6) neighbors_kernel(Fields F, Params P) {
+__global__ void __launch_bounds__(kNbrThreads, SPH_NBR_MINB) neighbors_kernel(Fields F, Params P) {
   __shared__ WarpSmem s_w[kNbrWarps];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const DevScalars* ds = F.ds;
