@@ -95,20 +95,31 @@ def _single(name):
 @pytest.mark.parametrize("name", ["turbulence16", "random", "sedov14", "sedov14_balsara",
                                   "random_gradh_vsig", "random_ve", "noh14_open"])
 def test_two_ranks_bit_identical_to_one(name):
+    _ranks_bit_identical(name, 2)
+
+
+@pytest.mark.parametrize("name,world", [("turbulence16", 4), ("noh14_open", 4), ("random", 8)])
+def test_more_ranks_bit_identical_to_one(name, world):
+    """The 4- and 8-rank paths (split points, 64-bit ghost masks, halo lists over
+    several peers): still bit-identical to one rank (all ranks on one GPU, gloo)."""
+    _ranks_bit_identical(name, world)
+
+
+def _ranks_bit_identical(name, world):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, name, q)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, name, q)) for r in range(world)]
     for p in procs:
         p.start()
-    res = dict(q.get(timeout=600) for _ in procs)
+    res = dict(q.get(timeout=900) for _ in procs)
     for p in procs:
         p.join(timeout=60)
     for v in res.values():
         if isinstance(v, Exception):
             raise v
     dts1, st1 = _single(name)
-    for r in (0, 1):
+    for r in range(world):
         dts2, st2, stats = res[r]
         assert dts2 == dts1, "dt is the same global minimum"
         assert stats["n_ghost"] > 0
