@@ -706,6 +706,10 @@ int sph_init(const sph_config* cfg, void* arena, size_t arena_bytes, void* strea
   c->P.dt_vsig = cfg->dt_vsig ? 1 : 0;
   c->P.key_box_set = 0;
   c->P.part = SPH_PART_ALL;
+  {
+    const char* mr = getenv("SPH_NBR_MERGE_RUNS");  // test hook: exercises the merged-run search path
+    c->P.nbr_merge_runs = mr ? atoi(mr) : -1;
+  }
   layout(cfg, (char*)arena, c);
   for (int p = 0; p < SPH_NPHASES; ++p) {
     c->pending[p] = false;

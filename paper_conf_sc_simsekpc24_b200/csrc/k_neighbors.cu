@@ -232,15 +232,29 @@ __device__ __forceinline__ unsigned long long fma2(unsigned long long a, unsigne
 }
 
 
-constexpr int kMaxRuns = 4 * kMaxWarpCells;  // <= 4 runs of children per cell
+// Run table size.  A cell contributes up to 4 runs of needed children; when the
+// group's runs would exceed kMaxRuns, each cell's needed children are merged into
+// one run (the unneeded children in between become candidates that fail the
+// test), so kMaxRuns >= kMaxWarpCells always suffices.  A small table leaves
+// more of the SM's 256 KB to L1.
+#ifndef SPH_NBR_MAXRUNS
+#define SPH_NBR_MAXRUNS 128
+#endif
+constexpr int kMaxRuns = SPH_NBR_MAXRUNS;
+static_assert(kMaxRuns >= kMaxWarpCells, "one merged run per cell must fit");
 
 struct WarpSmem {
   uint32_t cell[kMaxWarpCells];   // sorted coarse cell keys
   uint32_t ucs[kMaxWarpCells];    // their unwrapped coordinates (biased, packed)
   uint32_t mask[kMaxWarpCells];   // children any lane needs
-  uint32_t run_start[kMaxRuns];   // first particle of each run
-  uint32_t run_pos[kMaxRuns + 1]; // stream position of each run (exclusive prefix)
-  uint32_t run_cell[kMaxRuns];    // periodic image code of the run's cell (2 bits/axis)
+  union {
+    struct {
+      uint32_t run_start[kMaxRuns];   // first particle of each run
+      uint32_t run_pos[kMaxRuns + 1]; // stream position of each run (exclusive prefix)
+      uint32_t run_cell[kMaxRuns];    // periodic image code of the run's cell (2 bits/axis)
+    };
+    unsigned long long sortkey[kMaxWarpCells];  // build_cells scratch
+  };
   // staged chunk of 32 candidates (image-shifted fp32 position, SoA so that two
   // consecutive candidates are one 64-bit load for the packed f32x2 math)
   alignas(16) float cx[32];
@@ -317,7 +331,7 @@ __device__ __forceinline__ GroupBox build_cells(const Box& B, const int (&cc)[3]
     }
   }
   // rank sort (ties -> lower slot first), then drop duplicates
-  unsigned long long* sk = reinterpret_cast<unsigned long long*>(S.run_start);  // scratch (>= 1 KB)
+  unsigned long long* sk = S.sortkey;
 #pragma unroll
   for (int r = 0; r < kMaxWarpCells / 32; ++r) sk[r * 32 + lane] = v[r];
   __syncwarp();
@@ -374,7 +388,8 @@ __device__ __forceinline__ GroupBox build_cells(const Box& B, const int (&cc)[3]
 template <bool kFull>
 __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const Target& t, int64_t i,
                                           const GroupBox& G, WarpSmem& S, int lane, int& cnt,
-                                          bool& bnd, int32_t* __restrict__ rows, const L2Pol& pol) {
+                                          bool& bnd, int32_t* __restrict__ rows, const L2Pol& pol,
+                                          int merge_runs) {
   const int n = B.nside;
   const int T = G.T;
   const int ngmax = F.ngmax;
@@ -396,6 +411,16 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
   }
   __syncwarp();
   // ---- 2b. runs (one cell per lane), placed by a warp prefix sum in cell order
+  bool merge = false;  // one run per cell (see kMaxRuns)
+  const int run_lim = merge_runs < 0 ? kMaxRuns : min(merge_runs, kMaxRuns);
+  if (4 * T > run_lim) {
+    uint32_t tr = 0;
+    for (int u = lane; u < T; u += 32) {
+      const uint32_t mk = S.mask[u];
+      tr += __popc(mk & ~(mk << 1));  // runs of set bits
+    }
+    merge = __reduce_add_sync(0xffffffffu, tr) > (uint32_t)run_lim;
+  }
   uint32_t nruns = 0, ncand = 0;
   for (int r0 = 0; r0 < T; r0 += 32) {
     const int u = r0 + lane;
@@ -413,6 +438,7 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
 #pragma unroll
     for (int q = 0; q < 4; ++q) rs[q] = re[q] = 0;
     uint32_t m = mask;
+    if (merge && mask) m = ((2u << (31 - __clz(mask))) - 1u) & ~((1u << (__ffs(mask) - 1)) - 1u);
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
       if (m) {
@@ -663,9 +689,9 @@ __global__ void __launch_bounds__(kNbrThreads, SPH_NBR_MINB) neighbors_kernel(Fi
       Target tg = t;
       if (lane / g != gid) tg.r_out2 = tg.r_in2 = tg.rc = -1.f;  // not in this pass
       if (G.full[0] || G.full[1] || G.full[2])
-        warp_walk<true>(F, B, tg, i, G, s_w[warp], lane, cnt, bnd, rows, pol);
+        warp_walk<true>(F, B, tg, i, G, s_w[warp], lane, cnt, bnd, rows, pol, P.nbr_merge_runs);
       else
-        warp_walk<false>(F, B, tg, i, G, s_w[warp], lane, cnt, bnd, rows, pol);
+        warp_walk<false>(F, B, tg, i, G, s_w[warp], lane, cnt, bnd, rows, pol, P.nbr_merge_runs);
       __syncwarp();
     }
     if (active) {

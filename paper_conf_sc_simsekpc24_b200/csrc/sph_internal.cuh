@@ -145,6 +145,8 @@ struct Params {
   int gradh, dt_vsig, ve;
   int key_box_set;  // open axes take DevScalars::key_box (multi-rank: the global box)
   int part;         // SPH_PART_*: which targets IAD / MOMENTUM_ENERGY / EOS process (sph_set_part)
+  int nbr_merge_runs;  // search: merge each cell's runs above this many runs (-1: the table size;
+                       // test hook SPH_NBR_MERGE_RUNS, read at sph_init)
 };
 
 // Process-wide count of libsph kernel launches (sph_kernel_launches).

@@ -525,7 +525,8 @@ class Simulation:
     def find_neighbors(self, stats: bool = True):
         s = NbrStats()
         self._ok(self.L.sph_find_neighbors(self.ctx, C.byref(s) if stats else None))
-        return {"min_nc": s.min_nc, "max_nc": s.max_nc, "mean_nc": s.mean_nc, "total": s.total}
+        return {"min_nc": s.min_nc, "max_nc": s.max_nc, "mean_nc": s.mean_nc, "total": s.total,
+                "candidates": s.candidates, "passes": s.passes}
 
     def get_neighbors(self):
         off = np.zeros(self.n + 1, dtype=np.int64)

@@ -137,6 +137,56 @@ def test_lone_particle_is_singular():
     assert e.value.name == "ERR_SINGULAR"
 
 
+@pytest.mark.parametrize("wname,level", [("turbulence20", 2), ("turbulence20", 3), ("random_open", 3),
+                                         ("noh14", 3)])
+def test_neighbour_lists_coarse_grid(wname, level):
+    """A coarse cell grid (max_cell_level 2-3: 2-4 cells per axis) gives warps
+    thousands of candidates: more than the search's per-warp scratch holds in one
+    segment (nrows_ld chunks of 32 candidates), so the lists are expanded segment by
+    segment (lanes at different list positions), and at level 2 the periodic axes
+    are "full" (minimum image per candidate).  Lists stay bit-exact vs brute force."""
+    w = WORKLOADS[wname]
+    o = oracle.step({k: v.copy() for k, v in w.state.items()}, w.params, w.params.dt_first, True)[1]
+    sim = new_sim(w, max_cell_level=level)
+    sim.build_tree()
+    stats = sim.find_neighbors()
+    nb = o["nb"]
+    assert np.array_equal(sim.get_field("nc"), nb.nc)
+    off, idx = sim.get_neighbors()
+    assert np.array_equal(off, nb.offsets)
+    assert np.array_equal(idx.astype(np.int64), nb.idx)
+    # at level 2 (every axis "full") the candidate streams exceed one segment
+    nrows_ld = (w.params.ngmax + 8) // 8 * 8
+    if level == 2:
+        assert stats["candidates"] / max(stats["passes"], 1) > nrows_ld * 32
+    sim.finalize()
+
+
+@pytest.mark.parametrize("wname", ["turbulence20", "random_open", "sedov16"])
+def test_neighbour_lists_merged_runs(wname, monkeypatch):
+    """The search's run table overflow path: with SPH_NBR_MERGE_RUNS=0 every
+    cell's needed children are merged into one run (more candidates, the same
+    decisions), as happens when a group's runs exceed the table.  Lists stay
+    bit-exact and the candidate count does not drop."""
+    w = WORKLOADS[wname]
+    o = oracle.step({k: v.copy() for k, v in w.state.items()}, w.params, w.params.dt_first, True)[1]
+    cand = {}
+    for env in (None, "0"):
+        if env is None:
+            monkeypatch.delenv("SPH_NBR_MERGE_RUNS", raising=False)
+        else:
+            monkeypatch.setenv("SPH_NBR_MERGE_RUNS", env)
+        sim = new_sim(w)
+        sim.build_tree()
+        stats = sim.find_neighbors()
+        cand[env] = stats["candidates"]
+        off, idx = sim.get_neighbors()
+        assert np.array_equal(off, o["nb"].offsets)
+        assert np.array_equal(idx.astype(np.int64), o["nb"].idx)
+        sim.finalize()
+    assert cand["0"] >= cand[None]
+
+
 def test_capacity_error_reports_needed_size():
     from paper_conf_sc_simsekpc24_b200 import sph
     w = ics.sedov(10)
