@@ -237,6 +237,14 @@ __device__ __forceinline__ unsigned long long fma2(unsigned long long a, unsigne
 // one run (the unneeded children in between become candidates that fail the
 // test), so kMaxRuns >= kMaxWarpCells always suffices.  A small table leaves
 // more of the SM's 256 KB to L1.
+// 1: a chunk's candidates find their runs by one warp mask of the run starts in
+// the chunk; 0: each lane advances its own run pointer (a divergent loop).
+#ifndef SPH_NBR_RUNSCAN
+#define SPH_NBR_RUNSCAN 1
+#endif
+#ifndef SPH_NBR_IMGSKIP
+#define SPH_NBR_IMGSKIP 1
+#endif
 #ifndef SPH_NBR_MAXRUNS
 #define SPH_NBR_MAXRUNS 128
 #endif
@@ -411,6 +419,7 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
   }
   __syncwarp();
   // ---- 2b. runs (one cell per lane), placed by a warp prefix sum in cell order
+  bool img = false;    // any run of a periodic image cell (shifted candidates)
   bool merge = false;  // one run per cell (see kMaxRuns)
   const int run_lim = merge_runs < 0 ? kMaxRuns : min(merge_runs, kMaxRuns);
   if (4 * T > run_lim) {
@@ -480,6 +489,7 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
       for (int a = 0; a < 3; ++a)
         if (!(kFull && G.full[a])) code |= (uint32_t)(uc[a] < 0 ? 1 : (uc[a] >= n ? 2 : 0)) << (2 * a);
     }
+    img = img || __any_sync(0xffffffffu, code != 0u);
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
       if (q < (int)my_runs) {
@@ -502,22 +512,42 @@ __device__ __forceinline__ void warp_walk(const Fields& F, const Box& B, const T
   // ---- 3./4. stream, test, append
   const uint32_t nchunks = (ncand + 31) / 32;
   uint32_t run = 0;
+#if SPH_NBR_RUNSCAN
+  int rb = -1;  // warp-uniform: the last run starting before the chunk
+#endif
   float4 q = make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);  // NaN: fails every test
   float sx = 0.f, sy = 0.f, sz = 0.f;
   uint32_t qj = 0;
   auto load = [&](uint32_t c) {
     const uint32_t g = c * 32 + (uint32_t)lane;
+#if SPH_NBR_RUNSCAN
+    {
+      // each lane examines one of the next 32 run starts; the runs starting in
+      // this chunk become bits of a warp mask, and a lane's run is the number of
+      // starts at or below its slot (no per-lane search loop)
+      const int e = rb + 1 + lane;
+      const uint32_t st = e <= (int)nruns ? S.run_pos[e] : 0xffffffffu;
+      const uint32_t off = st - c * 32;  // >= 0: run rb + 1 starts after the previous chunk
+      const uint32_t smask = __reduce_or_sync(0xffffffffu, off < 32u ? 1u << off : 0u);
+      run = (uint32_t)(rb + __popc(smask & ((2u << lane) - 1u)));
+      rb += __popc(smask);
+    }
+#endif
     sx = sy = sz = 0.f;
     if (g >= ncand) {
       q = make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
       qj = 0;
       return;
     }
+#if !SPH_NBR_RUNSCAN
     while (S.run_pos[run + 1] <= g) ++run;
+#endif
     qj = S.run_start[run] + (g - S.run_pos[run]);
     q = F.pos4[qj];
     // unwrapped position of the candidate = stored + k L (k = -1, 0, 1); the
-    // shift is applied when the chunk is staged (keeps the load latency hidden)
+    // shift is applied when the chunk is staged (keeps the load latency hidden).
+    // Most warps have no image cell at all (warp-uniform skip).
+    if (SPH_NBR_IMGSKIP && !img) return;
     const uint32_t code = S.run_cell[run];
     const uint32_t c0 = code & 3u, c1 = (code >> 2) & 3u, c2 = (code >> 4) & 3u;
     sx = c0 == 1u ? -B.Lf[0] : (c0 == 2u ? B.Lf[0] : 0.f);
