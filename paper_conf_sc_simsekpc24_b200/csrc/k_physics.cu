@@ -36,7 +36,11 @@ constexpr double kPi2 = kPi * kPi;
 // persistent contiguous-range grid was slower: spills and tail imbalance).
 constexpr int kDensThreads = 1024;
 constexpr int kIadThreads = 768;
-constexpr int kMomThreads = 512;
+// A/B builds only: other CTA sizes of momentum-energy
+#ifndef SPH_MOM_THREADS
+#define SPH_MOM_THREADS 512
+#endif
+constexpr int kMomThreads = SPH_MOM_THREADS;
 
 struct Geom {
   double L[3], H[3], lo[3], hi[3];
@@ -615,7 +619,7 @@ __device__ __forceinline__ double momentum_body(const Fields& F, const Params& P
   return vs;
 }
 
-__global__ void __launch_bounds__(kMomThreads, 512 / kMomThreads) momentum_energy_kernel(Fields F, Params P) {
+__global__ void __launch_bounds__(kMomThreads, kMomThreads >= 512 ? 1 : 512 / kMomThreads) momentum_energy_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   // ghosts: no sums, not in the dt minimum; a split launch takes its class only
   const bool active = i < F.n && !is_ghost(F, i) && in_part(F, P.part, i);
