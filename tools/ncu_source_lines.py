@@ -41,3 +41,26 @@ def main(path, top=40):
 
 if __name__ == "__main__":
     main(sys.argv[1], int(sys.argv[2]) if len(sys.argv) > 2 else 40)
+
+
+def stalls(path, lines):
+    """Stall-reason breakdown (sampled) of the given source lines."""
+    hdr = None
+    f = None
+    out = {}
+    for row in csv.reader(open(path)):
+        if not row:
+            continue
+        if row[0] == "File Path":
+            f = row[1].split("/")[-1]
+            continue
+        if row[0] == "Line No":
+            hdr = row
+            continue
+        if hdr is None or not row[0]:
+            continue
+        key = f"{f}:{row[0]}"
+        if key in lines:
+            cols = [(h, row[k]) for k, h in enumerate(hdr) if h.startswith("stall_") and "Not Issued" not in h]
+            out[key] = {h[6:]: int(v) for h, v in cols if v not in ("", "-", "0")}
+    return out
