@@ -176,7 +176,13 @@ typedef struct sph_config {
                                C min h/c                                          */
   int32_t ve;               /* 1: generalized volume elements X = m/rho0 (reading
                                23): GRADH normalises the density                  */
-  int32_t reserved[5];
+  int32_t grav_fp64;        /* gravity with theta > 0: 0 (default) evaluates each
+                               multipole / direct term in fp32 from positions
+                               relative to the walking group's centre and adds it
+                               to fp64 accumulators (rounding ~1e-7 of a term,
+                               far below the tree's truncation error); 1 = fp64
+                               terms.  theta = 0 (the direct sum) is always fp64. */
+  int32_t reserved[4];
 } sph_config;
 
 typedef struct sph_nbr_stats {

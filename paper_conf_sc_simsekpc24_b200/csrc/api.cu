@@ -478,7 +478,8 @@ int body_simple(sph_ctx* c, int phase, int next_stage) {
       break;
     case SPH_PHASE_STIR: launch_stir(F, c->P, c->stir, c->st); break;
     case SPH_PHASE_GRAVITY: {
-      GravParams G{c->cfg.grav_G, c->cfg.grav_eps, c->cfg.grav_theta, c->cfg.grav_level};
+      GravParams G{c->cfg.grav_G, c->cfg.grav_eps, c->cfg.grav_theta, c->cfg.grav_level,
+                   (c->cfg.grav_theta > 0.0 && !c->cfg.grav_fp64) ? 1 : 0};
       launch_gravity(F, G, c->st);
       break;
     }

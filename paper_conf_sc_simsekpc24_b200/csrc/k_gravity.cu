@@ -119,6 +119,10 @@ struct GravSmem {
   uint32_t stack[kGravStack];   // parents whose 8 children are still to examine
   double mom[8][10];            // the accepted children's moments (m, com, Q)
   double px[32], py[32], pz[32], pm[32];  // a batch of leaf particles
+  // fp32 terms (GravParams::fp32): moments with the COM relative to the group's
+  // centre, and leaf particles relative to it
+  float momf[8][12];            // m, com - o (3), Q (6)
+  float pxf[32], pyf[32], pzf[32], pmf[32];
 };
 
 // Multipole (monopole + traceless quadrupole, unsoftened) of cell moments q at
@@ -140,6 +144,26 @@ __device__ __forceinline__ void add_multipole(const double* q, double xi, double
   phi += -Gc * q[0] * ir - 0.5 * Gc * rQr * ir5;
 }
 
+// The same multipole with fp32 terms: r = (x_i - o) - (com - o), both rounded
+// to fp32 relative to the group's centre o (|x_i - o| is within the group and
+// |com - o| <= |r| + the group's size, so the rounding of r is ~1e-7 of |r|).
+__device__ __forceinline__ void add_multipole_f(const float* q, float xf, float yf, float zf, float Gc,
+                                                float& ax, float& ay, float& az, float& phi) {
+  const float rx = xf - q[1], ry = yf - q[2], rz = zf - q[3];
+  const float r2 = fmaf(rx, rx, fmaf(ry, ry, rz * rz));
+  const float ir = rsqrtf(r2), ir2 = ir * ir, ir3 = ir * ir2, ir5 = ir3 * ir2;
+  const float Qx = fmaf(q[4], rx, fmaf(q[5], ry, q[6] * rz));
+  const float Qy = fmaf(q[5], rx, fmaf(q[7], ry, q[8] * rz));
+  const float Qz = fmaf(q[6], rx, fmaf(q[8], ry, q[9] * rz));
+  const float rQr = fmaf(rx, Qx, fmaf(ry, Qy, rz * Qz));
+  const float gi5 = Gc * ir5;
+  const float s = -Gc * q[0] * ir3 - 2.5f * rQr * gi5 * ir2;  // mono + quad (radial)
+  ax = fmaf(s, rx, fmaf(gi5, Qx, ax));
+  ay = fmaf(s, ry, fmaf(gi5, Qy, ay));
+  az = fmaf(s, rz, fmaf(gi5, Qz, az));
+  phi -= fmaf(0.5f * rQr, gi5, Gc * q[0] * ir);
+}
+
 // One warp per 32 consecutive targets.  The stack holds parents; popping one
 // examines its 8 children together (lanes 0-7 load and classify one child each:
 // one memory round trip per 8 cells instead of 8 dependent ones): accepted
@@ -151,6 +175,7 @@ __device__ __forceinline__ void add_multipole(const double* q, double xi, double
 // One walk for the lanes in `mine` (a group of the tile's targets): the
 // opening test uses the bounding box of the group's targets only; the other
 // lanes follow the warp-uniform walk and discard what they compute.
+template <bool kF32>
 __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G, GravSmem& S, int lane,
                                            int64_t i, bool active, bool mine, double& tax, double& tay,
                                            double& taz, double& tphi) {
@@ -172,6 +197,10 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
   const int Lt = G.level;
   double ax = 0, ay = 0, az = 0, phi = 0;
   unsigned long long n_mp = 0, n_pp = 0, n_pop = 0;  // diagnostics (warp-uniform)
+  // fp32 terms: positions relative to the group's centre o (warp-uniform)
+  const double ox = 0.5 * (lo[0] + hi[0]), oy = 0.5 * (lo[1] + hi[1]), oz = 0.5 * (lo[2] + hi[2]);
+  const float xf = (float)(xi - ox), yf = (float)(yi - oy), zf = (float)(zi - oz);
+  const float Gf = (float)Gc, eps2f = (float)eps2;
 
   // the root itself: accepted, a leaf (Lt = 0 is not allowed) or opened
   int sp = 0;
@@ -219,9 +248,17 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
         if (side * side < th2 * dd2) {
           acc = true;
           const Rec4 m1 = ldg4(F.gmom + 3 * (g0 + lane) + 1), m2 = ldg4(F.gmom + 3 * (g0 + lane) + 2);
-          double* q = S.mom[lane];
-          q[0] = m0.a; q[1] = m0.b; q[2] = m0.c; q[3] = m0.d;
-          q[4] = m1.a; q[5] = m1.b; q[6] = m1.c; q[7] = m1.d; q[8] = m2.a; q[9] = m2.b;
+          if (kF32) {
+            float* q = S.momf[lane];
+            q[0] = (float)m0.a;
+            q[1] = (float)(m0.b - ox); q[2] = (float)(m0.c - oy); q[3] = (float)(m0.d - oz);
+            q[4] = (float)m1.a; q[5] = (float)m1.b; q[6] = (float)m1.c; q[7] = (float)m1.d;
+            q[8] = (float)m2.a; q[9] = (float)m2.b;
+          } else {
+            double* q = S.mom[lane];
+            q[0] = m0.a; q[1] = m0.b; q[2] = m0.c; q[3] = m0.d;
+            q[4] = m1.a; q[5] = m1.b; q[6] = m1.c; q[7] = m1.d; q[8] = m2.a; q[9] = m2.b;
+          }
         } else if (l == Lt) {
           leaf = true;
         } else {
@@ -236,7 +273,22 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
     // multipoles, two at a time into separate accumulators (independent
     // dependency chains: the rsqrt + quadrupole chain is latency-bound)
     n_mp += __popc(am);
-    {
+    if (kF32) {
+      // this node's (<= 8) multipole terms summed in fp32, then added in fp64
+      float fx = 0.f, fy = 0.f, fz = 0.f, fphi = 0.f, gx = 0.f, gy = 0.f, gz = 0.f, gphi = 0.f;
+      uint32_t m = am;
+      for (; __popc(m) >= 2; m &= m - 1, m &= m - 1) {
+        const int k0 = __ffs(m) - 1;
+        const int k1 = __ffs(m & (m - 1)) - 1;
+        add_multipole_f(S.momf[k0], xf, yf, zf, Gf, fx, fy, fz, fphi);
+        add_multipole_f(S.momf[k1], xf, yf, zf, Gf, gx, gy, gz, gphi);
+      }
+      if (m) add_multipole_f(S.momf[__ffs(m) - 1], xf, yf, zf, Gf, fx, fy, fz, fphi);
+      ax += (double)fx + (double)gx;
+      ay += (double)fy + (double)gy;
+      az += (double)fz + (double)gz;
+      phi += (double)fphi + (double)gphi;
+    } else {
       double bx = 0, by = 0, bz = 0, bphi = 0;
       uint32_t m = am;
       for (; __popc(m) >= 2; m &= m - 1, m &= m - 1) {
@@ -262,28 +314,57 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
         __syncwarp();
         if ((uint32_t)lane < nb) {
           const Rec4 r = ldg4(F.rec_d + b + lane);
-          S.px[lane] = r.a;
-          S.py[lane] = r.b;
-          S.pz[lane] = r.c;
-          S.pm[lane] = r.d;
+          if (kF32) {
+            S.pxf[lane] = (float)(r.a - ox);
+            S.pyf[lane] = (float)(r.b - oy);
+            S.pzf[lane] = (float)(r.c - oz);
+            S.pmf[lane] = (float)r.d;
+          } else {
+            S.px[lane] = r.a;
+            S.py[lane] = r.b;
+            S.pz[lane] = r.c;
+            S.pm[lane] = r.d;
+          }
         }
         __syncwarp();
         // the self pair is skipped by a zero mass (branch-free, unrolled by 4
         // for independent rsqrt chains)
         const int64_t self = ii - (int64_t)b;
+        if (kF32) {
+          float fx = 0.f, fy = 0.f, fz = 0.f, fphi = 0.f;
 #pragma unroll 4
-        for (uint32_t t = 0; t < nb; ++t) {
-          const bool me = (int64_t)t == self;
-          const double mt = me ? 0.0 : S.pm[t];
-          const double dx = S.px[t] - xi, dy = S.py[t] - yi, dz = S.pz[t] - zi;
-          const double r2 = me ? 1.0 : dx * dx + dy * dy + dz * dz + eps2;  // finite with eps = 0
-          const double ir = rsqrt(r2);
-          const double gm = Gc * mt * ir;
-          const double s3 = gm * ir * ir;
-          ax = fma(s3, dx, ax);
-          ay = fma(s3, dy, ay);
-          az = fma(s3, dz, az);
-          phi -= gm;
+          for (uint32_t t = 0; t < nb; ++t) {
+            const bool me = (int64_t)t == self;
+            const float mt = me ? 0.f : S.pmf[t];
+            const float dx = S.pxf[t] - xf, dy = S.pyf[t] - yf, dz = S.pzf[t] - zf;
+            const float r2 = me ? 1.f : fmaf(dx, dx, fmaf(dy, dy, fmaf(dz, dz, eps2f)));
+            const float ir = rsqrtf(r2);
+            const float gm = Gf * mt * ir;
+            const float s3 = gm * ir * ir;
+            fx = fmaf(s3, dx, fx);
+            fy = fmaf(s3, dy, fy);
+            fz = fmaf(s3, dz, fz);
+            fphi -= gm;
+          }
+          ax += fx;
+          ay += fy;
+          az += fz;
+          phi += fphi;
+        } else {
+#pragma unroll 4
+          for (uint32_t t = 0; t < nb; ++t) {
+            const bool me = (int64_t)t == self;
+            const double mt = me ? 0.0 : S.pm[t];
+            const double dx = S.px[t] - xi, dy = S.py[t] - yi, dz = S.pz[t] - zi;
+            const double r2 = me ? 1.0 : dx * dx + dy * dy + dz * dz + eps2;  // finite with eps = 0
+            const double ir = rsqrt(r2);
+            const double gm = Gc * mt * ir;
+            const double s3 = gm * ir * ir;
+            ax = fma(s3, dx, ax);
+            ay = fma(s3, dy, ay);
+            az = fma(s3, dz, az);
+            phi -= gm;
+          }
         }
       }
     }
@@ -330,7 +411,8 @@ __device__ __forceinline__ void walk_tile(const Fields& F, const GravParams& G, 
     const int ld = __ffs(leaders) - 1;
     leaders &= leaders - 1;
     const uint32_t gm = __shfl_sync(0xffffffffu, peers, ld);
-    walk_group(F, G, S, lane, i, active, ((gm >> lane) & 1u) != 0, ax, ay, az, phi);
+    if (G.fp32) walk_group<true>(F, G, S, lane, i, active, ((gm >> lane) & 1u) != 0, ax, ay, az, phi);
+    else walk_group<false>(F, G, S, lane, i, active, ((gm >> lane) & 1u) != 0, ax, ay, az, phi);
   }
   if (active) {
     F.ax[i] += ax;

@@ -62,6 +62,7 @@ struct DevScalars {
 struct GravParams {
   double G, eps, theta;
   int level;
+  int fp32;  // theta > 0 and !cfg.grav_fp64: fp32 terms, fp64 accumulation
 };
 
 // Turbulence driving (k_stir.cu): the OU state and its inputs, in the arena.

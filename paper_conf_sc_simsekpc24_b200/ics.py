@@ -60,6 +60,7 @@ class StepParams:
     grav_eps: float = 0.01  # Plummer softening length
     grav_theta: float = 0.5  # tree opening angle (0 = direct summation)
     grav_level: int = 6     # leaf level of the gravity octree
+    grav_fp64: int = 0      # 1: fp64 multipole / direct terms also for theta > 0
     gradh: int = 0          # 1: NormalizationGradh, p/(Omega rho^2) in momentum (reading 21)
     dt_vsig: int = 0        # 1: signal-velocity time step (reading 22)
     ve: int = 0             # 1: generalized volume elements X = m/rho0 (reading 23)

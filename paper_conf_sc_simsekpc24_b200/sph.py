@@ -55,7 +55,7 @@ class Config(C.Structure):
         ("stir_steps", C.c_int32), ("divcurl", C.c_int32), ("av_switch", C.c_int32),
         ("gravity", C.c_int32), ("grav_level", C.c_int32), ("grav_G", C.c_double),
         ("grav_eps", C.c_double), ("grav_theta", C.c_double), ("gradh", C.c_int32),
-        ("dt_vsig", C.c_int32), ("ve", C.c_int32), ("reserved", C.c_int32 * 5),
+        ("dt_vsig", C.c_int32), ("ve", C.c_int32), ("grav_fp64", C.c_int32), ("reserved", C.c_int32 * 4),
     ]
 
 
@@ -230,6 +230,7 @@ def config_from_params(params, n_capacity: int, device: int = 0, accounting: int
         c.grav_G = float(params.grav_G)
         c.grav_eps = float(params.grav_eps)
         c.grav_theta = float(params.grav_theta)
+        c.grav_fp64 = int(getattr(params, "grav_fp64", 0))
     return c
 
 
