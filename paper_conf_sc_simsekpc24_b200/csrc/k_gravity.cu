@@ -113,15 +113,19 @@ __global__ void __launch_bounds__(256) grav_up_kernel(Fields F, int l) {
 
 constexpr int kGravThreads = 128;
 constexpr int kGravWarps = kGravThreads / 32;
-constexpr int kGravStack = 64;
+constexpr int kGravPop = 4;     // stack nodes examined per round (8 children each)
+constexpr int kGravStack = 256;
+// per level at most 32 - kGravPop children wait below the top round's 32
+static_assert(kGravStack >= 8 * (32 - kGravPop) + 32, "stack for leaf levels <= 8");
 
 struct GravSmem {
   uint32_t stack[kGravStack];   // parents whose 8 children are still to examine
-  double mom[8][10];            // the accepted children's moments (m, com, Q)
+  double mom[32][10];           // the accepted children's moments (m, com, Q)
   double px[32], py[32], pz[32], pm[32];  // a batch of leaf particles
+  uint32_t leafc[32];           // the leaf cell examined by each lane
   // fp32 terms (GravParams::fp32): moments with the COM relative to the group's
   // centre, and leaf particles relative to it
-  float momf[8][12];            // m, com - o (3), Q (6)
+  float momf[32][12];           // m, com - o (3), Q (6)
   float pxf[32], pyf[32], pzf[32], pmf[32];
 };
 
@@ -225,17 +229,26 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
     __syncwarp();
   }
   while (sp > 0) {
-    const uint32_t e = S.stack[sp - 1];
+    // up to kGravPop nodes from the top of the stack (the smallest first) are
+    // examined together: lane 8g + k takes child k of popped node g (one
+    // memory round trip for up to 32 cells).  With theta = 0 the order of the
+    // direct sums is unchanged: the popped nodes are ascending and no smaller
+    // popped node is shallower than a larger one, so leaves still come in
+    // ascending particle order.
+    const int np = min(sp, kGravPop);
+    const int gq = lane >> 3, kq = lane & 7;
+    const uint32_t e = gq < np ? S.stack[sp - 1 - gq] : 0u;
     __syncwarp();
-    --sp;
-    ++n_pop;
-    const int l = (int)(e >> 28) + 1;                 // the children's level
-    const int64_t c0 = 8 * (int64_t)(e & 0x0fffffffu);  // first child's index at level l
-    const int64_t g0 = grav_level_off(l) + c0;
-    // lanes 0-7: child k = lane
+    sp -= np;
+    n_pop += np;
     bool acc = false, open = false, leaf = false;
-    if (lane < 8) {
-      const Rec4 m0 = ldg4(F.gmom + 3 * (g0 + lane));
+    int l = 0;
+    uint32_t cl = 0;  // the child's index at level l
+    if (gq < np) {
+      l = (int)(e >> 28) + 1;
+      cl = 8u * (e & 0x0fffffffu) + (uint32_t)kq;
+      const int64_t gc = grav_level_off(l) + cl;
+      const Rec4 m0 = ldg4(F.gmom + 3 * gc);
       if (m0.a != 0.0) {
         const double side = Lmax / (double)(1 << l);
         double dd2 = 0;
@@ -247,7 +260,7 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
         }
         if (side * side < th2 * dd2) {
           acc = true;
-          const Rec4 m1 = ldg4(F.gmom + 3 * (g0 + lane) + 1), m2 = ldg4(F.gmom + 3 * (g0 + lane) + 2);
+          const Rec4 m1 = ldg4(F.gmom + 3 * gc + 1), m2 = ldg4(F.gmom + 3 * gc + 2);
           if (kF32) {
             float* q = S.momf[lane];
             q[0] = (float)m0.a;
@@ -261,6 +274,7 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
           }
         } else if (l == Lt) {
           leaf = true;
+          S.leafc[lane] = cl;
         } else {
           open = true;
         }
@@ -274,7 +288,7 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
     // dependency chains: the rsqrt + quadrupole chain is latency-bound)
     n_mp += __popc(am);
     if (kF32) {
-      // this node's (<= 8) multipole terms summed in fp32, then added in fp64
+      // this round's multipole terms summed in fp32, then added in fp64
       float fx = 0.f, fy = 0.f, fz = 0.f, fphi = 0.f, gx = 0.f, gy = 0.f, gz = 0.f, gphi = 0.f;
       uint32_t m = am;
       for (; __popc(m) >= 2; m &= m - 1, m &= m - 1) {
@@ -305,8 +319,7 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
     }
     // leaves, ascending: particles in batches of 32 through shared memory
     for (uint32_t m = lm; m; m &= m - 1) {
-      const int k = __ffs(m) - 1;
-      const int64_t c = c0 + k;
+      const uint32_t c = S.leafc[__ffs(m) - 1];
       const uint32_t s = F.gcell_start[c], en = F.gcell_start[c + 1];
       for (uint32_t b = s; b < en; b += 32) {
         const uint32_t nb = min(32u, en - b);
@@ -368,11 +381,11 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
         }
       }
     }
-    // opened children: push in reverse so they pop in ascending order
+    // opened children: pushed in reverse so they pop in ascending order
     const int no = __popc(om);
-    if (lane < 8 && open) {
+    if (open) {
       const int rank_from_top = __popc(om & ((1u << lane) - 1u));  // 0 for the lowest child
-      S.stack[sp + no - 1 - rank_from_top] = ((uint32_t)l << 28) | (uint32_t)(c0 + lane);
+      S.stack[sp + no - 1 - rank_from_top] = ((uint32_t)l << 28) | cl;
     }
     sp += no;
     __syncwarp();
