@@ -113,6 +113,9 @@ __global__ void __launch_bounds__(256) grav_up_kernel(Fields F, int l) {
 
 constexpr int kGravThreads = 128;
 constexpr int kGravWarps = kGravThreads / 32;
+#ifndef SPH_GRAV_SPEC
+#define SPH_GRAV_SPEC 1  // a child's three moment chunks loaded together
+#endif
 constexpr int kGravPop = 4;     // stack nodes examined per round (8 children each)
 constexpr int kGravStack = 256;
 // per level at most 32 - kGravPop children wait below the top round's 32
@@ -122,7 +125,7 @@ struct GravSmem {
   uint32_t stack[kGravStack];   // parents whose 8 children are still to examine
   double mom[32][10];           // the accepted children's moments (m, com, Q)
   double px[32], py[32], pz[32], pm[32];  // a batch of leaf particles
-  uint32_t leafc[32];           // the leaf cell examined by each lane
+  uint32_t pj[32];              // their particle indices (the self pair)
   // fp32 terms (GravParams::fp32): moments with the COM relative to the group's
   // centre, and leaf particles relative to it
   float momf[32][12];           // m, com - o (3), Q (6)
@@ -244,11 +247,18 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
     bool acc = false, open = false, leaf = false;
     int l = 0;
     uint32_t cl = 0;  // the child's index at level l
+    uint32_t leaf_s = 0, leaf_n = 0;  // a leaf child's particle range
     if (gq < np) {
       l = (int)(e >> 28) + 1;
       cl = 8u * (e & 0x0fffffffu) + (uint32_t)kq;
       const int64_t gc = grav_level_off(l) + cl;
+      // the whole record in one round trip (m1, m2 are needed if accepted)
       const Rec4 m0 = ldg4(F.gmom + 3 * gc);
+      Rec4 m1, m2;
+      if (SPH_GRAV_SPEC) {
+        m1 = ldg4(F.gmom + 3 * gc + 1);
+        m2 = ldg4(F.gmom + 3 * gc + 2);
+      }
       if (m0.a != 0.0) {
         const double side = Lmax / (double)(1 << l);
         double dd2 = 0;
@@ -260,7 +270,10 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
         }
         if (side * side < th2 * dd2) {
           acc = true;
-          const Rec4 m1 = ldg4(F.gmom + 3 * gc + 1), m2 = ldg4(F.gmom + 3 * gc + 2);
+          if (!SPH_GRAV_SPEC) {
+            m1 = ldg4(F.gmom + 3 * gc + 1);
+            m2 = ldg4(F.gmom + 3 * gc + 2);
+          }
           if (kF32) {
             float* q = S.momf[lane];
             q[0] = (float)m0.a;
@@ -274,7 +287,8 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
           }
         } else if (l == Lt) {
           leaf = true;
-          S.leafc[lane] = cl;
+          leaf_s = F.gcell_start[cl];
+          leaf_n = F.gcell_start[cl + 1] - leaf_s;
         } else {
           open = true;
         }
@@ -317,10 +331,96 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
       az += bz;
       phi += bphi;
     }
+    // leaves.  When the round's leaves hold <= 32 particles together (small
+    // leaves: the common case at the default level), their particles are
+    // concatenated in ascending lane (= cell) order and staged as one batch;
+    // otherwise each leaf is streamed in batches of 32 of its own.
+    uint32_t ltotal = 0, loff = 0;
+    if (lm) {
+      loff = leaf_n;  // inclusive prefix over lanes of the leaf sizes
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t v = __shfl_up_sync(0xffffffffu, loff, d);
+        if (lane >= d) loff += v;
+      }
+      ltotal = __shfl_sync(0xffffffffu, loff, 31);
+      loff -= leaf_n;  // exclusive
+    }
+    if (lm && ltotal <= 32u) {
+      const uint32_t total = ltotal, off = loff;
+      n_pp += total;
+      for (uint32_t b0 = 0; b0 < total; b0 += 32) {
+        const uint32_t nb = min(32u, total - b0);
+        const uint32_t g = b0 + (uint32_t)lane;
+        // owner leaf of item g: the leaf lanes are few; each claims its items
+        uint32_t j = 0;
+        for (uint32_t m = lm; m; m &= m - 1) {
+          const int q = __ffs(m) - 1;
+          const uint32_t oq = __shfl_sync(0xffffffffu, off, q), nq = __shfl_sync(0xffffffffu, leaf_n, q),
+                         sq = __shfl_sync(0xffffffffu, leaf_s, q);
+          if (g - oq < nq) j = sq + (g - oq);
+        }
+        __syncwarp();
+        if (g < total) {
+          const Rec4 r = ldg4(F.rec_d + j);
+          S.pj[lane] = j;
+          if (kF32) {
+            S.pxf[lane] = (float)(r.a - ox);
+            S.pyf[lane] = (float)(r.b - oy);
+            S.pzf[lane] = (float)(r.c - oz);
+            S.pmf[lane] = (float)r.d;
+          } else {
+            S.px[lane] = r.a;
+            S.py[lane] = r.b;
+            S.pz[lane] = r.c;
+            S.pm[lane] = r.d;
+          }
+        }
+        __syncwarp();
+        // the self pair is skipped by a zero mass (branch-free, unrolled by 4
+        // for independent rsqrt chains)
+        if (kF32) {
+          float fx = 0.f, fy = 0.f, fz = 0.f, fphi = 0.f;
+#pragma unroll 4
+          for (uint32_t t = 0; t < nb; ++t) {
+            const bool me = (int64_t)S.pj[t] == ii;
+            const float mt = me ? 0.f : S.pmf[t];
+            const float dx = S.pxf[t] - xf, dy = S.pyf[t] - yf, dz = S.pzf[t] - zf;
+            const float r2 = me ? 1.f : fmaf(dx, dx, fmaf(dy, dy, fmaf(dz, dz, eps2f)));
+            const float ir = rsqrtf(r2);
+            const float gm = Gf * mt * ir;
+            const float s3 = gm * ir * ir;
+            fx = fmaf(s3, dx, fx);
+            fy = fmaf(s3, dy, fy);
+            fz = fmaf(s3, dz, fz);
+            fphi -= gm;
+          }
+          ax += fx;
+          ay += fy;
+          az += fz;
+          phi += fphi;
+        } else {
+#pragma unroll 4
+          for (uint32_t t = 0; t < nb; ++t) {
+            const bool me = (int64_t)S.pj[t] == ii;
+            const double mt = me ? 0.0 : S.pm[t];
+            const double dx = S.px[t] - xi, dy = S.py[t] - yi, dz = S.pz[t] - zi;
+            const double r2 = me ? 1.0 : dx * dx + dy * dy + dz * dz + eps2;  // finite with eps = 0
+            const double ir = rsqrt(r2);
+            const double gm = Gc * mt * ir;
+            const double s3 = gm * ir * ir;
+            ax = fma(s3, dx, ax);
+            ay = fma(s3, dy, ay);
+            az = fma(s3, dz, az);
+            phi -= gm;
+          }
+        }
+      }
+    }
     // leaves, ascending: particles in batches of 32 through shared memory
-    for (uint32_t m = lm; m; m &= m - 1) {
-      const uint32_t c = S.leafc[__ffs(m) - 1];
-      const uint32_t s = F.gcell_start[c], en = F.gcell_start[c + 1];
+    for (uint32_t m = ltotal > 32u ? lm : 0u; m; m &= m - 1) {
+      const int q = __ffs(m) - 1;
+      const uint32_t s = __shfl_sync(0xffffffffu, leaf_s, q), en = s + __shfl_sync(0xffffffffu, leaf_n, q);
       for (uint32_t b = s; b < en; b += 32) {
         const uint32_t nb = min(32u, en - b);
         n_pp += nb;
