@@ -242,6 +242,9 @@ __device__ __forceinline__ unsigned long long fma2(unsigned long long a, unsigne
 #ifndef SPH_NBR_RUNSCAN
 #define SPH_NBR_RUNSCAN 1
 #endif
+#ifndef SPH_NBR_DISCARD
+#define SPH_NBR_DISCARD 0  // A/B: DRAM writes 4.51 -> 3.72 GB, time 7.13 -> 7.24 ms
+#endif
 #ifndef SPH_NBR_IMGSKIP
 #define SPH_NBR_IMGSKIP 1
 #endif
@@ -745,6 +748,13 @@ __global__ void __launch_bounds__(kNbrThreads, SPH_NBR_MINB) neighbors_kernel(Fi
         if (k0 + u < len) st_hint(col + (int64_t)(k0 + u) * F.cap, v[u], pol.first);
     }
     __syncwarp();  // the rows are reused by the next tile
+#if SPH_NBR_DISCARD
+    // the rows are dead: drop their (dirty) L2 lines instead of letting them be
+    // written back to DRAM when evicted later (the warp's scratch is nrows_ld
+    // whole 128-B lines)
+    for (int q = lane; q < (int)F.nrows_ld; q += 32)
+      asm volatile("discard.global.L2 [%0], 128;" ::"l"(rows + (int64_t)q * 32) : "memory");
+#endif
 
     // nc statistics (min, max, total) and the capacity flag.
     int mn = active ? cnt : 0x7fffffff, mx = active ? cnt : 0;
