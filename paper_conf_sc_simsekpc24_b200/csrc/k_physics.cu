@@ -25,6 +25,7 @@ namespace sph {
 #define SPH_MOM_DIAG 0
 #endif
 
+
 constexpr double kPi = 3.14159265358979323846;
 constexpr double kPi2Over4 = kPi * kPi / 4.0;
 constexpr double kPi2 = kPi * kPi;
@@ -34,7 +35,10 @@ constexpr double kPi2 = kPi * kPi;
 // (Morton-adjacent) targets, so the gathered records of its warps overlap in L1
 // instead of coming from several distant regions (momentum 11.5 -> 11.0 ms; a
 // persistent contiguous-range grid was slower: spills and tail imbalance).
-constexpr int kDensThreads = 1024;
+#ifndef SPH_DENS_THREADS
+#define SPH_DENS_THREADS 1024  // A/B builds only
+#endif
+constexpr int kDensThreads = SPH_DENS_THREADS;
 constexpr int kIadThreads = 768;
 // A/B builds only: other CTA sizes of momentum-energy
 #ifndef SPH_MOM_THREADS
