@@ -41,7 +41,10 @@ int level_cap_for(const sph_config* c) {
   return std::max(L, 0);
 }
 
-constexpr int kSortSkipDefault = 4;  // LSD passes over digits 4..7 (the top 31 key bits)
+#ifndef SPH_SORT_SKIP
+#define SPH_SORT_SKIP 4  // A/B builds
+#endif
+constexpr int kSortSkipDefault = SPH_SORT_SKIP;  // LSD passes over digits 4..7 (the top 31 key bits)
 constexpr unsigned long long kSortMaxRun = 64;
 
 struct PhaseRow {

@@ -21,7 +21,10 @@ enum StateField { FX = 0, FY, FZ, FVX, FVY, FVZ, FH, FM, FU, FDUM1 };
 
 // Onesweep radix sort geometry (k_sort.cu).
 constexpr int kSortThreads = 256;
-constexpr int kSortKPT = 8;
+#ifndef SPH_SORT_KPT
+#define SPH_SORT_KPT 8  // keys per thread (A/B builds)
+#endif
+constexpr int kSortKPT = SPH_SORT_KPT;
 constexpr int kSortTile = kSortThreads * kSortKPT;  // 2048 keys per tile (3 CTAs/SM)
 constexpr int kRadixBits = 8;
 constexpr int kRadix = 256;
