@@ -198,7 +198,9 @@ typedef struct sph_step_info {
   double dt;                /* the step's dt                                       */
   sph_nbr_stats nbr;
   int32_t cell_level;       /* cell-grid level used by the neighbour search        */
-  int32_t reserved;
+  int32_t graph;            /* 1: the step's phases ran as one CUDA graph launch
+                               (captured at the first step of a buffer parity /
+                               sort pass count / n; env SPH_NO_GRAPH=1 disables) */
   double phase_ms[SPH_NPHASES]; /* CUDA-event time of each phase in this step      */
   int64_t grav_multipoles;  /* diagnostic: multipoles evaluated per warp, summed    */
   int64_t grav_pairs;       /* diagnostic: direct pairs per warp (32 targets), sum */

@@ -131,6 +131,22 @@ struct sph_ctx {
   int64_t compact_scratch_len = 0;
   Stir stir{};          // turbulence driving (k_stir.cu)
   bool stir_on = false;
+  // sph_step as a CUDA graph: one captured step per (buffer parity, sort
+  // passes, n); a replay re-applies the host-side effects the capture recorded
+  struct StepGraph {
+    bool valid = false;
+    int cur = 0, skip = 0;
+    int64_t n = 0;
+    cudaGraphExec_t exec = nullptr;
+    int cur_after = 0;
+    uint32_t* last_perm = nullptr;
+    uint64_t* key_sorted = nullptr;
+    bool gradh_done = false;
+    bool ran[SPH_NPHASES] = {};
+    long long launches = 0;
+  } graphs[4];
+  int graph_next = 0;
+  bool graphs_off = false;  // env SPH_NO_GRAPH, or a capture failed
   // DVFS trace (sph_trace_start / sph_trace_stop)
   struct Trace {
     std::thread th;
@@ -330,6 +346,13 @@ void acct_stop(sph_ctx* c) {
   c->acct.active = false;
 }
 
+cudaError_t record_event(sph_ctx* c, cudaEvent_t ev) {
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  cudaStreamIsCapturing(c->st, &cs);
+  return cs == cudaStreamCaptureStatusActive ? cudaEventRecordWithFlags(ev, c->st, cudaEventRecordExternal)
+                                             : cudaEventRecord(ev, c->st);
+}
+
 int phase_begin(sph_ctx* c, int p) {
   trace_mark(c, p);
   if (c->pending[p]) {
@@ -338,11 +361,13 @@ int phase_begin(sph_ctx* c, int p) {
   }
   apply_clock(c, p);
   c->rows[p].locked = c->current_lock;
-  return cuda_check(c, cudaEventRecord(c->ev[p][0], c->st), "cudaEventRecord");
+  // (External: inside a captured step graph the record is a graph node that
+  // records the event when the graph runs, so the phase times stay valid)
+  return cuda_check(c, record_event(c, c->ev[p][0]), "cudaEventRecord");
 }
 
 int phase_end(sph_ctx* c, int p) {
-  int rc = cuda_check(c, cudaEventRecord(c->ev[p][1], c->st), "phase kernels");
+  int rc = cuda_check(c, record_event(c, c->ev[p][1]), "phase kernels");
   if (rc) return rc;
   trace_mark(c, -1);
   c->pending[p] = true;
@@ -713,6 +738,8 @@ int sph_init(const sph_config* cfg, void* arena, size_t arena_bytes, void* strea
   {
     const char* mr = getenv("SPH_NBR_MERGE_RUNS");  // test hook: exercises the merged-run search path
     c->P.nbr_merge_runs = mr ? atoi(mr) : -1;
+    const char* ng = getenv("SPH_NO_GRAPH");  // sph_step without its CUDA graph
+    c->graphs_off = ng && atoi(ng) != 0;
   }
   layout(cfg, (char*)arena, c);
   for (int p = 0; p < SPH_NPHASES; ++p) {
@@ -727,6 +754,15 @@ int sph_init(const sph_config* cfg, void* arena, size_t arena_bytes, void* strea
         return fail(nullptr, SPH_ERR_CUDA, "cudaEventCreate: %s", cudaGetErrorString(e));
       }
     }
+  }
+  // the arena is the caller's uninitialised memory: every device scalar starts
+  // at zero (accumulators such as the decomposition's red_ord are reset only by
+  // the kernel that consumes them)
+  e = cudaMemsetAsync(c->ds, 0, sizeof(DevScalars), c->st);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    delete c;
+    return fail(nullptr, SPH_ERR_CUDA, "scalar init: %s", cudaGetErrorString(e));
   }
   launch_reset_scalars(c->ds, c->P, c->st);
   set_time_kernel<<<1, 1, 0, c->st>>>(c->ds, 0.0, cfg->dt_first, 1); note_launch();
@@ -756,6 +792,8 @@ void sph_finalize(sph_ctx* c) {
   if (!c->poisoned) cudaStreamSynchronize(c->st);
   for (int p = 0; p < SPH_NPHASES; ++p)
     for (int k = 0; k < 2; ++k) cudaEventDestroy(c->ev[p][k]);
+  for (auto& g : c->graphs)
+    if (g.exec) cudaGraphExecDestroy(g.exec);
   cudaGetLastError();
   delete c;
 }
@@ -1409,9 +1447,9 @@ int sph_step(sph_ctx* c, sph_step_info* info) {
   return rc_step;
 }
 
-static int sph_step_all(sph_ctx* c, sph_step_info* info) {
-  int rc = check_ready(c, S_PART, "sph_step");
-  if (rc) return rc;
+// The phases of one step, enqueued (no synchronisation).
+static int step_body(sph_ctx* c) {
+  int rc;
   if ((rc = body_tree(c))) return rc;
   if ((rc = body_neighbors(c))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_DENSITY, S_DENS))) return rc;
@@ -1422,15 +1460,117 @@ static int sph_step_all(sph_ctx* c, sph_step_info* info) {
   if (c->cfg.gravity && (rc = body_simple(c, SPH_PHASE_GRAVITY, S_MOM))) return rc;
   if (c->stir_on && (rc = body_simple(c, SPH_PHASE_STIR, S_MOM))) return rc;
   if ((rc = body_simple(c, SPH_PHASE_TIMESTEP, S_DT))) return rc;
+  return body_simple(c, SPH_PHASE_UPDATE, S_PART);
+}
+
+// sph_step through a CUDA graph when nothing in the step needs the host between
+// phases (no PHASE accounting, DVFS trace or clock policy): the ~22 launches
+// and events of a step go to the device as one graph launch, so the short
+// phases after the step's synchronisation do not wait on host enqueue.  The
+// graph of a (buffer parity, sort passes, n) is captured from the eager body
+// once; a replay re-applies the host-side state changes recorded then.
+static bool graph_ok(const sph_ctx* c) {
+  return !c->graphs_off && !c->acct.active && !c->trace.active && c->clock_mode == SPH_CLOCK_DEFAULT &&
+         c->P.part == SPH_PART_ALL && !c->rec_m_dirty && c->n > 0;
+}
+
+static int step_graph(sph_ctx* c, bool* used) {
+  *used = false;
+  sph_ctx::StepGraph* g = nullptr;
+  for (auto& x : c->graphs)
+    if (x.valid && x.cur == c->cur && x.skip == c->sort_skip && x.n == c->n) g = &x;
+  if (g) {
+    cudaError_t e = cudaGraphLaunch(g->exec, c->st);
+    if (e != cudaSuccess) return cuda_check(c, e, "cudaGraphLaunch");
+    c->cur = g->cur_after;
+    c->last_perm = g->last_perm;
+    c->key_sorted = g->key_sorted;
+    c->inv_valid = false;
+    c->gradh_done = g->gradh_done;
+    for (int p = 0; p < SPH_NPHASES; ++p)
+      if (g->ran[p]) {
+        c->pending[p] = true;
+        c->rows[p].calls++;
+        c->rows[p].locked = 0;
+      }
+    note_launch((int)g->launches);
+    c->stage = S_PART;
+    *used = true;
+    return SPH_OK;
+  }
+  // capture: the eager body enqueues into the capturing stream (nothing runs)
+  const int cur0 = c->cur, skip0 = c->sort_skip;
+  uint32_t* perm0 = c->last_perm;
+  uint64_t* ks0 = c->key_sorted;
+  const bool inv0 = c->inv_valid, gd0 = c->gradh_done;
+  const int stage0 = c->stage;
+  bool pend0[SPH_NPHASES];
+  int64_t calls0[SPH_NPHASES];
+  for (int p = 0; p < SPH_NPHASES; ++p) pend0[p] = c->pending[p], calls0[p] = c->rows[p].calls;
+  const long long l0 = g_launches.load();
+  auto restore = [&]() {
+    c->cur = cur0;
+    c->last_perm = perm0;
+    c->key_sorted = ks0;
+    c->inv_valid = inv0;
+    c->gradh_done = gd0;
+    c->stage = stage0;
+    for (int p = 0; p < SPH_NPHASES; ++p) c->pending[p] = pend0[p], c->rows[p].calls = calls0[p];
+    c->poisoned = false;
+    c->err[0] = 0;
+    cudaGetLastError();
+    c->graphs_off = true;  // run eagerly from now on
+  };
+  if (cudaStreamBeginCapture(c->st, cudaStreamCaptureModeRelaxed) != cudaSuccess) {
+    restore();
+    return SPH_OK;
+  }
+  const int rc_body = step_body(c);
+  cudaGraph_t graph = nullptr;
+  const cudaError_t e_end = cudaStreamEndCapture(c->st, &graph);
+  cudaGraphExec_t exec = nullptr;
+  if (rc_body || e_end != cudaSuccess || !graph ||
+      cudaGraphInstantiate(&exec, graph, 0) != cudaSuccess) {
+    if (graph) cudaGraphDestroy(graph);
+    restore();
+    return SPH_OK;
+  }
+  cudaGraphDestroy(graph);
+  g = &c->graphs[c->graph_next];
+  c->graph_next = (c->graph_next + 1) % 4;
+  if (g->exec) cudaGraphExecDestroy(g->exec);
+  g->valid = true;
+  g->cur = cur0;
+  g->skip = skip0;
+  g->n = c->n;
+  g->exec = exec;
+  g->cur_after = c->cur;
+  g->last_perm = c->last_perm;
+  g->key_sorted = c->key_sorted;
+  g->gradh_done = c->gradh_done;
+  for (int p = 0; p < SPH_NPHASES; ++p) g->ran[p] = c->rows[p].calls != calls0[p];
+  g->launches = g_launches.load() - l0;
+  const cudaError_t e = cudaGraphLaunch(exec, c->st);
+  if (e != cudaSuccess) return cuda_check(c, e, "cudaGraphLaunch");
+  *used = true;
+  return SPH_OK;
+}
+
+static int sph_step_all(sph_ctx* c, sph_step_info* info) {
+  int rc = check_ready(c, S_PART, "sph_step");
+  if (rc) return rc;
+  bool used = false;
+  if (graph_ok(c) && (rc = step_graph(c, &used))) return rc;
   // A data error (capacity, singular, box) makes the update meaningless: check
   // the device status after the update is enqueued (one sync per step).
-  if ((rc = body_simple(c, SPH_PHASE_UPDATE, S_PART))) return rc;
+  if (!used && (rc = step_body(c))) return rc;
   rc = sync_scalars(c);
   if (info) {
     info->t = c->h_ds.t;
     info->dt = c->h_ds.dt;
     fill_stats(c, &info->nbr);
     info->cell_level = c->h_ds.cell_level;
+    info->graph = used ? 1 : 0;
     for (int p = 0; p < SPH_NPHASES; ++p) info->phase_ms[p] = c->last_ms[p];
     info->grav_multipoles = (int64_t)c->h_ds.grav_mp;
     info->grav_pairs = (int64_t)c->h_ds.grav_pp;

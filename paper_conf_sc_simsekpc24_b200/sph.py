@@ -66,7 +66,7 @@ class NbrStats(C.Structure):
 
 class StepInfo(C.Structure):
     _fields_ = [("t", C.c_double), ("dt", C.c_double), ("nbr", NbrStats),
-                ("cell_level", C.c_int32), ("reserved", C.c_int32),
+                ("cell_level", C.c_int32), ("graph", C.c_int32),
                 ("phase_ms", C.c_double * NPHASES), ("grav_multipoles", C.c_int64),
                 ("grav_pairs", C.c_int64), ("grav_pops", C.c_int64)]
 
@@ -576,7 +576,7 @@ class Simulation:
                 "search_candidates": info.nbr.candidates, "search_passes": info.nbr.passes,
                 "phase_ms": {PHASES[p]: info.phase_ms[p] for p in range(NPHASES)},
                 "grav_multipoles": info.grav_multipoles, "grav_pairs": info.grav_pairs,
-                "grav_pops": info.grav_pops}
+                "grav_pops": info.grav_pops, "graph": bool(info.graph)}
 
     # ---------------------------------------------------------------- energy / clocks
     def set_clock_policy(self, mode: int, mhz=None):

@@ -118,6 +118,34 @@ def test_deterministic_bitwise():
     assert len(hashes) == 1
 
 
+def test_step_graph_matches_eager(monkeypatch):
+    """sph_step replays a captured CUDA graph (one per buffer parity and sort
+    pass count); SPH_NO_GRAPH=1 runs the same phases eagerly.  Both give the
+    same state bit for bit, the same times and neighbour statistics, and the
+    graph path still reports per-phase times and kernel launches."""
+    from paper_conf_sc_simsekpc24_b200 import sph
+    w = ics.turbulence(16)
+    out = {}
+    for env in ("1", "0"):
+        monkeypatch.setenv("SPH_NO_GRAPH", env)
+        sim = new_sim(w)
+        l0 = sph.kernel_launches()
+        infos = [sim.step() for _ in range(5)]
+        launches = sph.kernel_launches() - l0
+        st = sim.get_state()
+        out[env] = (st, sim.get_time(), infos, launches)
+        sim.finalize()
+    (a, ta, ia, la), (b, tb, ib, lb) = out["1"], out["0"]
+    for k in a:
+        assert np.array_equal(a[k], b[k]), k
+    assert ta == tb
+    for x, y in zip(ia, ib):
+        assert x["dt"] == y["dt"] and x["max_nc"] == y["max_nc"] and x["mean_nc"] == y["mean_nc"]
+        assert y["phase_ms"]["neighbors"] > 0 and y["phase_ms"]["momentum_energy"] > 0
+    assert la == lb > 0
+    assert all(x["graph"] for x in ib) and not any(x["graph"] for x in ia)
+
+
 def test_empty_input():
     w = ics.sedov(4)
     from paper_conf_sc_simsekpc24_b200 import sph
