@@ -137,6 +137,9 @@ struct sph_ctx {
     bool valid = false;
     int cur = 0, skip = 0;
     int64_t n = 0;
+    Params P{};          // kernel arguments captured by value: any change -> new capture
+    Stir stir{};
+    bool stir_on = false;
     cudaGraphExec_t exec = nullptr;
     int cur_after = 0;
     uint32_t* last_perm = nullptr;
@@ -1478,7 +1481,9 @@ static int step_graph(sph_ctx* c, bool* used) {
   *used = false;
   sph_ctx::StepGraph* g = nullptr;
   for (auto& x : c->graphs)
-    if (x.valid && x.cur == c->cur && x.skip == c->sort_skip && x.n == c->n) g = &x;
+    if (x.valid && x.cur == c->cur && x.skip == c->sort_skip && x.n == c->n && x.stir_on == c->stir_on &&
+        !memcmp(&x.P, &c->P, sizeof(Params)) && !memcmp(&x.stir, &c->stir, sizeof(Stir)))
+      g = &x;
   if (g) {
     cudaError_t e = cudaGraphLaunch(g->exec, c->st);
     if (e != cudaSuccess) return cuda_check(c, e, "cudaGraphLaunch");
@@ -1543,6 +1548,9 @@ static int step_graph(sph_ctx* c, bool* used) {
   g->cur = cur0;
   g->skip = skip0;
   g->n = c->n;
+  g->P = c->P;
+  g->stir = c->stir;
+  g->stir_on = c->stir_on;
   g->exec = exec;
   g->cur_after = c->cur;
   g->last_perm = c->last_perm;
@@ -1874,6 +1882,7 @@ int sph_stir_init(sph_ctx* c, const sph_stir_params* prm, const double* w, const
   if (!(prm->t_decay > 0) || !(prm->sigma >= 0) || !(prm->sol_weight >= 0 && prm->sol_weight <= 1))
     return fail(c, SPH_ERR_ARG, "need t_decay > 0, sigma >= 0, 0 <= sol_weight <= 1");
   if (mem != SPH_MEM_HOST && mem != SPH_MEM_DEVICE) return fail(c, SPH_ERR_ARG, "mem must be HOST or DEVICE");
+  stir_upload_modes();
   const cudaMemcpyKind k = mem == SPH_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
   const size_t M6 = sizeof(double) * kStirModes * 6;
   rc = cuda_check(c, cudaMemcpyAsync(c->stir.w, w, sizeof(double) * kStirModes, k, c->st), "stir w");

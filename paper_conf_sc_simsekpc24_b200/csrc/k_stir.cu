@@ -133,7 +133,9 @@ __global__ void __launch_bounds__(256) stir_accel_kernel(Fields F, Stir S) {
   F.az[i] += az;
 }
 
-void launch_stir(const Fields& F, const Params& P, const Stir& S, cudaStream_t st) {
+// The mode table in constant memory; called by sph_stir_init (a synchronous
+// copy: never inside a captured step graph).
+void stir_upload_modes() {
   static bool modes_set = false;
   if (!modes_set) {
     int32_t n3[3 * kStirModes];
@@ -141,6 +143,10 @@ void launch_stir(const Fields& F, const Params& P, const Stir& S, cudaStream_t s
     cudaMemcpyToSymbol(c_modes, n3, sizeof(n3));
     modes_set = true;
   }
+}
+
+void launch_stir(const Fields& F, const Params& P, const Stir& S, cudaStream_t st) {
+  stir_upload_modes();  // no-op after sph_stir_init
   (void)P;
   // the box lengths of periodic axes are the configured ones (stirring is for
   // periodic boxes; open axes use the step's box)

@@ -336,6 +336,7 @@ void launch_timestep(const Fields& F, const Params& P, cudaStream_t st);
 void launch_update(const Fields& F, const Params& P, cudaStream_t st);
 void launch_advance_time(const Fields& F, cudaStream_t st);
 void launch_refresh_rec_m(const Fields& F, cudaStream_t st);
+void stir_upload_modes();
 void launch_stir(const Fields& F, const Params& P, const Stir& S, cudaStream_t st);
 void launch_gravity(const Fields& F, const GravParams& G, cudaStream_t st);
 int stir_modes(int32_t* n3);  // host: the fixed mode set (returns kStirModes)

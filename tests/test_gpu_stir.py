@@ -70,3 +70,28 @@ def test_noise_table_exhaustion_is_a_capacity_error():
     with pytest.raises(sph.SphError) as e:
         sim.step()
     assert e.value.name == "ERR_CAPACITY"
+
+
+def test_step_graph_recaptured_when_driving_starts(monkeypatch):
+    """sph_step's CUDA graph holds the kernel arguments of its capture: turning
+    the driving on after two graph steps (new phase, new arguments) must give a
+    new capture, and the run equals the eager one bit for bit."""
+    from paper_conf_sc_simsekpc24_b200 import sph
+    w = ics.turbulence(12)
+    si = ics.stir_inputs(oracle.stir_modes(), 4)
+    out = {}
+    for env in ("1", "0"):
+        monkeypatch.setenv("SPH_NO_GRAPH", env)
+        sim = sph.Simulation(w.params, n_capacity=w.n, stir_steps=4)
+        sim.set_particles({k: np.ascontiguousarray(v) for k, v in w.state.items()})
+        sim.set_time(0.0, w.params.dt_first, True)
+        infos = [sim.step(), sim.step()]
+        sim.stir_init(si.sigma, si.t_decay, si.zeta, si.w, si.noise)
+        infos += [sim.step() for _ in range(3)]
+        out[env] = (sim.get_state(), infos)
+        sim.finalize()
+    (a, ia), (b, ib) = out["1"], out["0"]
+    for k in a:
+        assert np.array_equal(a[k], b[k]), k
+    assert all(x["graph"] for x in ib) and not any(x["graph"] for x in ia)
+    assert all(x["phase_ms"]["stir"] > 0 for x in ib[2:]) and ib[1]["phase_ms"]["stir"] == 0
