@@ -145,6 +145,9 @@ def parse():
                     help="seconds of steps under the NVML DVFS trace (Fig. 9); 0 = off")
     ap.add_argument("--cpu-sample", type=int, default=0, help="oracle targets (0 = auto)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--force-decomp", action="store_true",
+                    help="N = 1: run the decomposed (N > 1) path on a one-rank NCCL group with every "
+                         "collective issued (checks that path on one GPU; not a headline number)")
     ap.add_argument("--out", default=None)
     return ap.parse_args()
 
@@ -516,7 +519,7 @@ def run_reference(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
-def run_decomposed(args, rank, world, local):
+def run_decomposed(args, rank, world, local, forced=False):
     """N > 1: SFC domain decomposition with halo exchange over NCCL (decomp.py),
     weak scaling: turbulence with ~8M particles per GPU in one periodic box
     (nside = round(200 N^(1/3)): 252^3, 317^3, 400^3 at N = 2, 4, 8 -- SURVEY
@@ -533,8 +536,10 @@ def run_decomposed(args, rank, world, local):
     ics.normalise_velocity(w, float(vsq.item()))
     n_total = nside ** 3
     cap = int(1.4 * n_total / world) + 1024
-    ds = decomp.DistributedSim(w.params, w.state, n_capacity=cap, device=local)
+    ds = decomp.DistributedSim(w.params, w.state, n_capacity=cap, device=local,
+                               force_exchange=forced, comm_always=forced)
     del w
+    stream = ds.sim.stream  # every event on the stream the step's kernels run on
 
     def barrier():
         dist.barrier()
@@ -549,10 +554,10 @@ def run_decomposed(args, rank, world, local):
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         barrier()
-        ev0.record()
+        ev0.record(stream)
         for _ in range(args.steps):
             ds.step()
-        ev1.record()
+        ev1.record(stream)
         barrier()
     e_end = ds.sim.energy_counter_mj()
     ms = torch.tensor([ev0.elapsed_time(ev1)], device="cuda")
@@ -566,19 +571,31 @@ def run_decomposed(args, rank, world, local):
     ghosts = torch.tensor([ds.stats["n_ghost"], ds.stats["n_local"]], device="cuda", dtype=torch.float64)
     dist.all_reduce(ghosts)
     launches = sph.kernel_launches() - l0
-    # e2e: each rank's particles copied in from pinned host memory and back out every step
-    host = {k: v.cpu().pin_memory() for k, v in ds.local.items()}
+    # e2e: each rank's particles copied in from pinned host memory and back out
+    # (into pinned buffers of the rank's capacity: the local count varies) every step
+    loc = ds.local
+    nloc = next(iter(loc.values())).shape[0]
+    pinned = {k: torch.empty((cap,), dtype=v.dtype).pin_memory() for k, v in loc.items()}
+    for k, v in loc.items():
+        pinned[k][:nloc].copy_(v)
+    del loc
     h2d = d2h = 0
     barrier()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record()
+    e0.record(stream)
     for _ in range(max(args.e2e_steps, 1)):
-        ds.local = {k: v.to("cuda", non_blocking=True) for k, v in host.items()}
-        h2d = sum(v.numel() * v.element_size() for v in host.values())
+        with torch.cuda.stream(stream):  # the copies in the step's stream order
+            ds.local = {k: v[:nloc].to("cuda", non_blocking=True) for k, v in pinned.items()}
+        h2d = sum(v[:nloc].numel() * v.element_size() for v in pinned.values())
         ds.step()
-        host = {k: v.to("cpu") for k, v in ds.local.items()}
-        d2h = sum(v.numel() * v.element_size() for v in host.values())
-    e1.record()
+        with torch.cuda.stream(stream):
+            loc = ds.local
+            nloc = next(iter(loc.values())).shape[0]
+            for k, v in loc.items():
+                pinned[k][:nloc].copy_(v, non_blocking=True)
+        stream.synchronize()
+        d2h = sum(v[:nloc].numel() * v.element_size() for v in pinned.values())
+    e1.record(stream)
     barrier()
     ems = torch.tensor([e0.elapsed_time(e1)], device="cuda")
     dist.all_reduce(ems, op=dist.ReduceOp.MAX)
@@ -589,7 +606,8 @@ def run_decomposed(args, rank, world, local):
                 "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
                 "config": {"workload": f"turbulence{nside}", "n_particles_total": n_total,
                            "n_particles_per_gpu": n_total / world,
-                           "parallelism": f"SFC domain decomposition over {world} GPUs, halo exchange ({dist.get_backend().upper()})",
+                           "parallelism": (f"SFC domain decomposition over {world} GPUs, halo exchange ({dist.get_backend().upper()})"
+                                           + (" -- forced at N = 1: every collective issued on a one-rank group" if forced else "")),
                            "ghost_fraction": float(ghosts[0] / ghosts[1]),
                            "l2": "inputs >> 126 MB L2; no flush"},
                 "phase_ms_rank0": phase_ms, "roofline": None,
@@ -614,6 +632,14 @@ def main():
     import torch.distributed as dist
     from paper_conf_sc_simsekpc24_b200 import sph
 
+    if world == 1 and args.force_decomp:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29511")
+        os.environ.setdefault("RANK", "0")
+        os.environ.setdefault("WORLD_SIZE", "1")
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", init_method="env://", device_id=torch.device("cuda", local))
+        return run_decomposed(args, rank, world, local, forced=True)
     if world > 1:
         # SPH_DIST_BACKEND=gloo lets several ranks share one GPU (tests); NCCL otherwise
         backend = os.environ.get("SPH_DIST_BACKEND", "nccl")

@@ -51,16 +51,21 @@ ROW = 11        # SPH_ROW_DOUBLES
 class Comm:
     """Collectives over the default process group; host tensors for gloo."""
 
-    def __init__(self):
+    def __init__(self, always: bool = False):
         self.rank = dist.get_rank() if dist.is_initialized() else 0
-        self.world = dist.get_world_size() if dist.is_initialized() else 1
+        world = dist.get_world_size() if dist.is_initialized() else 1
         self.host = (dist.get_backend() == "gloo") if dist.is_initialized() else True
+        # always: issue the collectives even on a one-rank group (exercises the
+        # NCCL data plane on a single GPU); `world` below is then the routing's
+        # world, and the short cuts test `self.world == 1` through `_local`
+        self.world = world
+        self._local = world == 1 and not (always and dist.is_initialized())
 
     def _to(self, t):
         return t.cpu() if self.host else t
 
     def all_reduce(self, t, op):
-        if self.world == 1:
+        if self._local:
             return t
         x = self._to(t.clone())
         dist.all_reduce(x, op=op)
@@ -68,7 +73,7 @@ class Comm:
 
     def all_reduce_(self, t, op):
         """In-place all-reduce of a device tensor (gloo: through a host copy)."""
-        if self.world == 1:
+        if self._local:
             return t
         if self.host:
             x = t.cpu()
@@ -81,7 +86,7 @@ class Comm:
     def all_to_all(self, recv, send, recv_counts, send_counts):
         """Rows send[sum send_counts, ...] -> recv[sum recv_counts, ...] (dim-0
         splits known on the host: no count exchange here)."""
-        if self.world == 1:
+        if self._local:
             if recv.numel():
                 recv.copy_(send)
             return recv
@@ -99,7 +104,7 @@ class Comm:
         """all_to_all that overlaps the caller's next kernels (NCCL: async on its
         own stream; all_to_all_finish makes the current stream wait).  gloo and
         world 1: completes here."""
-        if self.world == 1 or self.host:
+        if self._local or self.host:
             self.all_to_all(recv, send, recv_counts, send_counts)
             return None
         return dist.all_to_all_single(recv, send.contiguous(), [int(c) for c in recv_counts],
@@ -111,7 +116,7 @@ class Comm:
             work.wait()
 
     def all_gather(self, t):
-        if self.world == 1:
+        if self._local:
             return [t]
         x = self._to(t.contiguous())
         out = [torch.empty_like(x) for _ in range(self.world)]
@@ -120,7 +125,7 @@ class Comm:
 
     def alltoallv(self, parts):
         """parts[r]: tensor [n_r, ...] for rank r -> list of received [m_s, ...]."""
-        if self.world == 1:
+        if self._local:
             return [parts[0]]
         dev = parts[0].device
         tail = tuple(parts[0].shape[1:])
@@ -175,7 +180,7 @@ class DistributedSim:
         # overlap the H2 / H3 halos with the interior targets (not with grad-h / VE)
         self.overlap = kw.pop("overlap", True) and not (getattr(params, "gradh", 0) or getattr(params, "ve", 0))
         self.params = params
-        self.comm = Comm()
+        self.comm = Comm(always=kw.pop("comm_always", False))
         self.dev = torch.device("cuda", device)
         self.sim = sph.Simulation(params, n_capacity=n_capacity, device=device, **kw)
         self.box_len = [float(b - a) for a, b in zip(params.box_min, params.box_max)]
