@@ -763,17 +763,28 @@ def main():
     # --- e2e: same metric through the C ABI with host buffers ---
     # Every step copies its input state in from pinned host memory
     # (sph_set_particles) and reads the updated state back (sph_get_field x 11).
-    # Two contexts alternate so that step s+1's input copy and step s's
-    # read-back run on the copy engines while step s / s+1 compute (what a
-    # production loop with asynchronous I/O does; PCIe 704 MB each way per
-    # step at 8M).  The sequential variant (copy in, step, copy out, no
-    # overlap) is reported beside it.
+    # Two contexts alternate: step s+1's input is copied from pinned host
+    # memory (H2D) on a copy stream into a device staging buffer while step s
+    # computes and step s-1's read-back (D2H, sph_get_field async) runs on the
+    # other context's stream; sph_set_particles then moves the staged input in
+    # on that context's stream (device to device).  Both copy directions and the
+    # compute overlap (what a production loop with asynchronous I/O does; 704 MB
+    # each way per step at 8M, the host link does ~78 GB/s both ways together,
+    # tools/link_probe.py).  With the H2D on the context's own stream it queued
+    # behind that stream's D2H (~26.6 ms of serial copies per 24.4 ms step).
+    # The sequential variant (copy in, step, copy out, no overlap) is reported
+    # beside it.
     e2e = None
     if args.e2e_steps > 0:
         pinned = {k: torch.from_numpy(v).pin_memory() for k, v in sim.get_state().items()}
         h2d = sum(v.numel() * v.element_size() for v in pinned.values())
         d2h = h2d
-        sims = [sim, sph.Simulation(w.params, n_capacity=n, device=local)]
+        NCTX = 2
+        sims = [sim] + [sph.Simulation(w.params, n_capacity=n, device=local) for _ in range(NCTX - 1)]
+        copy_stream = torch.cuda.Stream(device=local)
+        stage = [{k: torch.empty(v.shape, dtype=v.dtype, device=f"cuda:{local}") for k, v in pinned.items()}
+                 for _ in sims]
+        staged = [torch.cuda.Event() for _ in sims]  # stage[c] consumed by context c
         t_now, dtp, first = sim.get_time()
         for sm in sims:
             sm.set_time(t_now, dtp, first)
@@ -797,15 +808,24 @@ def main():
                 dist.all_reduce(t, op=dist.ReduceOp.MAX)
             return float(t.item())
 
+        def load(c):
+            """H2D of the input into stage[c] on the copy stream, then into context c."""
+            copy_stream.wait_event(staged[c])
+            with torch.cuda.stream(copy_stream):
+                for k, v in pinned.items():
+                    stage[c][k].copy_(v, non_blocking=True)
+                sims[c].set_particles(stage[c])  # its stream waits for the copy stream
+            staged[c].record(sims[c].stream)
+
         def pipelined():
             K = args.e2e_steps
-            sims[0].set_particles(pinned)
+            load(0)
             for s_ in range(K):
-                cur, nxt = sims[s_ % 2], sims[(s_ + 1) % 2]
+                cur = sims[s_ % NCTX]
                 if s_ + 1 < K:
-                    nxt.set_particles(pinned)          # step s+1's input, on nxt's stream
+                    load((s_ + 1) % NCTX)             # step s+1's input
                 cur.step()                             # host waits for this step only
-                for k, v in outs[s_ % 2].items():
+                for k, v in outs[s_ % NCTX].items():
                     cur.get_field(k, out=v, async_=True)  # read-back overlaps the next step
             for sm in sims:
                 sm.sync()
@@ -817,13 +837,16 @@ def main():
                 for k, v in outs[0].items():
                     sim.get_field(k, out=v)
 
+        pipelined()  # untimed: each context's first steps capture its step graphs
         ms_pipe = timed(pipelined)
         ms_seq = timed(sequential)
-        sims[1].finalize()
+        for sm in sims[1:]:
+            sm.finalize()
         e2e = {"value": n * world * args.e2e_steps / (ms_pipe * 1e-3), "unit": UNIT,
                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-               "path": ("two libsph contexts alternating: sph_set_particles(pinned host) of step s+1 and "
-                        "sph_get_field x11 (pinned host, SPH_MEM_HOST_ASYNC) of step s overlap sph_step"),
+               "path": ("two libsph contexts alternating: step s+1's input H2D from pinned host (copy stream, "
+                        "then sph_set_particles device-to-device) and step s-1's sph_get_field x11 (pinned host, "
+                        "SPH_MEM_HOST_ASYNC) overlap sph_step of step s"),
                "sequential": {"value": n * world * args.e2e_steps / (ms_seq * 1e-3),
                               "path": "sph_set_particles(pinned host) + sph_step + sph_get_field x11 (host), no overlap"}}
 
