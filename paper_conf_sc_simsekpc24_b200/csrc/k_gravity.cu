@@ -128,7 +128,10 @@ struct GravSmem {
   uint32_t pj[32];              // their particle indices (the self pair)
   // fp32 terms (GravParams::fp32): moments with the COM relative to the group's
   // centre, and leaf particles relative to it
-  float momf[32][12];           // m, com - o (3), Q (6)
+  // fp32 terms: the accepted children's m, com - o (3), Q (6), compacted in
+  // rank order and interleaved by pairs: momp[r / 2][field][r % 2] (one
+  // 64-bit load = a field of two cells)
+  float momp[16][10][2];
   float pxf[32], pyf[32], pzf[32], pmf[32];
 };
 
@@ -171,6 +174,38 @@ __device__ __forceinline__ void add_multipole_f(const float* q, float xf, float 
   phi -= fmaf(0.5f * rQr, gi5, Gc * q[0] * ir);
 }
 
+// Two multipoles per instruction (packed f32x2, FFMA2 / FMUL2): q2 holds the
+// fields of cells a (low half) and b (high half); the sums go to packed
+// accumulators (low: a's, high: b's).  Same operations as add_multipole_f.
+__device__ __forceinline__ void add_multipole_f2(const float (*q2)[2], unsigned long long xf2,
+                                                 unsigned long long yf2, unsigned long long zf2,
+                                                 unsigned long long G2, unsigned long long& ax,
+                                                 unsigned long long& ay, unsigned long long& az,
+                                                 unsigned long long& phi) {
+  auto ld = [&](int k) { return *reinterpret_cast<const unsigned long long*>(q2[k]); };
+  const unsigned long long m = ld(0);
+  const unsigned long long rx = sub2(xf2, ld(1)), ry = sub2(yf2, ld(2)), rz = sub2(zf2, ld(3));
+  const unsigned long long r2 = fma2(rx, rx, fma2(ry, ry, mul2(rz, rz)));
+  float r2a, r2b;
+  unpack2(r2, r2a, r2b);
+  const unsigned long long ir = pack2(rsqrtf(r2a), rsqrtf(r2b));
+  const unsigned long long ir2 = mul2(ir, ir), ir3 = mul2(ir, ir2), ir5 = mul2(ir3, ir2);
+  const unsigned long long q4 = ld(4), q5 = ld(5), q6 = ld(6), q7 = ld(7), q8 = ld(8), q9 = ld(9);
+  const unsigned long long Qx = fma2(q4, rx, fma2(q5, ry, mul2(q6, rz)));
+  const unsigned long long Qy = fma2(q5, rx, fma2(q7, ry, mul2(q8, rz)));
+  const unsigned long long Qz = fma2(q6, rx, fma2(q8, ry, mul2(q9, rz)));
+  const unsigned long long rQr = fma2(rx, Qx, fma2(ry, Qy, mul2(rz, Qz)));
+  const unsigned long long gi5 = mul2(G2, ir5);
+  const unsigned long long Gm = mul2(G2, m);
+  // s = -G m ir3 - 2.5 rQr gi5 ir2
+  const unsigned long long s = fma2(mul2(splat2(-2.5f), rQr), mul2(gi5, ir2), mul2(splat2(-1.f), mul2(Gm, ir3)));
+  ax = fma2(s, rx, fma2(gi5, Qx, ax));
+  ay = fma2(s, ry, fma2(gi5, Qy, ay));
+  az = fma2(s, rz, fma2(gi5, Qz, az));
+  // phi -= 0.5 rQr gi5 + G m ir
+  phi = sub2(phi, fma2(mul2(splat2(0.5f), rQr), gi5, mul2(Gm, ir)));
+}
+
 // One warp per 32 consecutive targets.  The stack holds parents; popping one
 // examines its 8 children together (lanes 0-7 load and classify one child each:
 // one memory round trip per 8 cells instead of 8 dependent ones): accepted
@@ -208,6 +243,7 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
   const double ox = 0.5 * (lo[0] + hi[0]), oy = 0.5 * (lo[1] + hi[1]), oz = 0.5 * (lo[2] + hi[2]);
   const float xf = (float)(xi - ox), yf = (float)(yi - oy), zf = (float)(zi - oz);
   const float Gf = (float)Gc, eps2f = (float)eps2;
+  const unsigned long long xf2 = splat2(xf), yf2 = splat2(yf), zf2 = splat2(zf), G2 = splat2(Gf);
 
   // the root itself: accepted, a leaf (Lt = 0 is not allowed) or opened
   int sp = 0;
@@ -248,6 +284,7 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
     int l = 0;
     uint32_t cl = 0;  // the child's index at level l
     uint32_t leaf_s = 0, leaf_n = 0;  // a leaf child's particle range
+    float qf[10];                     // an accepted child's moments (fp32 terms)
     if (gq < np) {
       l = (int)(e >> 28) + 1;
       cl = 8u * (e & 0x0fffffffu) + (uint32_t)kq;
@@ -275,11 +312,10 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
             m2 = ldg4(F.gmom + 3 * gc + 2);
           }
           if (kF32) {
-            float* q = S.momf[lane];
-            q[0] = (float)m0.a;
-            q[1] = (float)(m0.b - ox); q[2] = (float)(m0.c - oy); q[3] = (float)(m0.d - oz);
-            q[4] = (float)m1.a; q[5] = (float)m1.b; q[6] = (float)m1.c; q[7] = (float)m1.d;
-            q[8] = (float)m2.a; q[9] = (float)m2.b;
+            qf[0] = (float)m0.a;
+            qf[1] = (float)(m0.b - ox); qf[2] = (float)(m0.c - oy); qf[3] = (float)(m0.d - oz);
+            qf[4] = (float)m1.a; qf[5] = (float)m1.b; qf[6] = (float)m1.c; qf[7] = (float)m1.d;
+            qf[8] = (float)m2.a; qf[9] = (float)m2.b;
           } else {
             double* q = S.mom[lane];
             q[0] = m0.a; q[1] = m0.b; q[2] = m0.c; q[3] = m0.d;
@@ -297,25 +333,37 @@ __device__ __forceinline__ void walk_group(const Fields& F, const GravParams& G,
     const uint32_t am = __ballot_sync(0xffffffffu, acc);
     const uint32_t lm = __ballot_sync(0xffffffffu, leaf);
     const uint32_t om = __ballot_sync(0xffffffffu, open);
+    if (kF32 && acc) {
+      const int r = __popc(am & ((1u << lane) - 1u));  // rank among the accepted
+#pragma unroll
+      for (int f = 0; f < 10; ++f) S.momp[r >> 1][f][r & 1] = qf[f];
+    }
     __syncwarp();
     // multipoles, two at a time into separate accumulators (independent
     // dependency chains: the rsqrt + quadrupole chain is latency-bound)
     n_mp += __popc(am);
     if (kF32) {
-      // this round's multipole terms summed in fp32, then added in fp64
-      float fx = 0.f, fy = 0.f, fz = 0.f, fphi = 0.f, gx = 0.f, gy = 0.f, gz = 0.f, gphi = 0.f;
-      uint32_t m = am;
-      for (; __popc(m) >= 2; m &= m - 1, m &= m - 1) {
-        const int k0 = __ffs(m) - 1;
-        const int k1 = __ffs(m & (m - 1)) - 1;
-        add_multipole_f(S.momf[k0], xf, yf, zf, Gf, fx, fy, fz, fphi);
-        add_multipole_f(S.momf[k1], xf, yf, zf, Gf, gx, gy, gz, gphi);
+      // this round's multipole terms, two cells per packed instruction, summed
+      // in fp32, then added in fp64 (an odd last cell pairs with a zero-mass,
+      // zero-Q slot: its terms are exactly 0)
+      const int na = __popc(am);
+      if (na & 1) {
+        // far away (r^2 ~ 1e36 stays finite), no mass, no Q: every term is 0
+        if (lane < 10) S.momp[na >> 1][lane][1] = lane >= 1 && lane <= 3 ? 1e18f : 0.f;
+        __syncwarp();
       }
-      if (m) add_multipole_f(S.momf[__ffs(m) - 1], xf, yf, zf, Gf, fx, fy, fz, fphi);
-      ax += (double)fx + (double)gx;
-      ay += (double)fy + (double)gy;
-      az += (double)fz + (double)gz;
-      phi += (double)fphi + (double)gphi;
+      unsigned long long fx = 0ull, fy = 0ull, fz = 0ull, fphi = 0ull;
+      for (int r = 0; r < na; r += 2)
+        add_multipole_f2(S.momp[r >> 1], xf2, yf2, zf2, G2, fx, fy, fz, fphi);
+      float a0, a1;
+      unpack2(fx, a0, a1);
+      ax += (double)a0 + (double)a1;
+      unpack2(fy, a0, a1);
+      ay += (double)a0 + (double)a1;
+      unpack2(fz, a0, a1);
+      az += (double)a0 + (double)a1;
+      unpack2(fphi, a0, a1);
+      phi += (double)a0 + (double)a1;
     } else {
       double bx = 0, by = 0, bz = 0, bphi = 0;
       uint32_t m = am;

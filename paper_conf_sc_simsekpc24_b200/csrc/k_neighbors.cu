@@ -205,32 +205,7 @@ __device__ __forceinline__ void slab_d2(const Box& B, const Target& t, int a, in
   d1 = a1 * a1;
 }
 
-// Packed fp32x2 arithmetic (FADD2/FMUL2/FFMA2 on sm_100a): two candidates per
-// instruction in the neighbour test.  Each lane is IEEE round-to-nearest.
-__device__ __forceinline__ unsigned long long pack2(float lo, float hi) {
-  return ((unsigned long long)__float_as_uint(hi) << 32) | (unsigned long long)__float_as_uint(lo);
-}
-__device__ __forceinline__ void unpack2(unsigned long long v, float& lo, float& hi) {
-  lo = __uint_as_float((uint32_t)v);
-  hi = __uint_as_float((uint32_t)(v >> 32));
-}
-__device__ __forceinline__ unsigned long long sub2(unsigned long long a, unsigned long long b) {
-  unsigned long long d;
-  asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
-  return d;
-}
-__device__ __forceinline__ unsigned long long mul2(unsigned long long a, unsigned long long b) {
-  unsigned long long d;
-  asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
-  return d;
-}
-__device__ __forceinline__ unsigned long long fma2(unsigned long long a, unsigned long long b,
-                                                   unsigned long long c) {
-  unsigned long long d;
-  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
-  return d;
-}
-
+// Packed fp32x2 arithmetic: pack2 / sub2 / mul2 / fma2 (sph_internal.cuh).
 
 // Run table size.  A cell contributes up to 4 runs of needed children; when the
 // group's runs would exceed kMaxRuns, each cell's needed children are merged into
