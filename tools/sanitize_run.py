@@ -55,6 +55,15 @@ sim.step()
 sim.finalize()
 w = ics.evrard(12)
 run(w, steps=1).finalize()
+w = ics.evrard(12)
+w.params = dataclasses.replace(w.params, grav_fp64=1)   # fp64 gravity terms
+run(w, steps=1).finalize()
+# search: coarse grid (multi-chunk streams, "full" periodic axes) and the
+# merged-run path of the run table
+run(ics.turbulence(12), steps=2, max_cell_level=2).finalize()
+os.environ["SPH_NBR_MERGE_RUNS"] = "0"
+run(ics.random_box(3000, seed=5, periodic=False), steps=2).finalize()
+del os.environ["SPH_NBR_MERGE_RUNS"]
 w = ics.sedov(14)
 w.params = dataclasses.replace(w.params, av_switch=1)
 ds = decomp.DistributedSim(w.params, w.state, n_capacity=w.n, device=0, force_exchange=True)
