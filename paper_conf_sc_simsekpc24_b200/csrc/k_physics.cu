@@ -39,7 +39,10 @@ constexpr double kPi2 = kPi * kPi;
 #define SPH_DENS_THREADS 1024  // A/B builds only
 #endif
 constexpr int kDensThreads = SPH_DENS_THREADS;
-constexpr int kIadThreads = 768;
+#ifndef SPH_IAD_THREADS
+#define SPH_IAD_THREADS 768  // A/B builds only
+#endif
+constexpr int kIadThreads = SPH_IAD_THREADS;
 // A/B builds only: other CTA sizes of momentum-energy
 #ifndef SPH_MOM_THREADS
 #define SPH_MOM_THREADS 512
