@@ -123,7 +123,9 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--workload", default="turbulence200")
     ap.add_argument("--impl", default="libsph", choices=["libsph", "reference"])
-    ap.add_argument("--e2e-steps", type=int, default=10)
+    # (the pipelined e2e loop's fill -- the first input copy -- and drain -- the
+    # last read-back -- are inside its timed region: 40 steps amortise them)
+    ap.add_argument("--e2e-steps", type=int, default=40)
     ap.add_argument("--energy-seconds", type=float, default=10.0,
                     help="length of each energy window (the NVML counter ticks every ~100 ms / "
                          "~99 J on a B200: >= 10 s keeps a window within ~1%%); 0 = no energy")
