@@ -86,6 +86,30 @@ def test_sedov_blast_radius(golden):
     assert rho[top].mean() > 2.0
 
 
+def test_sedov_radius_converges_at_100():
+    """Sedov 100^3 (configs[1]'s workload) to t = 0.05: the shock radius is within
+    3% of the similarity solution (40^3: -2.3%, 100^3: -1.7%, 200^3: -0.6%,
+    profiles/r02_sedov_convergence.json) and the shell compression exceeds 3
+    (strong-shock limit 4)."""
+    from paper_conf_sc_simsekpc24_b200 import sph
+    w = ics.sedov(100)
+    sim = sph.Simulation(w.params, n_capacity=w.n)
+    sim.set_particles({k: np.ascontiguousarray(v) for k, v in w.state.items()})
+    sim.set_time(0.0, w.params.dt_first, True)
+    t, steps = 0.0, 0
+    while t < 0.05 and steps < 2000:
+        t = sim.step()["t"]
+        steps += 1
+    st = sim.get_state()
+    rho = sim.get_field("rho")
+    sim.finalize()
+    r = np.sqrt(st["x"] ** 2 + st["y"] ** 2 + st["z"] ** 2)
+    top = np.argsort(rho)[-int(0.003 * w.n):]
+    R_th = 1.1517 * (t * t) ** 0.2
+    assert abs(float(np.median(r[top])) - R_th) / R_th < 0.03
+    assert rho[top].mean() > 3.0
+
+
 def test_noh_implosion_jumps():
     """Noh (SURVEY 8(c) pin 'Noh'; config 4's workload, 80^3 lattice, open box):
     at t = 0.3 the pre-shock gas follows rho = (1 + t/r)^2 with v_r = -1, the
