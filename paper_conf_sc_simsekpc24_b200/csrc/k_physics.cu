@@ -471,7 +471,10 @@ __device__ __forceinline__ void iad_dc_body(const Fields& F, const Params& P, co
 
 // 512 threads x 128 registers (640 x 102 spills with the two-pair loop;
 // one pair per iteration: 512 -> 6.02, 640 -> 5.53 ms; two pairs at 512: 4.78)
-constexpr int kIadDcThreads = 512;
+#ifndef SPH_IADDC_THREADS
+#define SPH_IADDC_THREADS 512  // A/B builds only
+#endif
+constexpr int kIadDcThreads = SPH_IADDC_THREADS;
 __global__ void __launch_bounds__(kIadDcThreads, 1) iad_dc_kernel(Fields F, Params P) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= F.n) return;
