@@ -20,31 +20,43 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 FIELDS = ("id", "x", "y", "z", "vx", "vy", "vz", "h", "u", "du_m1")
 
 
-def _make(name):
+def _make(name, rank=0, world=1, vsq=None):
+    """The whole initial state (rank 0 of 1) or rank's slice of it.  Turbulence
+    slices come from ics.turbulence_part (no rank generates the whole box) and
+    every run normalises with the same given sum of v^2, so the slices are
+    bit-identical to the single run's particles."""
     import dataclasses
     from paper_conf_sc_simsekpc24_b200 import ics
     if name.startswith("noh"):
         w = ics.noh(int(name[3:]))
         w.params = dataclasses.replace(w.params, ngmax=256)  # capacity for the shocked shell
+        if world > 1:
+            w.state = {k: np.ascontiguousarray(v[rank::world]) for k, v in w.state.items()}
     else:
-        w = ics.turbulence(int(name[len("turbulence"):]))
+        w = ics.turbulence_part(int(name[len("turbulence"):]), rank, world)
+        ics.normalise_velocity(w, vsq)
     return w
 
 
-def _worker(rank, world, port, name, steps, out):
+def _vsq(name):
+    from paper_conf_sc_simsekpc24_b200 import ics
+    if name.startswith("noh"):
+        return None
+    return ics.turbulence_part(int(name[len("turbulence"):]), 0, 1).meta["vsq_sum"]
+
+
+def _worker(rank, world, port, name, steps, out, vsq):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     import torch
     import torch.distributed as dist
     dist.init_process_group("gloo", rank=rank, world_size=world)
     from paper_conf_sc_simsekpc24_b200 import decomp
-    w = _make(name)
-    n = w.n
-    mine = {k: np.ascontiguousarray(v[rank::world]) for k, v in w.state.items()}
-    del w
+    w = _make(name, rank, world, vsq)
+    n = w.meta.get("n_total", w.n * world)
     cap = int(1.4 * n / world) + 4096
-    ds = decomp.DistributedSim(_make_params(name), mine, n_capacity=cap, device=0)
-    del mine
+    ds = decomp.DistributedSim(w.params, w.state, n_capacity=cap, device=0)
+    del w
     ms = []
     dts = []
     for _ in range(steps):
@@ -54,22 +66,20 @@ def _worker(rank, world, port, name, steps, out):
         dts.append(ds.step())
         torch.cuda.synchronize()
         ms.append(1e3 * (time.perf_counter() - t0))
-    st = ds.gather_state()
-    if rank == 0:
-        np.savez(out, **{k: st[k] for k in FIELDS}, dts=np.array(dts), ms=np.array(ms),
-                 n_ghost=ds.stats["n_ghost"], n_local=ds.stats["n_local"])
+    # every rank writes its own particles (an all-gather of the whole state to
+    # every rank does not fit when 8 ranks share one GPU); the parent merges
+    with torch.cuda.stream(ds.sim.stream):
+        loc = {k: v.cpu().numpy() for k, v in ds.local.items()}
+    np.savez(f"{out}.{rank}.npz", **{k: loc[k] for k in FIELDS}, dts=np.array(dts), ms=np.array(ms),
+             n_ghost=ds.stats["n_ghost"], n_local=ds.stats["n_local"])
     dist.barrier()
     dist.destroy_process_group()
 
 
-def _make_params(name):
-    return _make(name).params
-
-
-def _single(name, steps):
+def _single(name, steps, vsq):
     import torch
     from paper_conf_sc_simsekpc24_b200 import sph
-    w = _make(name)
+    w = _make(name, 0, 1, vsq)
     sim = sph.Simulation(w.params, n_capacity=w.n)
     sim.set_particles({k: np.ascontiguousarray(v) for k, v in w.state.items()})
     sim.set_time(0.0, w.params.dt_first, True)
@@ -98,10 +108,11 @@ def main():
     s.bind(("127.0.0.1", 0))
     port = s.getsockname()[1]
     s.close()
-    tmp = f"/tmp/decomp_fullsize_{os.getpid()}.npz"
+    vsq = _vsq(a.workload)
+    tmp = f"/tmp/decomp_fullsize_{os.getpid()}"
     ctx = mp.get_context("spawn")
     t0 = time.perf_counter()
-    procs = [ctx.Process(target=_worker, args=(r, a.world, port, a.workload, a.steps, tmp)) for r in range(a.world)]
+    procs = [ctx.Process(target=_worker, args=(r, a.world, port, a.workload, a.steps, tmp, vsq)) for r in range(a.world)]
     for p in procs:
         p.start()
     for p in procs:
@@ -110,8 +121,15 @@ def main():
     if bad:
         raise SystemExit(f"rank exit codes {bad}")
     t_dec = time.perf_counter() - t0
-    d = np.load(tmp)
-    dts1, ms1, st1 = _single(a.workload, a.steps)
+    parts = [dict(np.load(f"{tmp}.{r}.npz")) for r in range(a.world)]
+    for r in range(a.world):
+        os.remove(f"{tmp}.{r}.npz")
+    d = {k: np.concatenate([p[k] for p in parts]) for k in FIELDS}
+    o = np.argsort(d["id"])
+    d = {k: v[o] for k, v in d.items()}
+    d.update({k: parts[0][k] for k in ("dts", "ms", "n_ghost", "n_local")})
+    del parts
+    dts1, ms1, st1 = _single(a.workload, a.steps, vsq)
     same = {k: bool(np.array_equal(d[k], st1[k])) for k in FIELDS}
     rec = {"workload": a.workload, "n": int(st1["id"].size), "world": a.world, "steps": a.steps,
            "backend": "gloo (all ranks on cuda:0)",
@@ -120,7 +138,6 @@ def main():
            "rank0_ghosts": int(d["n_ghost"]), "rank0_local": int(d["n_local"]),
            "ms_per_step_decomposed_wall": d["ms"].tolist(), "ms_per_step_single_wall": ms1,
            "decomposed_run_wall_s": t_dec}
-    os.remove(tmp)
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     with open(a.out, "w") as f:
         json.dump(rec, f, indent=1)
