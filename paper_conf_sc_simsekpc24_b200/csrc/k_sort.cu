@@ -129,8 +129,12 @@ struct SortSmem {
   uint32_t tile;
 };
 
+// Resident CTAs per SM requested from the register allocator (A/B builds).
+#ifndef SPH_SORT_MINB
+#define SPH_SORT_MINB 4  // 4 x 256 threads: <= 64 registers, no spills (3 -> 4 CTAs per SM)
+#endif
 template <bool kFirst>
-__global__ void __launch_bounds__(kSortThreads) onesweep_kernel(
+__global__ void __launch_bounds__(kSortThreads, SPH_SORT_MINB) onesweep_kernel(
     const uint64_t* __restrict__ kin, const uint32_t* __restrict__ vin, uint64_t* __restrict__ kout,
     uint32_t* __restrict__ vout, int64_t n, int shift, const uint32_t* __restrict__ hist,
     uint32_t* __restrict__ status, uint32_t* __restrict__ tile_ctr) {

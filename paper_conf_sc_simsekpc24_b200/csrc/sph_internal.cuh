@@ -25,7 +25,7 @@ constexpr int kSortThreads = 256;
 #define SPH_SORT_KPT 8  // keys per thread (A/B builds)
 #endif
 constexpr int kSortKPT = SPH_SORT_KPT;
-constexpr int kSortTile = kSortThreads * kSortKPT;  // 2048 keys per tile (3 CTAs/SM)
+constexpr int kSortTile = kSortThreads * kSortKPT;  // 2048 keys per tile (4 CTAs/SM, SPH_SORT_MINB)
 constexpr int kRadixBits = 8;
 constexpr int kRadix = 256;
 constexpr int kSortPasses = 8;  // 8 x 8 bits >= 63-bit keys
