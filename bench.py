@@ -573,6 +573,21 @@ def run_decomposed(args, rank, world, local, forced=False):
     ghosts = torch.tensor([ds.stats["n_ghost"], ds.stats["n_local"]], device="cuda", dtype=torch.float64)
     dist.all_reduce(ghosts)
     launches = sph.kernel_launches() - l0
+    # roofline of the dominant kernel on rank 0 (its momentum-energy phase time,
+    # interior + boundary launches, over its own targets' pairs of the last step)
+    roofline = None
+    if rank == 0:
+        import numpy as np
+        nc = ds.sim.get_field("nc")
+        pairs0 = float(np.minimum(nc, ds.sim.cfg.ngmax).sum())
+        mom_s = phase_ms.get("momentum_energy", 0.0) * 1e-3
+        if mom_s > 0 and pairs0 > 0:
+            ach = FLOPS_PER_PAIR["momentum_energy"] * pairs0 / mom_s / 1e12
+            roofline = {"bound": "alu", "achieved": ach, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
+                        "frac": ach / FP64_PEAK_TFLOPS, "traffic": None, "kernel": "momentum_energy_kernel",
+                        "flops_per_pair": FLOPS_PER_PAIR["momentum_energy"], "scope": "rank 0",
+                        "peak_source": "derived: 148 SM x 64 DFMA/clk x 2 x 1.965 GHz",
+                        "frac_of_measured_peak": ach / FP64_PEAK_MEASURED_TFLOPS}
     # e2e: each rank's particles copied in from pinned host memory and back out
     # (into pinned buffers of the rank's capacity: the local count varies) every step
     loc = ds.local
@@ -612,7 +627,7 @@ def run_decomposed(args, rank, world, local, forced=False):
                                            + (" -- forced at N = 1: every collective issued on a one-rank group" if forced else "")),
                            "ghost_fraction": float(ghosts[0] / ghosts[1]),
                            "l2": "inputs >> 126 MB L2; no flush"},
-                "phase_ms_rank0": phase_ms, "roofline": None,
+                "phase_ms_rank0": phase_ms, "roofline": roofline,
                 "e2e": {"value": n_total * max(args.e2e_steps, 1) / (float(ems.item()) * 1e-3), "unit": UNIT,
                         "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": d2h * world,
                         "path": "rank-local state from pinned host -> DistributedSim.step -> host"},
