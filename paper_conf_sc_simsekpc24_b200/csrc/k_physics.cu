@@ -26,6 +26,26 @@ namespace sph {
 #endif
 
 
+// Neighbour-list index loads (A/B builds, SPH_IDX_POLICY): 0 = ld.global.nc;
+// 1 = L1::no_allocate (each list line is used once, by the whole warp at once:
+// keep L1 for the gathered records); 2 = L1::evict_first.
+#ifndef SPH_IDX_POLICY
+#define SPH_IDX_POLICY 1
+#endif
+__device__ __forceinline__ int ldg_idx(const int32_t* p) {
+#if SPH_IDX_POLICY == 1
+  int v;
+  asm("ld.global.nc.L1::no_allocate.b32 %0, [%1];" : "=r"(v) : "l"(p));
+  return v;
+#elif SPH_IDX_POLICY == 2
+  int v;
+  asm("ld.global.nc.L1::evict_first.b32 %0, [%1];" : "=r"(v) : "l"(p));
+  return v;
+#else
+  return __ldg(p);
+#endif
+}
+
 constexpr double kPi = 3.14159265358979323846;
 constexpr double kPi2Over4 = kPi * kPi / 4.0;
 constexpr double kPi2 = kPi * kPi;
@@ -114,15 +134,15 @@ __device__ __forceinline__ void density_body(const Fields& F, const Params& P, c
   // two neighbours per iteration (two independent sinc chains in flight; the sum
   // is still accumulated in list order), records one pair ahead, indices two
   const int64_t cap = F.cap;
-  Rec4 ra = ldg4(rec + (nci > 0 ? __ldg(nb) : 0)), rb = ldg4(rec + (nci > 1 ? __ldg(nb + cap) : 0));
-  int jc = nci > 2 ? __ldg(nb + 2 * cap) : 0, jd = nci > 3 ? __ldg(nb + 3 * cap) : 0;
+  Rec4 ra = ldg4(rec + (nci > 0 ? ldg_idx(nb) : 0)), rb = ldg4(rec + (nci > 1 ? ldg_idx(nb + cap) : 0));
+  int jc = nci > 2 ? ldg_idx(nb + 2 * cap) : 0, jd = nci > 3 ? ldg_idx(nb + 3 * cap) : 0;
   int k = 0;
   for (; k + 1 < nci; k += 2) {
     const Rec4 a = ra, b = rb;
     if (k + 2 < nci) ra = ldg4(rec + jc);
     if (k + 3 < nci) rb = ldg4(rec + jd);
-    if (k + 4 < nci) jc = __ldg(nb + (int64_t)(k + 4) * cap);
-    if (k + 5 < nci) jd = __ldg(nb + (int64_t)(k + 5) * cap);
+    if (k + 4 < nci) jc = ldg_idx(nb + (int64_t)(k + 4) * cap);
+    if (k + 5 < nci) jd = ldg_idx(nb + (int64_t)(k + 5) * cap);
     double dxa, dya, dza, dxb, dyb, dzb;
     pair_d<kWrap>(g, me.a, me.b, me.c, a.a, a.b, a.c, dxa, dya, dza);
     pair_d<kWrap>(g, me.a, me.b, me.c, b.a, b.b, b.c, dxb, dyb, dzb);
@@ -241,15 +261,15 @@ __device__ __forceinline__ void gradh_body(const Fields& F, const Params& P, con
     sum = fma(rj.d * S5, fma(6.0, cos_t(t), -3.0 * S), sum);
     if (kVE) sw = fma(rj.d, S5 * S, sw);
   };
-  Rec4 ra = ldg4(rec + (nci > 0 ? __ldg(nb) : 0)), rb = ldg4(rec + (nci > 1 ? __ldg(nb + cap) : 0));
-  int jc = nci > 2 ? __ldg(nb + 2 * cap) : 0, jd = nci > 3 ? __ldg(nb + 3 * cap) : 0;
+  Rec4 ra = ldg4(rec + (nci > 0 ? ldg_idx(nb) : 0)), rb = ldg4(rec + (nci > 1 ? ldg_idx(nb + cap) : 0));
+  int jc = nci > 2 ? ldg_idx(nb + 2 * cap) : 0, jd = nci > 3 ? ldg_idx(nb + 3 * cap) : 0;
   int k = 0;
   for (; k + 1 < nci; k += 2) {
     const Rec4 a = ra, b = rb;
     if (k + 2 < nci) ra = ldg4(rec + jc);
     if (k + 3 < nci) rb = ldg4(rec + jd);
-    if (k + 4 < nci) jc = __ldg(nb + (int64_t)(k + 4) * cap);
-    if (k + 5 < nci) jd = __ldg(nb + (int64_t)(k + 5) * cap);
+    if (k + 4 < nci) jc = ldg_idx(nb + (int64_t)(k + 4) * cap);
+    if (k + 5 < nci) jd = ldg_idx(nb + (int64_t)(k + 5) * cap);
     double dxa, dya, dza, dxb, dyb, dzb;
     pair_d<kWrap>(g, me.a, me.b, me.c, a.a, a.b, a.c, dxa, dya, dza);
     pair_d<kWrap>(g, me.a, me.b, me.c, b.a, b.b, b.c, dxb, dyb, dzb);
@@ -334,15 +354,15 @@ __device__ __forceinline__ void iad_body(const Fields& F, const Geom& g, int64_t
     t23 = fma(ay, dz, t23);
     t33 = fma(az, dz, t33);
   };
-  Rec4 ra = ldg4(rec + (nci > 0 ? __ldg(nb) : 0)), rb = ldg4(rec + (nci > 1 ? __ldg(nb + cap) : 0));
-  int jc = nci > 2 ? __ldg(nb + 2 * cap) : 0, jd = nci > 3 ? __ldg(nb + 3 * cap) : 0;
+  Rec4 ra = ldg4(rec + (nci > 0 ? ldg_idx(nb) : 0)), rb = ldg4(rec + (nci > 1 ? ldg_idx(nb + cap) : 0));
+  int jc = nci > 2 ? ldg_idx(nb + 2 * cap) : 0, jd = nci > 3 ? ldg_idx(nb + 3 * cap) : 0;
   int k = 0;
   for (; k + 1 < nci; k += 2) {
     const Rec4 a = ra, b = rb;
     if (k + 2 < nci) ra = ldg4(rec + jc);
     if (k + 3 < nci) rb = ldg4(rec + jd);
-    if (k + 4 < nci) jc = __ldg(nb + (int64_t)(k + 4) * cap);
-    if (k + 5 < nci) jd = __ldg(nb + (int64_t)(k + 5) * cap);
+    if (k + 4 < nci) jc = ldg_idx(nb + (int64_t)(k + 4) * cap);
+    if (k + 5 < nci) jd = ldg_idx(nb + (int64_t)(k + 5) * cap);
     add(a);
     add(b);
   }
@@ -409,9 +429,9 @@ __device__ __forceinline__ void iad_dc_body(const Fields& F, const Params& P, co
   };
   // two neighbours per iteration (as iad_body), records one pair ahead,
   // indices two ahead; the sums still run in list order
-  int j0 = nci > 0 ? __ldg(nb) : 0, j1 = nci > 1 ? __ldg(nb + cap) : 0;
+  int j0 = nci > 0 ? ldg_idx(nb) : 0, j1 = nci > 1 ? ldg_idx(nb + cap) : 0;
   Rec4 ra = ldg4(rec + j0), va = ldg4(rv + j0), rb = ldg4(rec + j1), vb = ldg4(rv + j1);
-  int jc = nci > 2 ? __ldg(nb + 2 * cap) : 0, jd = nci > 3 ? __ldg(nb + 3 * cap) : 0;
+  int jc = nci > 2 ? ldg_idx(nb + 2 * cap) : 0, jd = nci > 3 ? ldg_idx(nb + 3 * cap) : 0;
   int k = 0;
   for (; k + 1 < nci; k += 2) {
     const Rec4 a = ra, av = va, b = rb, bv = vb;
@@ -423,8 +443,8 @@ __device__ __forceinline__ void iad_dc_body(const Fields& F, const Params& P, co
       rb = ldg4(rec + jd);
       vb = ldg4(rv + jd);
     }
-    if (k + 4 < nci) jc = __ldg(nb + (int64_t)(k + 4) * cap);
-    if (k + 5 < nci) jd = __ldg(nb + (int64_t)(k + 5) * cap);
+    if (k + 4 < nci) jc = ldg_idx(nb + (int64_t)(k + 4) * cap);
+    if (k + 5 < nci) jd = ldg_idx(nb + (int64_t)(k + 5) * cap);
     add(a, av);
     add(b, bv);
   }
@@ -534,9 +554,9 @@ __device__ __forceinline__ double momentum_body(const Fields& F, const Params& P
   // first) two ahead; the other chunks are loaded at the top of the iteration
   // and arrive while the two sinc polynomials run.
   const int64_t cap = F.cap;
-  const Rec4* r0 = rec + (int64_t)kRecM * (nci > 0 ? __ldg(nb) : 0);
-  const Rec4* r1 = rec + (int64_t)kRecM * (nci > 1 ? __ldg(nb + cap) : 0);
-  int jn = nci > 2 ? __ldg(nb + 2 * cap) : 0;
+  const Rec4* r0 = rec + (int64_t)kRecM * (nci > 0 ? ldg_idx(nb) : 0);
+  const Rec4* r1 = rec + (int64_t)kRecM * (nci > 1 ? ldg_idx(nb + cap) : 0);
+  int jn = nci > 2 ? ldg_idx(nb + 2 * cap) : 0;
   Rec4 p0 = ldg4(r0), p1 = ldg4(r1);
   for (int k = 0; k < nci; ++k) {
     const Rec4* rcur = r0;
@@ -552,7 +572,7 @@ __device__ __forceinline__ double momentum_body(const Fields& F, const Params& P
 #endif
       p1 = ldg4(r1);
     }
-    if (k + 3 < nci) jn = __ldg(nb + (int64_t)(k + 3) * cap);
+    if (k + 3 < nci) jn = ldg_idx(nb + (int64_t)(k + 3) * cap);
 #if SPH_MOM_DIAG == 1
     // diagnostic: the gathers alone (every load, no pair arithmetic)
     ax += j0.a + j1.a + j2.b + j3.c;
