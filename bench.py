@@ -217,7 +217,16 @@ class ClockSampler:
             import threading
             import pynvml as N
             N.nvmlInit()
-            h = N.nvmlDeviceGetHandleByIndex(self.gpu)
+            h = None
+            try:  # the CUDA device's own board (CUDA and NVML may enumerate differently)
+                import torch
+                pr = torch.cuda.get_device_properties(self.gpu)
+                bus = f"{pr.pci_domain_id:08x}:{pr.pci_bus_id:02x}:{pr.pci_device_id:02x}.0"
+                h = N.nvmlDeviceGetHandleByPciBusId(bus)
+            except Exception:
+                h = None
+            if h is None:
+                h = N.nvmlDeviceGetHandleByIndex(self.gpu)
             self.th = threading.Thread(target=self._nvml_loop, args=(N, h), daemon=True)
             self.th.start()
         except Exception:
