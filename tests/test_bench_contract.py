@@ -51,3 +51,19 @@ def test_libsph_arm_line():
     assert d["roofline"]["flops_per_pair"] == 171
     assert d["parity"]["order_exact"] and d["parity"]["nbr_exact"] and d["parity"]["pass"], d["parity"]
     assert d["e2e"]["sequential"]["value"] > 0
+
+
+@pytest.mark.gpu
+def test_decomposed_arm_line():
+    """The N > 1 path of bench.py (SFC decomposition, halos, dt all-reduce) on one
+    GPU: a one-rank NCCL group with every collective issued (--force-decomp)."""
+    d = _run(["--force-decomp", "--workload", "turbulence40", "--steps", "3", "--warmup", "3", "--e2e-steps", "1"])
+    for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better",
+              "scaling", "dtype", "config", "roofline", "e2e", "clocks", "gpu_launches"):
+        assert k in d, k
+    assert d["scaling"] == "weak" and d["dtype"] == "f64" and d["value"] > 0
+    assert "NCCL" in d["config"]["parallelism"] and d["config"]["n_particles_total"] == 40 ** 3
+    r = d["roofline"]
+    assert r["bound"] == "alu" and r["scope"] == "rank 0" and 0 < r["frac"] < 1
+    assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["value"] > 0
+    assert d["gpu_launches"] > 0
